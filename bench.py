@@ -1,0 +1,345 @@
+#!/usr/bin/env python
+"""bench.py -- WY-based SBR on B200: the BASELINE.json headline metric.
+
+Metric (BASELINE.json): SBR seconds and effective TFLOP/s = (4/3) n^3 / seconds at
+n=32768, b=32 (config 4: random symmetric, nb=1024, FP16-in/FP32-acc mode), as a
+fraction of B200 tensor peak.  A "step" is one full sbr_reduce (all of SURVEY
+§8(a): panels, lazy updates, W merges, passes, trailing SYR2Ks, band extraction)
+over one synthetic n x n input resident in HBM.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+One process per GPU (torchrun for N>1).  The reduction of one matrix does not
+shard in this round: N>1 runs N independent replicas
+(weak scaling, no data-path collective), each rank timing its own steps; the
+max over ranks is reported.  ``--impl reference`` times the CPU oracle (this tier
+has no reference implementation; the oracle is the reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CONFIG4 = {"n": 32768, "b": 32, "nb": 1024, "mode": "fp16", "kind": "random_symmetric"}
+METRIC = "SBR seconds & effective TFLOPS ((4/3)n³) at n=32768,b=32 vs B200 tensor peak"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=5)
+    p.add_argument("--warmup", type=int, default=3)
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--n", type=int, default=CONFIG4["n"])
+    p.add_argument("--b", type=int, default=CONFIG4["b"])
+    p.add_argument("--nb", type=int, default=CONFIG4["nb"])
+    p.add_argument("--mode", default=CONFIG4["mode"])
+    p.add_argument("--e2e-steps", type=int, default=2)
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--cpu-sample-s", type=float, default=15.0)
+    return p.parse_args()
+
+
+def eff_tflops(n: int, seconds: float) -> float:
+    return (4.0 / 3.0) * n ** 3 / seconds / 1e12
+
+
+def load_peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+class ClockSampler:
+    """Samples SM clock and throttle reasons via NVML while the timed region runs."""
+
+    def __init__(self, index: int):
+        self.index = index
+        self.samples = []
+        self.reasons = set()
+        self.sm_max = None
+        self._stop = threading.Event()
+        self._t = None
+
+    def __enter__(self):
+        try:
+            import pynvml as nv
+
+            nv.nvmlInit()
+            self._nv = nv
+            self._h = nv.nvmlDeviceGetHandleByIndex(self.index)
+            self.sm_max = nv.nvmlDeviceGetMaxClockInfo(self._h, nv.NVML_CLOCK_SM)
+            self._t = threading.Thread(target=self._run, daemon=True)
+            self._t.start()
+        except Exception as e:  # pragma: no cover
+            self._err = str(e)
+        return self
+
+    def _run(self):
+        nv = self._nv
+        names = {
+            "gpu_idle": getattr(nv, "nvmlClocksEventReasonGpuIdle", 0x1),
+            "sw_power_cap": getattr(nv, "nvmlClocksEventReasonSwPowerCap", 0x4),
+            "hw_slowdown": getattr(nv, "nvmlClocksEventReasonHwSlowdown", 0x8),
+            "sw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonSwThermalSlowdown", 0x20),
+            "hw_thermal_slowdown": getattr(nv, "nvmlClocksEventReasonHwThermalSlowdown", 0x40),
+            "hw_power_brake_slowdown": getattr(nv, "nvmlClocksEventReasonHwPowerBrakeSlowdown", 0x80),
+        }
+        while not self._stop.is_set():
+            try:
+                self.samples.append(nv.nvmlDeviceGetClockInfo(self._h, nv.NVML_CLOCK_SM))
+                r = nv.nvmlDeviceGetCurrentClocksEventReasons(self._h)
+                for k, bit in names.items():
+                    if r & bit and k != "gpu_idle":
+                        self.reasons.add(k)
+            except Exception:
+                pass
+            self._stop.wait(0.1)
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self._t:
+            self._t.join()
+
+    def summary(self):
+        med = statistics.median(self.samples) if self.samples else None
+        return {"sm_mhz": med, "sm_max_mhz": self.sm_max, "reasons": sorted(self.reasons),
+                "samples": len(self.samples)}
+
+
+def cpu_oracle_sample(n: int, b: int, a_host, budget_s: float):
+    """Time the CPU oracle (oracle.sbr.sbr_unblocked, fp64, as it stands) on a prefix of
+    the same n x n reduction and extrapolate by per-column cost (n-c-b)."""
+    import numpy as np
+
+    from oracle import sbr as osbr
+
+    ncol_total = max(0, n - b - 1)
+    # first call: 2 columns to estimate the per-column cost, then size the sample
+    cols = 2
+    t0 = time.perf_counter()
+    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=cols)
+    t1 = time.perf_counter() - t0
+    per = t1 / cols
+    cols = int(max(2, min(ncol_total, budget_s / max(per, 1e-9))))
+    t0 = time.perf_counter()
+    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=cols)
+    ts = time.perf_counter() - t0
+    c = np.arange(ncol_total, dtype=np.float64)
+    w = (n - c - b)
+    frac = float(w[:cols].sum() / w.sum())
+    t_full = ts / frac
+    cores = len(os.sched_getaffinity(0))
+    try:
+        from threadpoolctl import threadpool_info
+
+        thr = max((i.get("num_threads", 1) for i in threadpool_info()), default=cores)
+    except Exception:
+        thr = cores
+    return {
+        "value": eff_tflops(n, t_full),
+        "unit": "TFLOP/s",
+        "cores": int(thr),
+        "kind": "oracle",
+        "sample": f"oracle.sbr.sbr_unblocked (fp64 numpy, as it stands) on the first {cols} of {ncol_total} "
+                  f"columns of the same n={n} b={b} input ({ts:.1f} s, incl. the fp64 copy), extrapolated "
+                  f"by per-column cost (n-c-b): full run ~{t_full:.0f} s",
+        "seconds_extrapolated": t_full,
+    }
+
+
+def dist_setup():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+
+        dist.init_process_group("nccl" if os.environ.get("SBR_BENCH_GLOO") is None else "gloo")
+    return rank, world, local
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle, as it stands, on bounded samples of config 4."""
+    if rank != 0:
+        return
+    import workloads
+
+    n, b = args.n, args.b
+    a_host = workloads.random_symmetric(n, workloads.config_seed(4))
+    vals = []
+    samples = []
+    for i in range(args.warmup + args.steps):
+        r = cpu_oracle_sample(n, b, a_host, budget_s=max(2.0, min(args.cpu_sample_s, 150.0 / max(1, args.steps))))
+        if i >= args.warmup:
+            vals.append(r["value"])
+            samples.append(r)
+    v = statistics.median(vals)
+    last = samples[-1]
+    line = {
+        "impl": "reference",
+        "metric": METRIC, "value": v, "unit": "TFLOP/s", "n_gpus": args.gpus, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": (4.0 / 3.0) * n ** 3 / (v * 1e12) * 1e3,
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": f"config4: n={n} random symmetric, b={b}, nb={args.nb} (oracle is unblocked)",
+                   "n": n, "b": b, "nb": args.nb, "parallelism": "cpu"},
+        "cpu_baseline": {k: last[k] for k in ("kind", "cores", "sample")} | {"value": v, "unit": "TFLOP/s"},
+        "e2e": {"value": v, "unit": "TFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_setup()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import numpy as np
+    import torch
+
+    torch.cuda.set_device(local)
+    import __graft_entry__
+
+    __graft_entry__.build()
+    import paper_conf_ppopp_zhangsoyw23_b200 as sbr
+    import workloads
+
+    n, b, nb, mode = args.n, args.b, args.nb, args.mode
+    seed = workloads.config_seed(4)
+    stream = torch.cuda.current_stream()
+    h = sbr.Handle(local, stream)
+    pristine = h.generate_symmetric(seed, n)              # device twin of workloads.random_symmetric
+    a = torch.empty_like(pristine)
+    ab = torch.empty((n, b + 1), dtype=torch.float32, device=a.device)
+    w = torch.empty((n - b, n), dtype=torch.float32, device=a.device)
+    # warm-up (untimed)
+    for _ in range(args.warmup):
+        a.copy_(pristine)
+        h.reduce(a, b, nb, mode=mode, ab=ab, w=w)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    # timed region: K steps, each bracketed by CUDA events on the launching stream; the
+    # input is restored from the pristine copy between steps, outside the events
+    h.reset_kernel_stats()
+    h.set_kernel_timing(True)
+    launches0 = h.launch_count()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for i in range(args.steps):
+            a.copy_(pristine)
+            evs[i][0].record(stream)
+            h.reduce(a, b, nb, mode=mode, ab=ab, w=w)
+            evs[i][1].record(stream)
+        torch.cuda.synchronize()
+    h.set_kernel_timing(False)
+    launches = h.launch_count() - launches0
+    step_ms = [e0.elapsed_time(e1) for e0, e1 in evs]
+    total_ms = sum(step_ms)
+    if world > 1:
+        t = torch.tensor([total_ms], device=a.device)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        torch.distributed.barrier()
+        total_ms = float(t.item())
+    ms_per_step = total_ms / args.steps
+    value = world * eff_tflops(n, ms_per_step / 1e3)
+
+    # per-kernel-class stats (events around every launch inside the timed region)
+    classes = ["panel", "lazy", "wmerge", "pass", "syr2k", "other"]
+    kst = {c: h.kernel_stats(c) for c in classes}
+    dom = max(["pass", "syr2k", "panel", "lazy", "wmerge"], key=lambda c: kst[c]["ms"])
+    peaks, src = load_peaks()
+    st = kst[dom]
+    avg_ms = st["ms"] / max(1, st["launches"])
+    if dom == "syr2k":
+        achieved = st["flops"] / max(1, st["launches"]) / (avg_ms / 1e3) / 1e12
+        peak = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
+        roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                "frac": achieved / peak, "traffic": None}
+    else:
+        achieved = st["bytes"] / max(1, st["launches"]) / (avg_ms / 1e3) / 1e9
+        peak = peaks["hbm_gbs"]
+        roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                "traffic": None}
+    roof.update({"kernel": dom, "peak_source": src, "launches": st["launches"], "avg_ms": avg_ms,
+                 "share_of_step": st["ms"] / total_ms if total_ms else None})
+    breakdown = {c: {"ms_per_step": kst[c]["ms"] / args.steps, "launches_per_step": kst[c]["launches"] / args.steps}
+                 for c in classes}
+
+    # end-to-end through the public API with HOST buffers (H2D of A + D2H of the band per step)
+    e2e = None
+    if args.e2e_steps > 0:
+        a_host = torch.empty((n, n), dtype=torch.float32, pin_memory=True)
+        a_host.copy_(pristine.cpu())   # same input bits (device generator == workloads generator)
+        ab_host = torch.empty((n, b + 1), dtype=torch.float32, pin_memory=True)
+        h.reduce_host(a_host, b, nb, mode=mode, ab=ab_host)   # warm-up of the device copies
+        e2e_ms = []
+        for _ in range(args.e2e_steps):
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            h.reduce_host(a_host, b, nb, mode=mode, ab=ab_host)
+            e2e_ms.append((time.perf_counter() - t0) * 1e3)
+        e2e_t = max(e2e_ms) if world == 1 else max(e2e_ms)
+        e2e = {"value": world * eff_tflops(n, statistics.median(e2e_ms) / 1e3), "unit": "TFLOP/s",
+               "h2d_bytes_per_step": 4 * n * n, "d2h_bytes_per_step": 4 * n * (b + 1),
+               "ms_per_step": statistics.median(e2e_ms), "steps": args.e2e_steps,
+               "note": "sbr_reduce_host: pinned host A -> device, reduce, band -> host (the paper's EVD "
+                       "pipeline moves only the band, P:415)"}
+        del a_host
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        a_np = workloads.random_symmetric(n, seed)
+        cpu = cpu_oracle_sample(n, b, a_np, args.cpu_sample_s)
+        cpu.pop("seconds_extrapolated", None)
+        del a_np
+
+    if rank == 0:
+        line = {
+            "metric": METRIC,
+            "value": value,
+            "unit": "TFLOP/s",
+            "n_gpus": world,
+            "steps": args.steps,
+            "warmup": args.warmup,
+            "ms_per_step": ms_per_step,
+            "seconds_per_step": ms_per_step / 1e3,
+            "higher_is_better": True,
+            "scaling": "weak",
+            "vs_baseline": None,
+            "dtype": "f32" if mode == "3xtf32" else "f16",
+            "data": "synthetic",
+            "config": {"workload": f"config4: n={n} random symmetric U[-1,1) (seed {seed}), b={b}, nb={nb}, "
+                                   f"{'FP16-in/FP32-acc' if mode == 'fp16' else '3xTF32'}",
+                       "n": n, "b": b, "nb": nb, "mode": mode,
+                       "parallelism": "replicas" if world > 1 else "single",
+                       "l2": f"inputs {4 * n * n / 2**30:.1f} GiB >> 126 MB L2 (no flush needed)"},
+            "frac_of_peak": {"fp16_spec_2250": value / world / 2250.0,
+                             "fp16_measured": value / world / peaks.get("bf16_tflops", 1642.5)},
+            "roofline": roof,
+            "breakdown": breakdown,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+            "step_ms": step_ms,
+        }
+        print(json.dumps(line), flush=True)
+    h.close()
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

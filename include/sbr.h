@@ -1,0 +1,160 @@
+/*
+ * sbr.h -- C ABI of libsbr: stage-one successive band reduction (SBR) of a dense
+ * symmetric matrix to band form with the WY formulation, on NVIDIA B200 (sm_100a).
+ *
+ * Method: Zhang, Shah, Ootomo, Yokota, Wu, "Fast Symmetric Eigenvalue
+ * Decomposition via WY Representation on Tensor Core", PPoPP'23.  "P:n" below is
+ * line n of the paper text (/root/reference/PAPER.md at authoring time).
+ *
+ *   A = Q B Q^T,  Q = H_1 H_2 ... H_{n-b},  B symmetric with bandwidth b
+ *   (Sec. 3.1; reading C2 of DESIGN.md for the product order).
+ *
+ * The reduction is Algorithm 1: b-wide panels are factored by a
+ * tall-skinny QR (TSQR) whose explicit Q is turned back into
+ * Householder vectors (Alg. 3 + sign matrix S); inside an nb-wide
+ * block every panel is updated lazily from the block's original trailing matrix
+ * OA and the accumulated (W, Y); the trailing matrix is
+ * updated once per block, A <- (I - W Y^T)^T A (I - W Y^T) (Eq. 1),
+ * evaluated as the lower-triangular rank-2nb update A - Y Z^T - Z Y^T with
+ * Z = X - 1/2 Y (W^T X), X = OA W (Eq. 2-3; reading C5).
+ *
+ * Conventions (all arrays column-major, 64-bit leading dimensions, fp32):
+ *   - Householder convention: LAPACK dlarfg (reading C1).  Entry for entry the
+ *     result equals LAPACK dsytrd_sy2sb(UPLO='L') up to rounding, except that a
+ *     panel whose column needs no reduction may yield H = I - 2 e e^T instead of
+ *     H = I (B -> D B D with D = diag(+-1)).
+ *   - Only the lower triangle of A is referenced (reading C14).
+ *
+ * Threading / streams: a handle is bound to one device and one CUDA stream; all
+ * calls on it are stream-ordered and return after enqueueing device work (no
+ * host synchronisation) unless stated.  A handle must not be used by two host
+ * threads at once.  Device pointers are plain CUDA device addresses.
+ *
+ * Errors: 0 = OK; -i = argument i invalid (LAPACK style); positive values:
+ */
+#ifndef SBR_H_
+#define SBR_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SBR_OK 0
+#define SBR_ERR_NONFINITE 1  /* input holds Inf/NaN (detected before any update)   */
+#define SBR_ERR_CUDA 2       /* CUDA runtime/driver error; see sbr_status_string    */
+#define SBR_ERR_NCCL 3       /* reserved for the multi-GPU path                     */
+#define SBR_ERR_NOMEM 4      /* device workspace allocation failed                  */
+#define SBR_ERR_UNSUPPORTED 5 /* valid arguments this build does not support        */
+
+typedef struct sbr_ctx* sbr_handle_t;
+
+/* Arithmetic of the GEMM-shaped steps (Sec. 5.3).  The panel QR,
+ * reconstruction and all accumulations are fp32 in every mode.
+ *   SBR_FP16_FP32ACC : operands rounded to fp16 (RN), fp32 accumulate on tcgen05
+ *                      (kind::f16) -- the paper's Tensor Core mode.
+ *   SBR_3XTF32       : FP32-accurate "EC-TCGEMM" mode (reading C11):
+ *                      a = hi + lo with hi = rna_tf32(a), lo = rna_tf32(a - hi);
+ *                      C = hi*hi' + (hi*lo' + lo*hi'). */
+typedef enum { SBR_FP16_FP32ACC = 0, SBR_3XTF32 = 1 } sbr_precision_t;
+
+/* Create a handle on CUDA device `device`, bound to `stream` (a cudaStream_t;
+ * NULL = the legacy default stream).  Allocates nothing large.
+ * Returns SBR_OK, -1 (h NULL), -2 (bad device) or SBR_ERR_CUDA. */
+int sbr_create(sbr_handle_t* h, int device, void* stream);
+
+/* Rebind the handle to another stream on the same device. */
+int sbr_set_stream(sbr_handle_t h, void* stream);
+
+/* Free the handle and its workspace (synchronises the handle's stream). */
+int sbr_destroy(sbr_handle_t h);
+
+/* Device workspace sbr_reduce needs for (n, b, nb, mode), in bytes.  The handle
+ * allocates and owns it (grown on demand, kept between calls). */
+int sbr_workspace_query(sbr_handle_t h, int64_t n, int b, int nb, int mode, size_t* bytes);
+
+/* Reduce the symmetric n x n matrix A (device, fp32, lower triangle referenced)
+ * to bandwidth b with outer block nb (Alg. 1).
+ *   mode  : sbr_precision_t.
+ *   n     : order, n >= 1.                                   (arg 3)
+ *   b     : bandwidth, 1 <= b <= 64.                          (arg 4)
+ *   nb    : outer block, nb >= b, nb % b == 0, nb <= 4096.    (arg 5)
+ *   A     : in: symmetric matrix (lower).  out: LAPACK dsytrd_sy2sb layout --
+ *           the band (diagonal blocks and the upper-triangular R factors) in the
+ *           lower band, and the Householder vector of reflector column c
+ *           (0 <= c < n-b; unit at row c+b, implicit) in A[c+b+1:n, c].
+ *           Entries above the diagonal are left unspecified.           (arg 6)
+ *   lda   : >= max(1, n).                                     (arg 7)
+ *   AB    : out: band in LAPACK lower band storage, AB[d + j*ldab] = B[j+d, j],
+ *           0 <= d <= b; may alias nothing else.             (arg 8)
+ *   ldab  : >= b + 1.                                         (arg 9)
+ *   W     : out (may be NULL): per-block W factors: for block J
+ *           (columns c0 = J*nb .. c0+k_J-1), Q_J = I - W_J Y_J^T acting on
+ *           rows/cols c0+b .. n-1, W_J stored in W[c0+b : n, c0 : c0+k_J];
+ *           Q = Q_0 Q_1 ... .  Other entries are not referenced.  n x (n-b).
+ *           If NULL, W lives in handle workspace (per block) and is dropped. (arg 10)
+ *   ldw   : >= n if W != NULL.                                (arg 11)
+ * Trivial case n <= b+1: AB = band of A, W untouched, no reflectors.
+ * Returns 0, -i, SBR_ERR_NONFINITE, SBR_ERR_CUDA, SBR_ERR_NOMEM.  Synchronises
+ * the stream once at the start (4-byte read of the input's finiteness flag). */
+int sbr_reduce(sbr_handle_t h, int mode, int64_t n, int b, int nb,
+               float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw);
+
+/* End-to-end variant with HOST buffers (pinned or pageable): copies A to the
+ * device, reduces, copies the band AB back and, as selected by `outputs`
+ * (bitmask of SBR_OUT_*), A (holding Y) and W; all on the handle's stream,
+ * returning after the results are on the host.  The band alone is what the
+ * paper's eigenvalue pipeline moves to the host.  Same arguments and
+ * errors as sbr_reduce (outputs is argument 12).  Device copies are owned by the
+ * handle (grown on demand). */
+#define SBR_OUT_BAND 1
+#define SBR_OUT_Y 2
+#define SBR_OUT_W 4
+int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb,
+                    float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw,
+                    int outputs);
+
+/* Wait for all work enqueued on the handle's stream. */
+int sbr_sync(sbr_handle_t h);
+
+/* Human-readable text for a status code (static storage; includes the last
+ * CUDA error seen by any handle when status == SBR_ERR_CUDA). */
+const char* sbr_status_string(int status);
+
+/* Seeded input generator, bit-identical to workloads.random_symmetric (host):
+ * A[i + j*lda] = U[-1,1) from splitmix64(seed ^ (max(i,j) << 32 | min(i,j))),
+ * top 24 bits u -> (u - 2^23) * 2^-23.  Full (both triangles) n x n.  Not part
+ * of the method; used to create large inputs without a host copy. */
+int sbr_generate_symmetric(sbr_handle_t h, uint64_t seed, int64_t n, float* A, int64_t lda);
+
+/* Per-kernel timing for roofline reporting.  When enabled, sbr_reduce records a
+ * CUDA event pair (on the handle's stream) around every launch of each kernel
+ * class; sbr_kernel_stats returns, for class `kid` (see SBR_K_*), the number of
+ * launches, their summed device time (ms, elapsed between each pair) and the
+ * summed algorithmic bytes and flops since the last
+ * reset.  sbr_kernel_stats synchronises the stream. */
+#define SBR_K_PANEL 0   /* TSQR + reconstruction (a1, a2)          */
+#define SBR_K_LAZY 1    /* lazy next-panel update (a5)             */
+#define SBR_K_WMERGE 2  /* W merge + W^T X (a3)                    */
+#define SBR_K_PASS 3    /* X_t = OA W_t (a4)                       */
+#define SBR_K_SYR2K 4   /* trailing update (a6, with Z formation)  */
+#define SBR_K_OTHER 5   /* setup, band extraction                  */
+#define SBR_K_COUNT 6
+int sbr_set_kernel_timing(sbr_handle_t h, int enable);
+int sbr_reset_kernel_stats(sbr_handle_t h);
+int sbr_kernel_stats(sbr_handle_t h, int kid, int64_t* launches, double* ms,
+                     double* bytes, double* flops);
+
+/* Number of kernels libsbr launched since the handle was created (a counter
+ * incremented on every launch, including those replayed from graphs). */
+int64_t sbr_launch_count(sbr_handle_t h);
+
+/* Build identification, e.g. "libsbr 0.1 sm_100a". */
+const char* sbr_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SBR_H_ */

@@ -1,0 +1,115 @@
+// k_misc.cu -- small kernels: input generator, finiteness check, band extraction,
+// symmetric mirrors, the k x b correction of the lazy panel update.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace sbr {
+
+SBR_DEV uint64_t splitmix64(uint64_t x) {
+  uint64_t z = x + 0x9E3779B97F4A7C15ull;
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+__global__ void gen_symmetric_kernel(uint64_t seed, int64_t n, int64_t j0, float* A, int64_t lda) {
+  const int64_t j = j0 + blockIdx.y;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    const uint64_t hi = (uint64_t)(i > j ? i : j), lo = (uint64_t)(i > j ? j : i);
+    const uint64_t h = splitmix64(seed ^ ((hi << 32) | lo));
+    const int64_t u = (int64_t)(h >> 40);
+    A[i + j * lda] = (float)((double)(u - (1ll << 23)) * (1.0 / 8388608.0));
+  }
+}
+
+cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaStream_t st) {
+  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, n - j0);
+    dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 64), (unsigned)nc);
+    gen_symmetric_kernel<<<grid, 256, 0, st>>>(seed, n, j0, A, lda);
+  }
+  return cudaGetLastError();
+}
+
+__global__ void check_finite_kernel(int64_t n, const float* A, int64_t lda, unsigned* flag) {
+  const int64_t j = blockIdx.y;
+  for (int64_t i = j + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    if (!isfinite(A[i + j * lda])) { atomicOr(flag, 1u); return; }
+  }
+}
+
+cudaError_t check_finite(int64_t n, const float* A, int64_t lda, unsigned* flag, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(flag, 0, sizeof(unsigned), st);
+  if (e != cudaSuccess) return e;
+  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, n - j0);
+    dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 16), (unsigned)nc);
+    check_finite_kernel<<<grid, 256, 0, st>>>(n - j0, A + j0 + j0 * lda, lda, flag);
+  }
+  return cudaGetLastError();
+}
+
+__global__ void extract_band_kernel(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab) {
+  const int64_t j = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
+  const int d = threadIdx.x;
+  if (j >= n || d > b) return;
+  AB[d + j * ldab] = (j + d < n) ? A[(j + d) + j * lda] : 0.f;
+}
+
+cudaError_t extract_band(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab, cudaStream_t st) {
+  const int dx = b + 1;
+  const int dy = max(1, 256 / dx);
+  extract_band_kernel<<<(unsigned)((n + dy - 1) / dy), dim3(dx, dy), 0, st>>>(n, b, A, lda, AB, ldab);
+  return cudaGetLastError();
+}
+
+__global__ void mirror_lower_block_kernel(int b, float* A, int64_t lda) {
+  for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
+    const int i = e % b, j = e / b;
+    if (i < j) A[i + (int64_t)j * lda] = A[j + (int64_t)i * lda];
+  }
+}
+
+cudaError_t mirror_lower_block(int b, float* A, int64_t lda, cudaStream_t st) {
+  mirror_lower_block_kernel<<<1, 256, 0, st>>>(b, A, lda);
+  return cudaGetLastError();
+}
+
+// P[q, p] = X(c+p, q) - sum_r WtX[q, r] Y(c+p, r)   (k x b), i.e.
+// W^T R = X(c,:)^T - (W^T X) Y_c^T   (reading C3/C5)
+__global__ void lazy_small_p_kernel(int k, int b, const float* Xc, int64_t ldx, const float* WtX, int64_t ldwx,
+                                    const float* Yc, int64_t ldy, float* P) {
+  const int q = blockIdx.x * blockDim.x + threadIdx.x;
+  const int p = blockIdx.y;
+  if (q >= k) return;
+  float acc = Xc[p + (int64_t)q * ldx];
+  for (int r = 0; r < k; ++r) acc = fmaf(-WtX[q + (int64_t)r * ldwx], Yc[p + (int64_t)r * ldy], acc);
+  P[q + (int64_t)p * k] = acc;
+}
+
+cudaError_t lazy_small_p(int k, int b, const float* Xc, int64_t ldx, const float* WtX, int64_t ldwx,
+                         const float* Yc, int64_t ldy, float* P, cudaStream_t st) {
+  dim3 grid((k + 127) / 128, b);
+  lazy_small_p_kernel<<<grid, 128, 0, st>>>(k, b, Xc, ldx, WtX, ldwx, Yc, ldy, P);
+  return cudaGetLastError();
+}
+
+// WtX[k+p, q] = WtX[q, k+p]  for q < k, p < b
+__global__ void mirror_wtx_kernel(int k, int b, float* WtX, int64_t ld) {
+  const int q = blockIdx.x * blockDim.x + threadIdx.x;
+  const int p = blockIdx.y;
+  if (q < k) WtX[(k + p) + (int64_t)q * ld] = WtX[q + (int64_t)(k + p) * ld];
+}
+
+cudaError_t mirror_wtx(int k, int b, float* WtX, int64_t ld, cudaStream_t st) {
+  if (k <= 0) return cudaSuccess;
+  mirror_wtx_kernel<<<dim3((k + 127) / 128, b), 128, 0, st>>>(k, b, WtX, ld);
+  return cudaGetLastError();
+}
+
+cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaStream_t st) {
+  if (rows <= 0 || cols <= 0) return cudaSuccess;
+  return cudaMemset2DAsync(A, lda * sizeof(float), 0, rows * sizeof(float), cols, st);
+}
+
+}  // namespace sbr

@@ -1,0 +1,271 @@
+// k_simt.cu -- fp32 SIMT building blocks for the skinny WY steps (a3, a5) and the
+// first (pre-tensor-core) versions of the pass (a4) and trailing SYR2K (a6).
+#include "common.cuh"
+#include "kernels.h"
+
+namespace sbr {
+
+// ---------------------------------------------------------------- gemm_tn
+// C[m1 x n2] += alpha * A^T B over `rows` rows; each CTA: 64x64 output tile over a
+// row chunk, atomically accumulated (C zeroed by the caller).
+constexpr int TN_T = 64, TN_KC = 32;
+
+__global__ void __launch_bounds__(256) gemm_tn_kernel(int64_t rows, int64_t chunk, int m1, int n2, float alpha,
+                                                      const float* __restrict__ A, int64_t lda,
+                                                      const float* __restrict__ B, int64_t ldb, float* C,
+                                                      int64_t ldc) {
+  __shared__ float As[TN_KC][TN_T + 1];
+  __shared__ float Bs[TN_KC][TN_T + 1];
+  const int i0 = blockIdx.x * TN_T, j0 = blockIdx.y * TN_T;
+  const int64_t r_beg = (int64_t)blockIdx.z * chunk;
+  const int64_t r_end = min(rows, r_beg + chunk);
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  float acc[4][4] = {};
+  for (int64_t r0 = r_beg; r0 < r_end; r0 += TN_KC) {
+    for (int e = threadIdx.x; e < TN_KC * TN_T; e += 256) {
+      const int rr = e % TN_KC, cc = e / TN_KC;
+      const int64_t r = r0 + rr;
+      const bool ok = r < r_end;
+      As[rr][cc] = (ok && i0 + cc < m1) ? A[r + (int64_t)(i0 + cc) * lda] : 0.f;
+      Bs[rr][cc] = (ok && j0 + cc < n2) ? B[r + (int64_t)(j0 + cc) * ldb] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll 8
+    for (int rr = 0; rr < TN_KC; ++rr) {
+      float a[4], bb[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) { a[u] = As[rr][ty * 4 + u]; bb[u] = Bs[rr][tx * 4 + u]; }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) acc[u][v] = fmaf(a[u], bb[v], acc[u][v]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      const int i = i0 + ty * 4 + u, j = j0 + tx * 4 + v;
+      if (i < m1 && j < n2) atomicAdd(&C[i + (int64_t)j * ldc], alpha * acc[u][v]);
+    }
+}
+
+cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, int64_t lda, const float* B,
+                    int64_t ldb, float* C, int64_t ldc, cudaStream_t st) {
+  if (rows <= 0 || m1 <= 0 || n2 <= 0) return cudaSuccess;
+  const int gx = (m1 + TN_T - 1) / TN_T, gy = (n2 + TN_T - 1) / TN_T;
+  int64_t want = std::max<int64_t>(1, 296 / (gx * gy));
+  int64_t chunk = (rows + want - 1) / want;
+  chunk = std::max<int64_t>(chunk, 256);
+  chunk = (chunk + TN_KC - 1) / TN_KC * TN_KC;
+  const int gz = (int)((rows + chunk - 1) / chunk);
+  gemm_tn_kernel<<<dim3(gx, gy, gz), 256, 0, st>>>(rows, chunk, m1, n2, alpha, A, lda, B, ldb, C, ldc);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------- gemm_nn
+// D = beta*C + alpha*A*op(B); 64x64 tiles, K in chunks of 32; C/D may alias.
+constexpr int NN_T = 64, NN_KC = 32;
+
+__global__ void __launch_bounds__(256) gemm_nn_kernel(int64_t M, int N, int K, float alpha,
+                                                      const float* __restrict__ A, int64_t lda,
+                                                      const float* __restrict__ B, int64_t ldb, bool transB,
+                                                      float beta, const float* C, int64_t ldc, float* D,
+                                                      int64_t ldd) {
+  __shared__ float As[NN_KC][NN_T + 1];
+  __shared__ float Bs[NN_KC][NN_T + 1];
+  const int64_t i0 = (int64_t)blockIdx.x * NN_T;
+  const int j0 = blockIdx.y * NN_T;
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  float acc[4][4] = {};
+  for (int k0 = 0; k0 < K; k0 += NN_KC) {
+    for (int e = threadIdx.x; e < NN_KC * NN_T; e += 256) {
+      {  // A tile: rows i0.., k k0..; coalesce along rows
+        const int ii = e % NN_T, kk = e / NN_T;
+        const int64_t i = i0 + ii;
+        const int k = k0 + kk;
+        As[kk][ii] = (i < M && k < K) ? A[i + (int64_t)k * lda] : 0.f;
+      }
+      if (!transB) {  // B(k, j) at B[k + j ldb]; coalesce along k
+        const int kk = e % NN_KC, jj = e / NN_KC;
+        const int k = k0 + kk, j = j0 + jj;
+        Bs[kk][jj] = (k < K && j < N) ? B[k + (int64_t)j * ldb] : 0.f;
+      } else {        // op(B)(k, j) = B[j + k ldb]; coalesce along j
+        const int jj = e % NN_T, kk = e / NN_T;
+        const int k = k0 + kk, j = j0 + jj;
+        Bs[kk][jj] = (k < K && j < N) ? B[j + (int64_t)k * ldb] : 0.f;
+      }
+    }
+    __syncthreads();
+#pragma unroll 8
+    for (int kk = 0; kk < NN_KC; ++kk) {
+      float a[4], bb[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) { a[u] = As[kk][ty + 16 * u]; bb[u] = Bs[kk][tx * 4 + u]; }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) acc[u][v] = fmaf(a[u], bb[v], acc[u][v]);
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      const int64_t i = i0 + ty + 16 * u;
+      const int j = j0 + tx * 4 + v;
+      if (i < M && j < N) {
+        const float c = (beta != 0.f) ? beta * C[i + (int64_t)j * ldc] : 0.f;
+        D[i + (int64_t)j * ldd] = c + alpha * acc[u][v];
+      }
+    }
+}
+
+cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_t lda, const float* B,
+                    int64_t ldb, bool transB, float beta, const float* C, int64_t ldc, float* D, int64_t ldd,
+                    cudaStream_t st) {
+  if (M <= 0 || N <= 0) return cudaSuccess;
+  dim3 grid((unsigned)((M + NN_T - 1) / NN_T), (N + NN_T - 1) / NN_T);
+  gemm_nn_kernel<<<grid, 256, 0, st>>>(M, N, K, alpha, A, lda, B, ldb, transB, beta, C, ldc, D, ldd);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------- sym_pass (SIMT v1)
+// X = OA * W, OA symmetric (lower storage).  CTA = 64-row block x a range of 64-col
+// tiles; tiles above the diagonal are read transposed from the lower triangle.
+constexpr int SP_T = 64;
+
+template <int BW>
+__global__ void __launch_bounds__(256) sym_pass_kernel(int64_t M, int b, int tiles_per_cta,
+                                                       const float* __restrict__ OA, int64_t ld,
+                                                       const float* __restrict__ S, int64_t lds, int sw,
+                                                       const float* __restrict__ W, int64_t ldw, float* X,
+                                                       int64_t ldx) {
+  __shared__ float Ts[SP_T][SP_T + 1];
+  __shared__ float Ws[SP_T][BW + 1];
+  const int64_t I0 = (int64_t)blockIdx.x * SP_T;
+  const int64_t nt = (M + SP_T - 1) / SP_T;
+  const int64_t jt0 = (int64_t)blockIdx.y * tiles_per_cta;
+  const int64_t jt1 = min(nt, jt0 + tiles_per_cta);
+  constexpr int OPT = SP_T * BW / 256;  // outputs per thread
+  float acc[OPT];
+#pragma unroll
+  for (int u = 0; u < OPT; ++u) acc[u] = 0.f;
+  const int ri = threadIdx.x % SP_T;          // output row within block
+  const int cgrp = threadIdx.x / SP_T;        // 4 column groups
+  for (int64_t jt = jt0; jt < jt1; ++jt) {
+    const int64_t J0 = jt * SP_T;
+    for (int e = threadIdx.x; e < SP_T * SP_T; e += 256) {
+      const int a = e % SP_T, c = e / SP_T;
+      // coalesced index a runs along the stored-contiguous dimension
+      int64_t i, j;
+      if (J0 <= I0) { i = I0 + a; j = J0 + c; }   // lower (or diagonal) tile: rows contiguous
+      else { j = J0 + a; i = I0 + c; }            // upper tile: read (j, i) from lower storage
+      float v = 0.f;
+      if (i < M && j < M) {
+        const int64_t hi = i >= j ? i : j, lo = i >= j ? j : i;
+        v = (lo < sw) ? S[hi + lo * lds] : OA[hi + lo * ld];
+      }
+      if (J0 <= I0) Ts[a][c] = v; else Ts[c][a] = v;
+    }
+    for (int e = threadIdx.x; e < SP_T * BW; e += 256) {
+      const int jj = e % SP_T, c = e / SP_T;
+      const int64_t j = J0 + jj;
+      Ws[jj][c] = (j < M && c < b) ? W[j + c * ldw] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll 4
+    for (int jj = 0; jj < SP_T; ++jj) {
+      const float t = Ts[ri][jj];
+#pragma unroll
+      for (int u = 0; u < OPT; ++u) acc[u] = fmaf(t, Ws[jj][cgrp + 4 * u], acc[u]);
+    }
+    __syncthreads();
+  }
+  const int64_t i = I0 + ri;
+  if (i < M) {
+#pragma unroll
+    for (int u = 0; u < OPT; ++u) {
+      const int c = cgrp + 4 * u;
+      if (c < b) atomicAdd(&X[i + c * ldx], acc[u]);
+    }
+  }
+}
+
+cudaError_t sym_pass(int64_t M, int b, const float* OA, int64_t ldoa, const float* S, int64_t lds, int sw,
+                     const float* W, int64_t ldw, float* X, int64_t ldx, cudaStream_t st) {
+  cudaError_t e = zero_matrix(M, b, X, ldx, st);
+  if (e != cudaSuccess) return e;
+  const int64_t nt = (M + SP_T - 1) / SP_T;
+  const int tpc = 16;
+  dim3 grid((unsigned)nt, (unsigned)((nt + tpc - 1) / tpc));
+  if (b <= 16) sym_pass_kernel<16><<<grid, 256, 0, st>>>(M, b, tpc, OA, ldoa, S, lds, sw, W, ldw, X, ldx);
+  else if (b <= 32) sym_pass_kernel<32><<<grid, 256, 0, st>>>(M, b, tpc, OA, ldoa, S, lds, sw, W, ldw, X, ldx);
+  else sym_pass_kernel<64><<<grid, 256, 0, st>>>(M, b, tpc, OA, ldoa, S, lds, sw, W, ldw, X, ldx);
+  return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------- syr2k_lower (SIMT v1)
+constexpr int SY_T = 64, SY_KC = 16;
+
+__global__ void __launch_bounds__(256) syr2k_lower_kernel(int64_t M, int K, const float* __restrict__ Y,
+                                                          int64_t ldy, const float* __restrict__ Z, int64_t ldz,
+                                                          float* C, int64_t ldc) {
+  __shared__ float Yi[SY_KC][SY_T + 1], Zi[SY_KC][SY_T + 1], Yj[SY_KC][SY_T + 1], Zj[SY_KC][SY_T + 1];
+  // linear lower-tile index -> (I, J), I >= J
+  const int64_t t = blockIdx.x;
+  int64_t I = (int64_t)((sqrt(8.0 * (double)t + 1.0) - 1.0) * 0.5);
+  while (I * (I + 1) / 2 > t) --I;
+  while ((I + 1) * (I + 2) / 2 <= t) ++I;
+  const int64_t J = t - I * (I + 1) / 2;
+  const int64_t i0 = I * SY_T, j0 = J * SY_T;
+  const int tx = threadIdx.x % 16, ty = threadIdx.x / 16;
+  float acc[4][4] = {};
+  for (int k0 = 0; k0 < K; k0 += SY_KC) {
+    for (int e = threadIdx.x; e < SY_KC * SY_T; e += 256) {
+      const int rr = e % SY_T, kk = e / SY_T;
+      const int k = k0 + kk;
+      const int64_t ri = i0 + rr, rj = j0 + rr;
+      const bool okk = k < K;
+      Yi[kk][rr] = (okk && ri < M) ? Y[ri + (int64_t)k * ldy] : 0.f;
+      Zi[kk][rr] = (okk && ri < M) ? Z[ri + (int64_t)k * ldz] : 0.f;
+      Yj[kk][rr] = (okk && rj < M) ? Y[rj + (int64_t)k * ldy] : 0.f;
+      Zj[kk][rr] = (okk && rj < M) ? Z[rj + (int64_t)k * ldz] : 0.f;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int kk = 0; kk < SY_KC; ++kk) {
+      float yi[4], zi[4], yj[4], zj[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        yi[u] = Yi[kk][ty + 16 * u]; zi[u] = Zi[kk][ty + 16 * u];
+        yj[u] = Yj[kk][tx * 4 + u]; zj[u] = Zj[kk][tx * 4 + u];
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) acc[u][v] = fmaf(yi[u], zj[v], fmaf(zi[u], yj[v], acc[u][v]));
+    }
+    __syncthreads();
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 4; ++v) {
+      const int64_t i = i0 + ty + 16 * u, j = j0 + tx * 4 + v;
+      if (i < M && j < M && i >= j) C[i + j * ldc] -= acc[u][v];
+    }
+}
+
+cudaError_t syr2k_lower(int64_t M, int K, const float* Y, int64_t ldy, const float* Z, int64_t ldz, float* C,
+                        int64_t ldc, cudaStream_t st) {
+  if (M <= 0) return cudaSuccess;
+  const int64_t nt = (M + SY_T - 1) / SY_T;
+  const int64_t ntiles = nt * (nt + 1) / 2;
+  syr2k_lower_kernel<<<(unsigned)ntiles, 256, 0, st>>>(M, K, Y, ldy, Z, ldz, C, ldc);
+  return cudaGetLastError();
+}
+
+}  // namespace sbr

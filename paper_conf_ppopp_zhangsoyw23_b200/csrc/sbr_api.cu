@@ -1,0 +1,491 @@
+// sbr_api.cu -- C ABI and host driver of libsbr (see include/sbr.h).
+//
+// Host loop = Algorithm 1 of the paper in the reading of DESIGN.md:
+//   for each nb-block (origin c0, OA = A[c0+b:, c0+b:] frozen at block start):
+//     for each b-panel t:
+//       a5 (t>=1)  lazy panel update  GA = OA(:,c) - [X | Y] [Y_c^T ; W^T R]
+//       a1/a2      TSQR + reconstruction -> Y_t, W_t^0 = Y_t T_t, R    (k_panel.cu)
+//       a3 (t>=1)  W merge  W_t = W_t^0 - W (Y^T W_t^0)
+//       a4         pass     X_t = OA W_t ;  W^T X column block
+//     a6          Z = X - 1/2 Y (W^T X);  A_trail -= Y Z^T + Z Y^T  (lower)   (Eq. 1-3)
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "../../include/sbr.h"
+#include "kernels.h"
+
+using namespace sbr;
+
+namespace {
+
+std::mutex g_err_mu;
+std::string g_last_err = "";
+
+void set_err(const char* what, cudaError_t e) {
+  std::lock_guard<std::mutex> lk(g_err_mu);
+  g_last_err = std::string(what) + ": " + cudaGetErrorName(e) + " (" + cudaGetErrorString(e) + ")";
+}
+
+struct Stat {
+  int64_t launches = 0;
+  double ms = 0, bytes = 0, flops = 0;
+};
+
+struct Pending {
+  cudaEvent_t e0, e1;
+  int kid;
+  double bytes, flops;
+};
+
+}  // namespace
+
+struct sbr_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  int nsm = 0;
+  // workspace
+  void* ws = nullptr;
+  size_t ws_bytes = 0;
+  int64_t ws_n = -1;
+  int ws_b = -1, ws_nb = -1, ws_mode = -1;
+  float *Yb = nullptr, *Xb = nullptr, *Zb = nullptr, *Wws = nullptr, *Strip = nullptr, *WtX = nullptr,
+        *Pb = nullptr, *Gb = nullptr;
+  float *pv = nullptr, *ptau = nullptr, *pr = nullptr, *pq = nullptr, *pmisc = nullptr;
+  unsigned* flag = nullptr;
+  int panel_ctas = 0;
+  // host-buffer (e2e) device copies
+  void* e2e = nullptr;
+  size_t e2e_bytes = 0;
+  // stats
+  bool timing = false;
+  std::vector<cudaEvent_t> ev_pool;
+  std::vector<Pending> pending;
+  Stat stats[SBR_K_COUNT];
+  int64_t launches = 0;
+};
+
+namespace {
+
+cudaEvent_t get_event(sbr_ctx* h) {
+  if (!h->ev_pool.empty()) {
+    cudaEvent_t e = h->ev_pool.back();
+    h->ev_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e;
+  cudaEventCreate(&e);
+  return e;
+}
+
+struct Scope {  // per-kernel-class timing scope (CUDA events on the handle's stream)
+  sbr_ctx* h;
+  int kid;
+  double bytes, flops;
+  cudaEvent_t e0 = nullptr;
+  Scope(sbr_ctx* h_, int kid_, double bytes_, double flops_) : h(h_), kid(kid_), bytes(bytes_), flops(flops_) {
+    if (h->timing) {
+      e0 = get_event(h);
+      cudaEventRecord(e0, h->stream);
+    }
+  }
+  ~Scope() {
+    if (h->timing) {
+      cudaEvent_t e1 = get_event(h);
+      cudaEventRecord(e1, h->stream);
+      h->pending.push_back({e0, e1, kid, bytes, flops});
+    }
+  }
+};
+
+void drain_stats(sbr_ctx* h) {
+  if (h->pending.empty()) return;
+  cudaStreamSynchronize(h->stream);
+  for (auto& p : h->pending) {
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, p.e0, p.e1);
+    Stat& s = h->stats[p.kid];
+    s.launches += 1;
+    s.ms += ms;
+    s.bytes += p.bytes;
+    s.flops += p.flops;
+    h->ev_pool.push_back(p.e0);
+    h->ev_pool.push_back(p.e1);
+  }
+  h->pending.clear();
+}
+
+#define SBR_CK(expr, what)                 \
+  do {                                     \
+    cudaError_t _e = (expr);               \
+    if (_e != cudaSuccess) {               \
+      set_err(what, _e);                   \
+      return SBR_ERR_CUDA;                 \
+    }                                      \
+  } while (0)
+
+size_t align_up(size_t x) { return (x + 255) & ~size_t(255); }
+
+int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out) {
+  const int64_t M = n - b;
+  const PanelWs pw = panel_ws_sizes(M, b);
+  size_t off = 0;
+  auto take = [&](size_t floats) {
+    size_t o = off;
+    off += align_up(floats * sizeof(float));
+    return o;
+  };
+  const size_t oY = take((size_t)n * nb), oX = take((size_t)n * nb), oZ = take((size_t)n * nb),
+               oW = take((size_t)n * nb), oS = take((size_t)n * nb), oWtX = take((size_t)nb * nb),
+               oP = take((size_t)nb * 64), oG = take((size_t)nb * 64), oPv = take(pw.v), oPt = take(pw.tau),
+               oPr = take(pw.r), oPq = take(pw.q), oPm = take(pw.misc), oF = take(64);
+  if (bytes_out) *bytes_out = off;
+  if (!h) return SBR_OK;
+  if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
+  if (h->ws) {
+    cudaFree(h->ws);
+    h->ws = nullptr;
+    h->ws_bytes = 0;
+  }
+  if (cudaMalloc(&h->ws, off) != cudaSuccess) {
+    cudaGetLastError();
+    return SBR_ERR_NOMEM;
+  }
+  h->ws_bytes = off;
+  h->ws_n = n;
+  h->ws_b = b;
+  h->ws_nb = nb;
+  h->ws_mode = mode;
+  char* base = (char*)h->ws;
+  h->Yb = (float*)(base + oY);
+  h->Xb = (float*)(base + oX);
+  h->Zb = (float*)(base + oZ);
+  h->Wws = (float*)(base + oW);
+  h->Strip = (float*)(base + oS);
+  h->WtX = (float*)(base + oWtX);
+  h->Pb = (float*)(base + oP);
+  h->Gb = (float*)(base + oG);
+  h->pv = (float*)(base + oPv);
+  h->ptau = (float*)(base + oPt);
+  h->pr = (float*)(base + oPr);
+  h->pq = (float*)(base + oPq);
+  h->pmisc = (float*)(base + oPm);
+  h->flag = (unsigned*)(base + oF);
+  h->panel_ctas = panel_max_ctas(b);
+  return SBR_OK;
+}
+
+int validate(sbr_ctx* h, int mode, int64_t n, int b, int nb, const float* A, int64_t lda, const float* AB,
+             int64_t ldab, const float* W, int64_t ldw) {
+  if (!h) return -1;
+  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32) return -2;
+  if (n < 1) return -3;
+  if (b < 1 || b > 64) return -4;
+  if (nb < b || nb % b != 0 || nb > 4096) return -5;
+  if (!A) return -6;
+  if (lda < std::max<int64_t>(1, n)) return -7;
+  if (!AB) return -8;
+  if (ldab < b + 1) return -9;
+  if (W && ldw < n) return -11;
+  return SBR_OK;
+}
+
+// Algorithm 1 on device buffers (arguments already validated).
+int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB, int64_t ldab,
+                  float* W, int64_t ldw) {
+  cudaStream_t st = h->stream;
+  if (n <= b + 1) {
+    Scope sc(h, SBR_K_OTHER, 0, 0);
+    SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
+    h->launches++;
+    return SBR_OK;
+  }
+  int rc = ensure_ws(h, n, b, nb, mode, nullptr);
+  if (rc != SBR_OK) return rc;
+  {
+    Scope sc(h, SBR_K_OTHER, 2.0 * n * n, 0);
+    SBR_CK(check_finite(n, A, lda, h->flag, st), "check_finite");
+    h->launches += (n + 65534) / 65535;
+  }
+  unsigned flag = 0;
+  SBR_CK(cudaMemcpyAsync(&flag, h->flag, sizeof(unsigned), cudaMemcpyDeviceToHost, st), "flag D2H");
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  if (flag) return SBR_ERR_NONFINITE;
+
+  const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
+  const int64_t ldn = n;        // ld of the block buffers
+  for (int64_t c0 = 0; c0 < ncols; c0 += nb) {
+    const int64_t r0 = c0 + b, M = n - r0;
+    const int kJ = (int)std::min<int64_t>(nb, ncols - c0);
+    const int p = (kJ + b - 1) / b;
+    float* Wb = W ? W + r0 + c0 * ldw : h->Wws;
+    const int64_t ldwb = W ? ldw : ldn;
+    float* OA = A + r0 + r0 * lda;
+    const int sw = std::min<int64_t>((int64_t)(p - 1) * b, M);  // OA columns rewritten during the block
+    if (sw > 0) {
+      SBR_CK(cudaMemcpy2DAsync(h->Strip, ldn * sizeof(float), OA, lda * sizeof(float), M * sizeof(float), sw,
+                               cudaMemcpyDeviceToDevice, st),
+             "strip copy");
+    }
+    for (int t = 0; t < p; ++t) {
+      const int64_t g = c0 + (int64_t)t * b;
+      const int64_t tb = (int64_t)t * b;
+      const int64_t m = M - tb;
+      const int k = t * b;
+      if (t >= 1) {  // ---- a5: lazy update of panel t's columns (Alg.1 l.8-10)
+        const int64_t c = tb - b;  // OA column of the panel's first column
+        const int64_t rows = M - c;
+        Scope sc(h, SBR_K_LAZY, 4.0 * rows * (2.0 * k + 2 * b), 4.0 * rows * k * b);
+        SBR_CK(lazy_small_p(k, b, h->Xb + c, ldn, h->WtX, nb, h->Yb + c, ldn, h->Pb, st), "lazy_p");
+        SBR_CK(mirror_lower_block(b, A + g + g * lda, lda, st), "mirror");
+        float* Ablk = A + g + g * lda;
+        SBR_CK(gemm_nn(rows, b, k, -1.f, h->Xb + c, ldn, h->Yb + c, ldn, true, 1.f, Ablk, lda, Ablk, lda, st),
+               "lazy X Yc^T");
+        SBR_CK(gemm_nn(rows, b, k, -1.f, h->Yb + c, ldn, h->Pb, k, false, 1.f, Ablk, lda, Ablk, lda, st),
+               "lazy Y P");
+        h->launches += 4;
+      }
+      {  // ---- a1/a2: TSQR + reconstruction
+        Scope sc(h, SBR_K_PANEL, 4.0 * m * b * 4, 4.0 * m * b * b * 2);
+        PanelArgs pa{};
+        pa.P = A + (g + b) + g * lda;
+        pa.ldp = lda;
+        pa.m = (int)m;
+        pa.b = b;
+        pa.Y = h->Yb + tb * ldn;
+        pa.ldy = ldn;
+        pa.W = Wb + tb * ldwb;
+        pa.ldw = ldwb;
+        pa.row0 = tb;
+        pa.M = M;
+        pa.ws_v = h->pv;
+        pa.ws_tau = h->ptau;
+        pa.ws_r = h->pr;
+        pa.ws_q = h->pq;
+        pa.ws_misc = h->pmisc;
+        SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
+        h->launches += 1;
+      }
+      if (t >= 1) {  // ---- a3: W merge
+        Scope sc(h, SBR_K_WMERGE, 4.0 * (M - tb) * (k + b) + 4.0 * M * (k + 2 * b), 2.0 * (2.0 * M - tb) * k * b);
+        SBR_CK(zero_matrix(k, b, h->Gb, k, st), "zero G");
+        SBR_CK(gemm_tn(M - tb, k, b, 1.f, h->Yb + tb, ldn, Wb + tb + tb * ldwb, ldwb, h->Gb, k, st), "Y^T W0");
+        SBR_CK(gemm_nn(M, b, k, -1.f, Wb, ldwb, h->Gb, k, false, 1.f, Wb + tb * ldwb, ldwb, Wb + tb * ldwb, ldwb,
+                       st),
+               "W merge");
+        h->launches += 2;
+      }
+      {  // ---- a4: pass X_t = OA W_t (symmetric, OA frozen = A + strip copy)
+        Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 8.0 * M * b, 2.0 * M * M * b);
+        SBR_CK(sym_pass(M, b, OA, lda, h->Strip, ldn, sw, Wb + tb * ldwb, ldwb, h->Xb + tb * ldn, ldn, st),
+               "pass");
+        h->launches += 1;
+      }
+      {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
+        Scope sc(h, SBR_K_WMERGE, 4.0 * M * (k + 2 * b), 2.0 * M * (k + b) * b);
+        SBR_CK(zero_matrix(k + b, b, h->WtX + tb * nb, nb, st), "zero wtx");
+        SBR_CK(gemm_tn(M, k + b, b, 1.f, Wb, ldwb, h->Xb + tb * ldn, ldn, h->WtX + tb * nb, nb, st), "W^T X");
+        SBR_CK(mirror_wtx(k, b, h->WtX, nb, st), "mirror wtx");
+        h->launches += 2;
+      }
+    }
+    // ---- a6: trailing update once per block (Alg.1 l.12-13)
+    const int64_t s = (int64_t)p * b - b;
+    const int64_t Mt = M - s;
+    const int kk = p * b;
+    if (Mt > 0) {
+      Scope sc(h, SBR_K_SYR2K, 4.0 * Mt * Mt + 4.0 * Mt * kk * 3, 2.0 * Mt * Mt * kk + 2.0 * Mt * kk * kk);
+      SBR_CK(gemm_nn(Mt, kk, kk, -0.5f, h->Yb + s, ldn, h->WtX, nb, false, 1.f, h->Xb + s, ldn, h->Zb + s, ldn, st),
+             "Z");
+      SBR_CK(syr2k_lower(Mt, kk, h->Yb + s, ldn, h->Zb + s, ldn, A + (r0 + s) + (r0 + s) * lda, lda, st), "syr2k");
+      h->launches += 2;
+    }
+  }
+  {
+    Scope sc(h, SBR_K_OTHER, 8.0 * (b + 1) * n, 0);
+    SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
+    h->launches += 1;
+  }
+  return SBR_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int sbr_create(sbr_handle_t* out, int device, void* stream) {
+  if (!out) return -1;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess) {
+    cudaGetLastError();
+    return SBR_ERR_CUDA;
+  }
+  if (device < 0 || device >= ndev) return -2;
+  SBR_CK(cudaSetDevice(device), "cudaSetDevice");
+  sbr_ctx* h = new sbr_ctx();
+  h->device = device;
+  h->stream = (cudaStream_t)stream;
+  cudaDeviceGetAttribute(&h->nsm, cudaDevAttrMultiProcessorCount, device);
+  *out = h;
+  return SBR_OK;
+}
+
+int sbr_set_stream(sbr_handle_t h, void* stream) {
+  if (!h) return -1;
+  h->stream = (cudaStream_t)stream;
+  return SBR_OK;
+}
+
+int sbr_destroy(sbr_handle_t h) {
+  if (!h) return -1;
+  cudaSetDevice(h->device);
+  cudaStreamSynchronize(h->stream);
+  drain_stats(h);
+  for (auto e : h->ev_pool) cudaEventDestroy(e);
+  if (h->ws) cudaFree(h->ws);
+  if (h->e2e) cudaFree(h->e2e);
+  delete h;
+  return SBR_OK;
+}
+
+int sbr_workspace_query(sbr_handle_t h, int64_t n, int b, int nb, int mode, size_t* bytes) {
+  if (!bytes) return -6;
+  if (n < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (nb < b || nb % b != 0 || nb > 4096) return -4;
+  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32) return -5;
+  if (n <= b + 1) {
+    *bytes = 0;
+    return SBR_OK;
+  }
+  (void)h;
+  return ensure_ws(nullptr, n, b, nb, mode, bytes);
+}
+
+int sbr_reduce(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB, int64_t ldab,
+               float* W, int64_t ldw) {
+  int rc = validate(h, mode, n, b, nb, A, lda, AB, ldab, W, ldw);
+  if (rc != SBR_OK) return rc;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  return reduce_device(h, mode, n, b, nb, A, lda, AB, ldab, W, ldw);
+}
+
+int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB,
+                    int64_t ldab, float* W, int64_t ldw, int outputs) {
+  int rc = validate(h, mode, n, b, nb, A, lda, AB, ldab, W, ldw);
+  if (rc != SBR_OK) return rc;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  const size_t sa = align_up((size_t)n * n * sizeof(float));
+  const size_t sab = align_up((size_t)(b + 1) * n * sizeof(float));
+  const size_t sw = W ? align_up((size_t)n * std::max<int64_t>(1, n - b) * sizeof(float)) : 0;
+  const size_t need = sa + sab + sw;
+  if (h->e2e_bytes < need) {
+    if (h->e2e) cudaFree(h->e2e);
+    h->e2e = nullptr;
+    h->e2e_bytes = 0;
+    if (cudaMalloc(&h->e2e, need) != cudaSuccess) {
+      cudaGetLastError();
+      return SBR_ERR_NOMEM;
+    }
+    h->e2e_bytes = need;
+  }
+  float* dA = (float*)h->e2e;
+  float* dAB = (float*)((char*)h->e2e + sa);
+  float* dW = W ? (float*)((char*)h->e2e + sa + sab) : nullptr;
+  cudaStream_t st = h->stream;
+  SBR_CK(cudaMemcpy2DAsync(dA, n * sizeof(float), A, lda * sizeof(float), n * sizeof(float), n,
+                           cudaMemcpyHostToDevice, st),
+         "H2D A");
+  rc = reduce_device(h, mode, n, b, nb, dA, n, dAB, b + 1, dW, n);
+  if (rc != SBR_OK) return rc;
+  SBR_CK(cudaMemcpy2DAsync(AB, ldab * sizeof(float), dAB, (b + 1) * sizeof(float), (b + 1) * sizeof(float), n,
+                           cudaMemcpyDeviceToHost, st),
+         "D2H AB");
+  if (outputs & SBR_OUT_Y) {
+    SBR_CK(cudaMemcpy2DAsync(A, lda * sizeof(float), dA, n * sizeof(float), n * sizeof(float), n,
+                             cudaMemcpyDeviceToHost, st),
+           "D2H A");
+  }
+  if (W && (outputs & SBR_OUT_W) && n > b) {
+    SBR_CK(cudaMemcpy2DAsync(W, ldw * sizeof(float), dW, n * sizeof(float), n * sizeof(float), n - b,
+                             cudaMemcpyDeviceToHost, st),
+           "D2H W");
+  }
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
+
+int sbr_sync(sbr_handle_t h) {
+  if (!h) return -1;
+  SBR_CK(cudaStreamSynchronize(h->stream), "sync");
+  return SBR_OK;
+}
+
+const char* sbr_status_string(int status) {
+  static thread_local std::string s;
+  switch (status) {
+    case SBR_OK: return "ok";
+    case SBR_ERR_NONFINITE: return "input contains Inf or NaN";
+    case SBR_ERR_CUDA: {
+      std::lock_guard<std::mutex> lk(g_err_mu);
+      s = "CUDA error: " + g_last_err;
+      return s.c_str();
+    }
+    case SBR_ERR_NCCL: return "NCCL error";
+    case SBR_ERR_NOMEM: return "device out of memory";
+    case SBR_ERR_UNSUPPORTED: return "unsupported argument combination";
+    default:
+      if (status < 0) {
+        s = "invalid argument " + std::to_string(-status);
+        return s.c_str();
+      }
+      return "unknown status";
+  }
+}
+
+int sbr_generate_symmetric(sbr_handle_t h, uint64_t seed, int64_t n, float* A, int64_t lda) {
+  if (!h) return -1;
+  if (n < 0) return -3;
+  if (!A) return -4;
+  if (lda < std::max<int64_t>(1, n)) return -5;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  SBR_CK(gen_symmetric(seed, n, A, lda, h->stream), "gen_symmetric");
+  h->launches += (n + 65534) / 65535;
+  return SBR_OK;
+}
+
+int sbr_set_kernel_timing(sbr_handle_t h, int enable) {
+  if (!h) return -1;
+  h->timing = enable != 0;
+  return SBR_OK;
+}
+
+int sbr_reset_kernel_stats(sbr_handle_t h) {
+  if (!h) return -1;
+  drain_stats(h);
+  for (auto& s : h->stats) s = Stat();
+  return SBR_OK;
+}
+
+int sbr_kernel_stats(sbr_handle_t h, int kid, int64_t* launches, double* ms, double* bytes, double* flops) {
+  if (!h) return -1;
+  if (kid < 0 || kid >= SBR_K_COUNT) return -2;
+  drain_stats(h);
+  const Stat& s = h->stats[kid];
+  if (launches) *launches = s.launches;
+  if (ms) *ms = s.ms;
+  if (bytes) *bytes = s.bytes;
+  if (flops) *flops = s.flops;
+  return SBR_OK;
+}
+
+int64_t sbr_launch_count(sbr_handle_t h) { return h ? h->launches : -1; }
+
+const char* sbr_version(void) { return "libsbr 0.1 sm_100a"; }
+
+}  // extern "C"

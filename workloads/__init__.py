@@ -70,12 +70,28 @@ def random_symmetric_columns(n: int, seed: int, c0: int, c1: int) -> np.ndarray:
 
 
 def random_symmetric(n: int, seed: int) -> np.ndarray:
-    """n x n fp32, bit-symmetric, entries U[-1,1) on a 2^-23 grid."""
+    """n x n fp32, bit-symmetric, entries U[-1,1) on a 2^-23 grid.
+
+    Hashes only the lower triangle (column blocks, rows >= the block's first
+    column) and mirrors it block by block."""
     out = np.empty((n, n), dtype=np.float32)
-    step = max(1, (1 << 24) // max(n, 1))
+    step = 256
     for c0 in range(0, n, step):
         c1 = min(n, c0 + step)
-        out[:, c0:c1] = random_symmetric_columns(n, seed, c0, c1)
+        i = np.arange(c0, n, dtype=np.uint64)[:, None]
+        j = np.arange(c0, c1, dtype=np.uint64)[None, :]
+        hi = np.maximum(i, j)
+        lo = np.minimum(i, j)
+        key = (hi << np.uint64(32)) | lo
+        key ^= np.uint64(seed & 0xFFFFFFFFFFFFFFFF)
+        h = splitmix64(key)
+        h >>= np.uint64(40)
+        v = h.astype(np.int64)
+        v -= 1 << 23
+        blk = v.astype(np.float32)
+        blk *= np.float32(2.0 ** -23)
+        out[c0:, c0:c1] = blk
+        out[c0:c1, c0:] = blk.T
     return out
 
 
