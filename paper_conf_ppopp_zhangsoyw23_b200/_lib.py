@@ -45,6 +45,10 @@ SIGNATURES = {
                               ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]),
     "sbr_launch_count": (_i64, [_h]),
     "sbr_version": (ctypes.c_char_p, []),
+    # kernel-level test hooks (include/sbr_testing.h)
+    "sbr_test_pass_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_test_syr2k_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_test_zform_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
 }
 
 _LIB = None

@@ -1,0 +1,220 @@
+// k_gemm_tc.cu -- the per-block trailing update (step a6) on tcgen05 tensor cores.
+//
+//   ZFORM : Z = X - 1/2 Y (W^T X)                       (Eq. 2 analogue; reading C5)
+//   SYR2K : A_low[s:, s:] -= Y_s Z_s^T + Z_s Y_s^T       (Eq. 3; Alg. 1 l.13)
+//           computed as ONE GEMM with K = 2 nb: [Y | Z] [Z | Y]^T, lower tiles only --
+//           the Tensor-Core syr2k the paper lists as future work.
+//
+// Operands are fp16, row-major (K contiguous = K-major for UMMA), fed by TMA with
+// 128-byte swizzle into a 4-stage smem ring; 128 x 256 output tiles accumulate in TMEM
+// (double-buffered: the epilogue of tile i overlaps the MMAs of tile i+1).
+// SYR2K epilogue: C_new = C_old - acc on the fp32 master (lower elements only) and the
+// fp16 shadow of the next block's OA (strict lower, half diagonal; see k_pass_tc.cu).
+// ZFORM epilogue: Zh = fp16(X - acc/2), row-major.
+#include "kernels.h"
+#include "tc.cuh"
+
+namespace sbr {
+
+using namespace tc;
+
+namespace {
+constexpr int G_BM = 128, G_BN = 256, G_BK = 64, G_NS = 4;
+constexpr int G_SA = G_BM * G_BK * 2;  // 16 KB
+constexpr int G_SB = G_BN * G_BK * 2;  // 32 KB
+constexpr int G_STAGE = G_SA + G_SB;
+constexpr int G_OFF_BAR = G_NS * G_STAGE;
+constexpr int G_SMEM = G_OFF_BAR + (2 * G_NS + 4) * 8 + 16 + 1024;
+}  // namespace
+
+// tile index -> (I, Jc)
+template <int MODE>
+SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
+  if (MODE == 1) {  // ZFORM: full grid, row-major
+    I = t / ntn;
+    Jc = t % ntn;
+  } else {          // SYR2K: row I has floor(I/2)+1 tiles of 256 columns
+    int i = 0;
+    while (true) {
+      const int cnt = i / 2 + 1;
+      if (t < cnt) { I = i; Jc = t; return; }
+      t -= cnt;
+      ++i;
+    }
+  }
+}
+
+template <int MODE>
+__global__ void __launch_bounds__(256, 1)
+    gemm_tc_kernel(const __grid_constant__ CUtensorMap mapA0, const __grid_constant__ CUtensorMap mapA1,
+                   const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
+                   int nhalves, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles, float* C,
+                   int64_t ldc, __half* shadow, int64_t ldsh, const float* X, int64_t ldx, __half* Zh, int64_t ldz) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint64_t* bars = (uint64_t*)(smem + G_OFF_BAR);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + G_NS;
+  uint64_t* acc_full = bars + 2 * G_NS;
+  uint64_t* acc_empty = acc_full + 2;
+  uint32_t* tmem_slot = (uint32_t*)(bars + 2 * G_NS + 4);
+  const int warp = warp_id(), lane = lane_id();
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < G_NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 128); }
+    mbar_fence_init();
+  }
+  if (warp == 0 && lane == 0) {
+    tma_prefetch(&mapA0); tma_prefetch(&mapB0);
+    if (nhalves > 1) { tma_prefetch(&mapA1); tma_prefetch(&mapB1); }
+  }
+  if (warp == 2) tmem_alloc(tmem_slot, 512);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const int nk = nhalves * kpb;
+
+  if (warp == 0) {
+    if (lane == 0) {  // ---------------- TMA producer
+      int st = 0; uint32_t ph = 0;
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        int I, Jc;
+        gemm_tile<MODE>(t, ntn, I, Jc);
+        for (int kc = 0; kc < nk; ++kc) {
+          const int half = kc / kpb, kin = (kc % kpb) * G_BK;
+          mbar_wait(&empty[st], ph ^ 1);
+          mbar_expect_tx(&full[st], G_STAGE);
+          uint8_t* sa = smem + st * G_STAGE;
+          tma_load_2d(sa, half ? &mapA1 : &mapA0, &full[st], kin, arow0 + I * G_BM);
+          tma_load_2d(sa + G_SA, half ? &mapB1 : &mapB0, &full[st], kin, brow0 + Jc * G_BN);
+          if (++st == G_NS) { st = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {  // ---------------- MMA issuer
+      constexpr uint32_t idesc = idesc_make(G_BM, G_BN, 0, 0, 0);
+      int st = 0; uint32_t ph = 0;
+      int ab = 0; uint32_t aph = 0;
+      const uint32_t s0 = smem_u32(smem);
+      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        mbar_wait(&acc_empty[ab], aph ^ 1);
+        tc_fence_after();
+        const uint32_t d = tmem + ab * G_BN;
+        for (int kc = 0; kc < nk; ++kc) {
+          mbar_wait(&full[st], ph);
+          tc_fence_after();
+          const uint32_t sa = s0 + st * G_STAGE, sb = sa + G_SA;
+#pragma unroll
+          for (int s = 0; s < G_BK / 16; ++s)
+            mma_f16(d, sdesc_sw128(sa + s * 32, 16, 1024), sdesc_sw128(sb + s * 32, 16, 1024), idesc,
+                    (kc > 0 || s > 0) ? 1u : 0u);
+          mma_commit(&empty[st]);
+          if (++st == G_NS) { st = 0; ph ^= 1; }
+        }
+        mma_commit(&acc_full[ab]);
+        if (++ab == 2) { ab = 0; aph ^= 1; }
+      }
+    }
+  } else if (warp >= 4) {  // ---------------- epilogue
+    const int q = warp - 4;
+    const int rit = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    int ab = 0; uint32_t aph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      int I, Jc;
+      gemm_tile<MODE>(t, ntn, I, Jc);
+      mbar_wait(&acc_full[ab], aph);
+      tc_fence_after();
+      const int64_t row = (int64_t)I * G_BM + rit;
+#pragma unroll 1
+      for (int cc = 0; cc < G_BN / 32; ++cc) {
+        const int64_t col0 = (int64_t)Jc * G_BN + cc * 32;
+        if (MODE == 0 && col0 > (int64_t)I * G_BM + G_BM - 1) break;  // chunk entirely above the diagonal
+        if (col0 >= Ncols) break;
+        float v[32];
+        tmem_ld32(tmem + ab * G_BN + cc * 32 + lane_off, v);
+        if (row >= Mrows) continue;
+        if (MODE == 0) {
+#pragma unroll
+          for (int c = 0; c < 32; ++c) {
+            const int64_t col = col0 + c;
+            if (col <= row) {
+              float* cp = C + row + col * ldc;
+              const float nv = *cp - v[c];
+              *cp = nv;
+              shadow[row + col * ldsh] = __float2half_rn(col == row ? 0.5f * nv : nv);
+            }
+          }
+        } else {
+          __align__(16) __half z[32];
+#pragma unroll
+          for (int c = 0; c < 32; ++c) {
+            const int64_t col = col0 + c;
+            const float xv = (col < Ncols) ? X[row + col * ldx] : 0.f;
+            z[c] = __float2half_rn(fmaf(-0.5f, v[c], xv));
+          }
+          __half* zp = Zh + row * ldz + col0;
+          if (col0 + 32 <= Ncols) {
+#pragma unroll
+            for (int c = 0; c < 32; c += 8) *reinterpret_cast<uint4*>(zp + c) = *reinterpret_cast<const uint4*>(z + c);
+          } else {
+            for (int c = 0; c < 32 && col0 + c < Ncols; ++c) zp[c] = z[c];
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&acc_empty[ab]);
+      if (++ab == 2) { ab = 0; aph ^= 1; }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc_fence_after();
+    tmem_dealloc(tmem, 512);
+  }
+}
+
+template <int MODE>
+static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
+  auto kern = gemm_tc_kernel<MODE>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, G_SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap mA0, mA1, mB0, mB1;
+  cudaError_t e;
+  if ((e = make_tmap_2d(&mA0, p.A0, true, p.K, p.a_rows, p.ld_a, G_BK, G_BM)) != cudaSuccess) return e;
+  if ((e = make_tmap_2d(&mB0, p.B0, true, p.K, p.b_rows, p.ld_b, G_BK, G_BN)) != cudaSuccess) return e;
+  if (MODE == 0) {
+    if ((e = make_tmap_2d(&mA1, p.A1, true, p.K, p.a_rows, p.ld_a, G_BK, G_BM)) != cudaSuccess) return e;
+    if ((e = make_tmap_2d(&mB1, p.B1, true, p.K, p.b_rows, p.ld_b, G_BK, G_BN)) != cudaSuccess) return e;
+  } else {
+    mA1 = mA0;
+    mB1 = mB0;
+  }
+  const int kpb = (int)((p.K + G_BK - 1) / G_BK);
+  const int ntm = (int)((p.Mrows + G_BM - 1) / G_BM);
+  const int ntn = (int)((p.Ncols + G_BN - 1) / G_BN);
+  int ntiles;
+  if (MODE == 0) {
+    ntiles = 0;
+    for (int i = 0; i < ntm; ++i) ntiles += i / 2 + 1;
+  } else {
+    ntiles = ntm * ntn;
+  }
+  if (ntiles == 0) return cudaSuccess;
+  const int grid = std::min(ntiles, p.num_sms);
+  kern<<<grid, 256, G_SMEM, st>>>(mA0, mA1, mB0, mB1, kpb, MODE == 0 ? 2 : 1, (int)p.arow0, (int)p.brow0, p.Mrows,
+                                  p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx, p.Zh, p.ldz);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0>(p, st); }
+cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1>(p, st); }
+
+}  // namespace sbr

@@ -112,4 +112,40 @@ cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaS
   return cudaMemset2DAsync(A, lda * sizeof(float), 0, rows * sizeof(float), cols, st);
 }
 
+// fp16 shadow of the lower triangle: strict lower as is, HALF the diagonal, zero above
+// (so that a diagonal tile T satisfies T + T^T = L; see k_pass_tc.cu).
+__global__ void shadow_init_kernel(int64_t n, int64_t j0, const float* A, int64_t lda, __half* Sh, int64_t ldsh) {
+  const int64_t j = j0 + blockIdx.y;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    float v = 0.f;
+    if (i > j) v = A[i + j * lda];
+    else if (i == j) v = 0.5f * A[i + j * lda];
+    Sh[i + j * ldsh] = __float2half_rn(v);
+  }
+}
+
+cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int64_t ldsh, cudaStream_t st) {
+  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, n - j0);
+    dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 32), (unsigned)nc);
+    shadow_init_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, Sh, ldsh);
+  }
+  return cudaGetLastError();
+}
+
+__global__ void to_half_cm_kernel(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd) {
+  const int c = blockIdx.y;
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += (int64_t)gridDim.x * blockDim.x)
+    dst[r + c * ldd] = __float2half_rn(c < cols ? src[r + c * lds] : 0.f);
+}
+
+// dst[r + c*ldd] = fp16(src[r + c*lds]) for c < cols, 0 for cols <= c < cols_pad
+cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
+                       int64_t ldd, cudaStream_t st) {
+  if (rows <= 0 || cols_pad <= 0) return cudaSuccess;
+  dim3 grid((unsigned)std::min<int64_t>((rows + 255) / 256, 64), (unsigned)cols_pad);
+  to_half_cm_kernel<<<grid, 256, 0, st>>>(rows, cols, src, lds, dst, ldd);
+  return cudaGetLastError();
+}
+
 }  // namespace sbr

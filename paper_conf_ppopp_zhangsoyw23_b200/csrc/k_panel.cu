@@ -244,12 +244,14 @@ __global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
     for (int64_t i = threadIdx.x; i < M; i += blockDim.x) {
       if (i < row0) {
         for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
+        if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
         continue;
       }
       const int64_t il = i - row0;
       for (int c = 0; c < b; ++c) {
         const float y = Vs[il + c * RS];
         a.Y[i + c * a.ldy] = y;
+        if (a.Yh) a.Yh[i * a.ldyh + c] = __float2half_rn(y);
         a.P[il + c * a.ldp] = (il > c) ? y : (il < b ? Rs[il + c * b] : 0.f);
         float w = 0.f;
         for (int k = 0; k <= c; ++k) w = fmaf(Vs[il + k * RS], Ts[k + c * B], w);
@@ -264,9 +266,9 @@ __global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
     for (int k = blockIdx.x; k < a.nodes[lev]; k += gridDim.x) {
       const NodeInfo ni = node_info(a, lev, k);
       const float* vs = node_v(a, lev, k, ni);
-      for (int e = threadIdx.x; e < ni.rows * b; e += blockDim.x) {
-        const int i = e % ni.rows, c = e / ni.rows;
-        Vs[i + c * RS] = vs[e];
+      for (int e = threadIdx.x; e < RS * b; e += blockDim.x) {   // rows >= ni.rows must read 0
+        const int i = e % RS, c = e / RS;
+        Vs[e] = (i < ni.rows) ? vs[i + c * ni.rows] : 0.f;
       }
       if (threadIdx.x < b) taus[threadIdx.x] = a.ws_tau[a.toff[lev] + (int64_t)k * b + threadIdx.x];
       __syncthreads();
@@ -370,6 +372,7 @@ __global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
       const float rfin = Ss[i] * rroot[i + c * b];
       a.P[i + (int64_t)c * a.ldp] = (i > c) ? Ls[i + c * B] : rfin;
       a.Y[(row0 + i) + c * a.ldy] = Ls[i + c * B];
+      if (a.Yh) a.Yh[(row0 + i) * a.ldyh + c] = __float2half_rn(Ls[i + c * B]);
       float w = 0.f;
       for (int k = 0; k <= min(i, c); ++k) w = fmaf(Ls[i + k * B], Tn[k + c * B], w);
       a.W[(row0 + i) + c * a.ldw] = w;
@@ -386,6 +389,7 @@ __global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
   const int64_t nth = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = tid; i < row0; i += nth) {
     for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
+    if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
   }
   for (int64_t il = b + tid; il < a.m; il += nth) {
     float q[B];
@@ -405,6 +409,7 @@ __global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
       if (c < b) {
         a.P[il + (int64_t)c * a.ldp] = q[c];
         a.Y[(row0 + il) + c * a.ldy] = q[c];
+        if (a.Yh) a.Yh[(row0 + il) * a.ldyh + c] = __float2half_rn(q[c]);
       }
     }
 #pragma unroll

@@ -1,0 +1,279 @@
+// k_pass_tc.cu -- the per-panel pass X_t = OA W_t (step a4; Alg. 1 l.9)
+// on tcgen05 tensor cores, reading each lower 128x128 tile of the fp16 shadow of OA
+// from HBM exactly once and using it twice:
+//     X_I += L_IJ   W_J      (A = L_IJ,   MN-major view of the smem tile)
+//     X_J += L_IJ^T W_I      (A = L_IJ^T, K-major view of the SAME smem bytes)
+// The shadow stores the strict lower triangle, HALF the diagonal and zeros above it,
+// so a diagonal tile contributes T W + T^T W = L W with no special case.
+//
+// Work item = (tile-column group of C tiles, segment of tile rows).  One CTA (persistent,
+// 1 per SM) per item stream: TMA producer warp -> single-thread MMA warp -> 4 epilogue
+// warps.  Row accumulators (X_I, double-buffered) and the C column accumulators (X_J)
+// live in TMEM; they are flushed with fp32 reductions into the L2-resident X.
+// Roofline: HBM-bound (2 bytes per stored element, 4 flops/byte at b = 32).
+#include "kernels.h"
+#include "tc.cuh"
+
+namespace sbr {
+
+using namespace tc;
+
+template <int BN, int C, int NS>
+struct PassCfg {
+  static constexpr int WT = 256 * BN;          // bytes of one 128-row W tile (2 K-chunks of BN x 128 B)
+  static constexpr int LT = 32768;             // one 128x128 fp16 tile (4 boxes of 64x64)
+  static constexpr int OFF_WJ = 0;
+  static constexpr int OFF_WI = C * WT;
+  static constexpr int OFF_L = (C + 2) * WT;
+  static constexpr int OFF_BAR = OFF_L + NS * LT;
+  static constexpr int NBAR = 2 * NS + 4 + 4 + 4;
+  static constexpr int SMEM = OFF_BAR + NBAR * 8 + 16 + 1024;  // + alignment slack
+  static constexpr int TMEM_USED = (C + 2) * BN;
+  static constexpr int TMEM_COLS = TMEM_USED <= 32 ? 32 : TMEM_USED <= 64 ? 64 : TMEM_USED <= 128 ? 128
+                                   : TMEM_USED <= 256 ? 256 : 512;
+};
+
+// item index -> (group g, tile rows [i0, i1)): group g spans tile columns [gC, gC+C) and
+// rows gC .. NT-1, cut into segments of SEG rows.
+template <int C>
+SBR_DEV int4 pass_item(int it, int NT, int SEG) {
+  for (int g = 0;; ++g) {
+    const int cnt = (NT - g * C + SEG - 1) / SEG;
+    if (it < cnt) {
+      const int i0 = g * C + it * SEG;
+      return make_int4(g, i0, min(NT, i0 + SEG), 0);
+    }
+    it -= cnt;
+  }
+}
+
+template <int BN, int C, int NS>
+__global__ void __launch_bounds__(256, 1)
+    pass_tc_kernel(const __grid_constant__ CUtensorMap mapL, const __grid_constant__ CUtensorMap mapW, int r0, int M,
+                   int NT, int SEG, int nitems, int b, float* X, int64_t ldx) {
+  using Cfg = PassCfg<BN, C, NS>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* sWj = smem + Cfg::OFF_WJ;
+  uint8_t* sWi = smem + Cfg::OFF_WI;
+  uint8_t* sL = smem + Cfg::OFF_L;
+  uint64_t* bars = (uint64_t*)(smem + Cfg::OFF_BAR);
+  uint64_t* l_full = bars;
+  uint64_t* l_empty = bars + NS;
+  uint64_t* wi_full = bars + 2 * NS;
+  uint64_t* wi_empty = wi_full + 2;
+  uint64_t* racc_full = wi_empty + 2;
+  uint64_t* racc_empty = racc_full + 2;
+  uint64_t* wj_full = racc_empty + 2;
+  uint64_t* wj_empty = wj_full + 1;
+  uint64_t* cacc_full = wj_empty + 1;
+  uint64_t* cacc_empty = cacc_full + 1;
+  uint32_t* tmem_slot = (uint32_t*)(bars + Cfg::NBAR);
+
+  const int warp = warp_id(), lane = lane_id();
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < NS; ++i) { mbar_init(&l_full[i], 1); mbar_init(&l_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&wi_full[i], 1); mbar_init(&wi_empty[i], 1);
+      mbar_init(&racc_full[i], 1); mbar_init(&racc_empty[i], 128);
+    }
+    mbar_init(wj_full, 1); mbar_init(wj_empty, 1);
+    mbar_init(cacc_full, 1); mbar_init(cacc_empty, 128);
+    mbar_fence_init();
+  }
+  if (warp == 0 && lane == 0) { tma_prefetch(&mapL); tma_prefetch(&mapW); }
+  if (warp == 2) tmem_alloc(tmem_slot, Cfg::TMEM_COLS);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+  const uint32_t t_col = tmem;                 // C column accumulators: cols [jj*BN, jj*BN+BN)
+  const uint32_t t_row = tmem + C * BN;        // 2 row accumulators
+
+  if (warp == 0) {
+    // ------------------------------------------------ TMA producer
+    if (lane == 0) {
+      int st = 0; uint32_t ph = 0;            // L ring
+      int ws = 0; uint32_t wph = 0;           // W_I ring
+      uint32_t jph = 0;
+      for (int it = blockIdx.x; it < nitems; it += gridDim.x) {
+        const int4 item = pass_item<C>(it, NT, SEG);
+        const int J0 = item.x * C, i0 = item.y, i1 = item.z;
+        const int ceff = min(C, NT - J0);
+        mbar_wait(wj_empty, jph ^ 1);
+        jph ^= 1;
+        mbar_expect_tx(wj_full, ceff * Cfg::WT);
+        for (int jj = 0; jj < ceff; ++jj)
+          for (int h = 0; h < 2; ++h)
+            tma_load_2d(sWj + jj * Cfg::WT + h * (Cfg::WT / 2), &mapW, wj_full, (J0 + jj) * 128 + h * 64, 0);
+        for (int I = i0; I < i1; ++I) {
+          mbar_wait(&wi_empty[ws], wph ^ 1);
+          mbar_expect_tx(&wi_full[ws], Cfg::WT);
+          for (int h = 0; h < 2; ++h)
+            tma_load_2d(sWi + ws * Cfg::WT + h * (Cfg::WT / 2), &mapW, &wi_full[ws], I * 128 + h * 64, 0);
+          if (++ws == 2) { ws = 0; wph ^= 1; }
+          const int jend = min(J0 + ceff, I + 1);
+          for (int J = J0; J < jend; ++J) {
+            mbar_wait(&l_empty[st], ph ^ 1);
+            mbar_expect_tx(&l_full[st], Cfg::LT);
+            uint8_t* dst = sL + st * Cfg::LT;
+            for (int rb = 0; rb < 2; ++rb)
+              for (int cb = 0; cb < 2; ++cb)
+                tma_load_2d(dst + (rb * 2 + cb) * 8192, &mapL, &l_full[st], r0 + I * 128 + rb * 64,
+                            r0 + J * 128 + cb * 64);
+            if (++st == NS) { st = 0; ph ^= 1; }
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------ MMA issuer (one thread)
+    if (lane == 0) {
+      constexpr uint32_t idesc_dir = idesc_make(128, BN, 0, /*a MN-major*/ 1, 0);
+      constexpr uint32_t idesc_tr = idesc_make(128, BN, 0, 0, 0);
+      int st = 0; uint32_t ph = 0;
+      int ws = 0; uint32_t wph = 0;
+      int rb = 0; uint32_t rph = 0;
+      uint32_t jph = 0, cph = 0;
+      const uint32_t aL = smem_u32(sL), aWj = smem_u32(sWj), aWi = smem_u32(sWi);
+      for (int it = blockIdx.x; it < nitems; it += gridDim.x) {
+        const int4 item = pass_item<C>(it, NT, SEG);
+        const int J0 = item.x * C, i0 = item.y, i1 = item.z;
+        const int ceff = min(C, NT - J0);
+        mbar_wait(wj_full, jph);
+        jph ^= 1;
+        mbar_wait(cacc_empty, cph ^ 1);
+        cph ^= 1;
+        tc_fence_after();
+        uint32_t cinit = 0;
+        for (int I = i0; I < i1; ++I) {
+          mbar_wait(&wi_full[ws], wph);
+          mbar_wait(&racc_empty[rb], rph ^ 1);
+          tc_fence_after();
+          const uint32_t d_row = t_row + rb * BN;
+          const int jend = min(J0 + ceff, I + 1);
+          for (int J = J0; J < jend; ++J) {
+            const int jj = J - J0;
+            mbar_wait(&l_full[st], ph);
+            tc_fence_after();
+            const uint32_t lt = aL + st * Cfg::LT;
+#pragma unroll
+            for (int s = 0; s < 8; ++s) {  // X_I += L W_J : A MN-major (LBO = 16 KB between 64-row atoms)
+              const uint64_t a = sdesc_sw128(lt + (s >> 2) * 8192 + (s & 3) * 2048, 16384, 1024);
+              const uint64_t bd = sdesc_sw128(aWj + jj * Cfg::WT + (s >> 2) * (Cfg::WT / 2) + (s & 3) * 32, 16, 1024);
+              mma_f16(d_row, a, bd, idesc_dir, (J > J0 || s > 0) ? 1u : 0u);
+            }
+            const uint32_t d_col = t_col + jj * BN;
+            const uint32_t acc0 = (cinit >> jj) & 1u;
+#pragma unroll
+            for (int s = 0; s < 8; ++s) {  // X_J += L^T W_I : A K-major (same bytes)
+              const uint64_t a = sdesc_sw128(lt + (s >> 2) * 16384 + (s & 3) * 32, 16, 1024);
+              const uint64_t bd = sdesc_sw128(aWi + ws * Cfg::WT + (s >> 2) * (Cfg::WT / 2) + (s & 3) * 32, 16, 1024);
+              mma_f16(d_col, a, bd, idesc_tr, (acc0 || s > 0) ? 1u : 0u);
+            }
+            cinit |= 1u << jj;
+            mma_commit(&l_empty[st]);
+            if (++st == NS) { st = 0; ph ^= 1; }
+          }
+          mma_commit(&racc_full[rb]);
+          mma_commit(&wi_empty[ws]);
+          if (++ws == 2) { ws = 0; wph ^= 1; }
+          if (++rb == 2) { rb = 0; rph ^= 1; }
+        }
+        mma_commit(cacc_full);
+        mma_commit(wj_empty);
+      }
+    }
+  } else if (warp >= 4) {
+    // ------------------------------------------------ epilogue: TMEM -> fp32 reductions into X
+    const int q = warp - 4;                       // TMEM lane quarter
+    const int row_in_tile = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    int rb = 0; uint32_t rph = 0;
+    uint32_t cph = 0;
+    for (int it = blockIdx.x; it < nitems; it += gridDim.x) {
+      const int4 item = pass_item<C>(it, NT, SEG);
+      const int J0 = item.x * C, i0 = item.y, i1 = item.z;
+      const int ceff = min(C, NT - J0);
+      for (int I = i0; I < i1; ++I) {
+        mbar_wait(&racc_full[rb], rph);
+        tc_fence_after();
+        const int64_t row = (int64_t)I * 128 + row_in_tile;
+#pragma unroll
+        for (int c0 = 0; c0 < BN; c0 += 32) {
+          float v[32];
+          tmem_ld32(t_row + rb * BN + c0 + lane_off, v);
+          if (row < M) {
+#pragma unroll
+            for (int c = 0; c < 32; ++c)
+              if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
+          }
+        }
+        tc_fence_before();
+        mbar_arrive(&racc_empty[rb]);
+        if (++rb == 2) { rb = 0; rph ^= 1; }
+      }
+      mbar_wait(cacc_full, cph);
+      cph ^= 1;
+      tc_fence_after();
+      for (int jj = 0; jj < ceff; ++jj) {
+        if (i1 - 1 < J0 + jj) continue;           // no tile of this column in the segment
+        const int64_t row = (int64_t)(J0 + jj) * 128 + row_in_tile;
+#pragma unroll
+        for (int c0 = 0; c0 < BN; c0 += 32) {
+          float v[32];
+          tmem_ld32(t_col + jj * BN + c0 + lane_off, v);
+          if (row < M) {
+#pragma unroll
+            for (int c = 0; c < 32; ++c)
+              if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(cacc_empty);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    tc_fence_after();
+    tmem_dealloc(tmem, Cfg::TMEM_COLS);
+  }
+}
+
+// ---------------------------------------------------------------- host
+template <int BN, int C, int NS>
+static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
+  using Cfg = PassCfg<BN, C, NS>;
+  auto kern = pass_tc_kernel<BN, C, NS>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  CUtensorMap mapL, mapW;
+  cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 64);
+  if (e != cudaSuccess) return e;
+  e = make_tmap_2d(&mapW, p.Wh, true, p.M, BN, p.ld_wh, 64, BN);
+  if (e != cudaSuccess) return e;
+  const int NT = (int)((p.M + 127) / 128);
+  const int G = (NT + C - 1) / C;
+  const int SEG = p.seg_rows > 0 ? p.seg_rows : 8;
+  int nitems = 0;
+  for (int g = 0; g < G; ++g) nitems += (NT - g * C + SEG - 1) / SEG;
+  const int grid = std::min(nitems, p.num_sms);
+  kern<<<grid, 256, Cfg::SMEM, st>>>(mapL, mapW, (int)p.r0, (int)p.M, NT, SEG, nitems, p.b, p.X, p.ldx);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st) {
+  if (p.b <= 16) return launch_pass_t<16, 8, 4>(p, st);
+  if (p.b <= 32) return launch_pass_t<32, 8, 4>(p, st);
+  return launch_pass_t<64, 4, 3>(p, st);
+}
+
+int pass_bn(int b) { return b <= 16 ? 16 : b <= 32 ? 32 : 64; }
+
+}  // namespace sbr

@@ -3,6 +3,7 @@
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
 #include <stdint.h>
+#include <cuda.h>
 
 namespace sbr {
 
@@ -18,6 +19,8 @@ struct PanelArgs {
   int64_t ldy;
   float* W;
   int64_t ldw;
+  __half* Yh;     // optional fp16 row-major copy of Y (row r, column c at Yh[r*ldyh + c])
+  int64_t ldyh;
   int64_t row0, M;
   // workspace
   float* ws_v;
@@ -67,5 +70,45 @@ cudaError_t sym_pass(int64_t M, int b, const float* OA, int64_t ldoa, const floa
 // C (M x M, lower) -= Y Z^T + Z Y^T, Y, Z: M x K
 cudaError_t syr2k_lower(int64_t M, int K, const float* Y, int64_t ldy, const float* Z, int64_t ldz,
                         float* C, int64_t ldc, cudaStream_t st);
+
+// ---- tcgen05 / TMA path (FP16 mode) ----
+cudaError_t make_tmap_2d(CUtensorMap* map, const void* base, bool fp16, uint64_t inner, uint64_t outer, uint64_t ld,
+                         uint32_t box_inner, uint32_t box_outer);
+
+struct PassLaunch {
+  const __half* shadow;  // n x n fp16 shadow of the trailing matrix (strict lower, half diag, zero upper)
+  int64_t n, ld_shadow;
+  const __half* Wh;      // M x BN fp16, column-major, ld_wh >= M (multiple of 8)
+  int64_t M, ld_wh;
+  int64_t r0;            // OA origin (global row/col of OA(0,0))
+  int b;
+  float* X;              // M x b fp32 output (zeroed by the caller), column-major
+  int64_t ldx;
+  int num_sms;
+  int seg_rows;
+};
+cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st);
+int pass_bn(int b);
+
+struct GemmTcLaunch {
+  // fp16 row-major operands (K contiguous): A rows = output rows, B rows = output cols
+  const __half *A0, *A1, *B0, *B1;  // SYR2K: A=[Y|Z] (A0=Yh, A1=Zh), B=[Z|Y]; ZFORM: A0=Yh, B0=WtXh
+  int64_t K;                        // K per half (columns of the operand arrays used)
+  int64_t a_rows, ld_a, b_rows, ld_b;
+  int64_t arow0, brow0;             // first operand row of output row/col 0
+  int64_t Mrows, Ncols;             // output size
+  float* C; int64_t ldc;            // SYR2K: fp32 master (lower), column-major
+  __half* shadow; int64_t ld_shadow;
+  const float* X; int64_t ldx;      // ZFORM: X (column-major fp32)
+  __half* Zh; int64_t ldz;          // ZFORM: Z out (row-major fp16)
+  int num_sms;
+};
+cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st);
+cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st);
+
+// fp16 conversions
+cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int64_t ldsh, cudaStream_t st);
+cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
+                       int64_t ldd, cudaStream_t st);
 
 }  // namespace sbr

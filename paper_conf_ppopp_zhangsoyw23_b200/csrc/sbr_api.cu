@@ -58,6 +58,8 @@ struct sbr_ctx {
         *Pb = nullptr, *Gb = nullptr;
   float *pv = nullptr, *ptau = nullptr, *pr = nullptr, *pq = nullptr, *pmisc = nullptr;
   unsigned* flag = nullptr;
+  __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr;
+  int64_t ldwh = 0, ldsh = 0, ldk = 0;
   int panel_ctas = 0;
   // host-buffer (e2e) device copies
   void* e2e = nullptr;
@@ -144,6 +146,13 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oW = take((size_t)n * nb), oS = take((size_t)n * nb), oWtX = take((size_t)nb * nb),
                oP = take((size_t)nb * 64), oG = take((size_t)nb * 64), oPv = take(pw.v), oPt = take(pw.tau),
                oPr = take(pw.r), oPq = take(pw.q), oPm = take(pw.misc), oF = take(64);
+  // fp16 operands of the tensor-core path (sizes in floats = halves / 2)
+  const int64_t ldwh = (M + 7) / 8 * 8;       // TMA strides must be multiples of 16 bytes
+  const int64_t ldsh = (n + 7) / 8 * 8;
+  const int64_t ldk = (nb + 7) / 8 * 8;
+  const size_t oSh = take((size_t)ldsh * n / 2 + 8), oYh = take((size_t)n * ldk / 2 + 8),
+               oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
+               oWtXh = take((size_t)nb * ldk / 2 + 8);
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
   if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
@@ -176,6 +185,14 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->pq = (float*)(base + oPq);
   h->pmisc = (float*)(base + oPm);
   h->flag = (unsigned*)(base + oF);
+  h->Sh = (__half*)(base + oSh);
+  h->Yh = (__half*)(base + oYh);
+  h->Zh = (__half*)(base + oZh);
+  h->Wh = (__half*)(base + oWh);
+  h->WtXh = (__half*)(base + oWtXh);
+  h->ldwh = ldwh;
+  h->ldsh = ldsh;
+  h->ldk = ldk;
   h->panel_ctas = panel_max_ctas(b);
   return SBR_OK;
 }
@@ -219,6 +236,12 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
 
   const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
   const int64_t ldn = n;        // ld of the block buffers
+  const bool tc16 = (mode == SBR_FP16_FP32ACC);  // tcgen05 kind::f16 path
+  if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper)
+    Scope sc(h, SBR_K_OTHER, 6.0 * n * n, 0);
+    SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, st), "shadow_init");
+    h->launches += (n + 65534) / 65535;
+  }
   for (int64_t c0 = 0; c0 < ncols; c0 += nb) {
     const int64_t r0 = c0 + b, M = n - r0;
     const int kJ = (int)std::min<int64_t>(nb, ncols - c0);
@@ -227,7 +250,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int64_t ldwb = W ? ldw : ldn;
     float* OA = A + r0 + r0 * lda;
     const int sw = std::min<int64_t>((int64_t)(p - 1) * b, M);  // OA columns rewritten during the block
-    if (sw > 0) {
+    if (sw > 0 && !tc16) {
       SBR_CK(cudaMemcpy2DAsync(h->Strip, ldn * sizeof(float), OA, lda * sizeof(float), M * sizeof(float), sw,
                                cudaMemcpyDeviceToDevice, st),
              "strip copy");
@@ -263,6 +286,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.ldw = ldwb;
         pa.row0 = tb;
         pa.M = M;
+        pa.Yh = tc16 ? h->Yh + tb : nullptr;
+        pa.ldyh = h->ldk;
         pa.ws_v = h->pv;
         pa.ws_tau = h->ptau;
         pa.ws_r = h->pr;
@@ -280,7 +305,27 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
                "W merge");
         h->launches += 2;
       }
-      {  // ---- a4: pass X_t = OA W_t (symmetric, OA frozen = A + strip copy)
+      if (tc16) {  // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA)
+        Scope sc(h, SBR_K_PASS, 1.0 * M * M + 6.0 * M * b, 2.0 * M * M * b);
+        const int bn = pass_bn(b);
+        SBR_CK(to_half_cm(M, b, bn, Wb + tb * ldwb, ldwb, h->Wh, h->ldwh, st), "W -> fp16");
+        SBR_CK(zero_matrix(M, b, h->Xb + tb * ldn, ldn, st), "zero X");
+        PassLaunch pl{};
+        pl.shadow = h->Sh;
+        pl.n = n;
+        pl.ld_shadow = h->ldsh;
+        pl.Wh = h->Wh;
+        pl.M = M;
+        pl.ld_wh = h->ldwh;
+        pl.r0 = r0;
+        pl.b = b;
+        pl.X = h->Xb + tb * ldn;
+        pl.ldx = ldn;
+        pl.num_sms = h->nsm;
+        pl.seg_rows = 8;
+        SBR_CK(launch_pass_tc(pl, st), "pass_tc");
+        h->launches += 2;
+      } else {  // ---- a4 (3xTF32 mode, SIMT fp32 for now): OA frozen = A + strip copy
         Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 8.0 * M * b, 2.0 * M * M * b);
         SBR_CK(sym_pass(M, b, OA, lda, h->Strip, ldn, sw, Wb + tb * ldwb, ldwb, h->Xb + tb * ldn, ldn, st),
                "pass");
@@ -298,7 +343,46 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int64_t s = (int64_t)p * b - b;
     const int64_t Mt = M - s;
     const int kk = p * b;
-    if (Mt > 0) {
+    if (Mt > 0 && tc16) {
+      Scope sc(h, SBR_K_SYR2K, 10.0 * Mt * Mt / 2 + 2.0 * Mt * kk * 4 + 4.0 * Mt * kk,
+               2.0 * Mt * Mt * kk + 2.0 * Mt * kk * kk);
+      SBR_CK(to_half_cm(kk, kk, kk, h->WtX, nb, h->WtXh, h->ldk, st), "WtX -> fp16");
+      GemmTcLaunch gz{};
+      gz.A0 = gz.A1 = h->Yh;
+      gz.B0 = gz.B1 = h->WtXh;
+      gz.K = kk;
+      gz.a_rows = M;
+      gz.ld_a = h->ldk;
+      gz.b_rows = kk;
+      gz.ld_b = h->ldk;
+      gz.arow0 = s;
+      gz.brow0 = 0;
+      gz.Mrows = Mt;
+      gz.Ncols = kk;
+      gz.X = h->Xb + s;
+      gz.ldx = ldn;
+      gz.Zh = h->Zh + s * h->ldk;
+      gz.ldz = h->ldk;
+      gz.num_sms = h->nsm;
+      SBR_CK(launch_zform_tc(gz, st), "zform_tc");
+      GemmTcLaunch gs{};
+      gs.A0 = h->Yh;
+      gs.A1 = h->Zh;
+      gs.B0 = h->Zh;
+      gs.B1 = h->Yh;
+      gs.K = kk;
+      gs.a_rows = gs.b_rows = M;
+      gs.ld_a = gs.ld_b = h->ldk;
+      gs.arow0 = gs.brow0 = s;
+      gs.Mrows = gs.Ncols = Mt;
+      gs.C = A + (r0 + s) + (r0 + s) * lda;
+      gs.ldc = lda;
+      gs.shadow = h->Sh + (r0 + s) + (r0 + s) * h->ldsh;
+      gs.ld_shadow = h->ldsh;
+      gs.num_sms = h->nsm;
+      SBR_CK(launch_syr2k_tc(gs, st), "syr2k_tc");
+      h->launches += 3;
+    } else if (Mt > 0) {
       Scope sc(h, SBR_K_SYR2K, 4.0 * Mt * Mt + 4.0 * Mt * kk * 3, 2.0 * Mt * Mt * kk + 2.0 * Mt * kk * kk);
       SBR_CK(gemm_nn(Mt, kk, kk, -0.5f, h->Yb + s, ldn, h->WtX, nb, false, 1.f, h->Xb + s, ldn, h->Zb + s, ldn, st),
              "Z");
@@ -487,5 +571,146 @@ int sbr_kernel_stats(sbr_handle_t h, int kid, int64_t* launches, double* ms, dou
 int64_t sbr_launch_count(sbr_handle_t h) { return h ? h->launches : -1; }
 
 const char* sbr_version(void) { return "libsbr 0.1 sm_100a"; }
+
+}  // extern "C"
+
+// ====================================================================== test hooks
+#include "../../include/sbr_testing.h"
+
+namespace {
+
+__global__ void f32cm_to_f16rm_kernel(int64_t rows, int cols, const float* src, int64_t lds, __half* dst,
+                                      int64_t ldd) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < rows * cols;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = e / cols;
+    const int c = (int)(e % cols);
+    dst[r * ldd + c] = __float2half_rn(src[r + c * lds]);
+  }
+}
+
+__global__ void f16_to_f32_kernel(int64_t rows, int cols, const __half* src, int64_t lds, bool rowmajor, float* dst,
+                                  int64_t ldd) {
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < rows * cols;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = e % rows;
+    const int c = (int)(e / rows);
+    dst[r + c * ldd] = __half2float(rowmajor ? src[r * lds + c] : src[r + c * lds]);
+  }
+}
+
+struct DevBuf {
+  void* p = nullptr;
+  explicit DevBuf(size_t bytes) {
+    if (cudaMalloc(&p, bytes) != cudaSuccess) p = nullptr;
+  }
+  ~DevBuf() {
+    if (p) cudaFree(p);
+  }
+};
+
+}  // namespace
+
+extern "C" {
+
+int sbr_test_pass_fp16(sbr_handle_t h, int64_t M, int b, const float* OA, int64_t ldoa, const float* W, int64_t ldw,
+                       float* X, int64_t ldx) {
+  if (!h) return -1;
+  if (M < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t ldwh = (M + 7) / 8 * 8;
+  const int64_t ldsh = (M + 7) / 8 * 8;
+  DevBuf sh(sizeof(__half) * ldsh * M), wh(sizeof(__half) * ldwh * 64);
+  if (!sh.p || !wh.p) return SBR_ERR_NOMEM;
+  SBR_CK(shadow_init(M, OA, ldoa, (__half*)sh.p, ldsh, st), "shadow");
+  SBR_CK(to_half_cm(M, b, pass_bn(b), W, ldw, (__half*)wh.p, ldwh, st), "W->fp16");
+  SBR_CK(zero_matrix(M, b, X, ldx, st), "zero X");
+  PassLaunch pl{};
+  pl.shadow = (__half*)sh.p;
+  pl.n = M;
+  pl.ld_shadow = ldsh;
+  pl.Wh = (__half*)wh.p;
+  pl.M = M;
+  pl.ld_wh = ldwh;
+  pl.r0 = 0;
+  pl.b = b;
+  pl.X = X;
+  pl.ldx = ldx;
+  pl.num_sms = h->nsm;
+  pl.seg_rows = 8;
+  SBR_CK(launch_pass_tc(pl, st), "pass_tc");
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
+
+int sbr_test_syr2k_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* Z, int64_t ldz,
+                        float* C, int64_t ldc, float* S, int64_t lds) {
+  if (!h) return -1;
+  if (M < 1) return -2;
+  if (K < 1) return -3;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t kp = (K + 7) / 8 * 8;
+  const int64_t ldsh = (M + 7) / 8 * 8;
+  DevBuf yh(sizeof(__half) * M * kp), zh(sizeof(__half) * M * kp), sh(sizeof(__half) * ldsh * M);
+  if (!yh.p || !zh.p || !sh.p) return SBR_ERR_NOMEM;
+  SBR_CK(cudaMemsetAsync(sh.p, 0, sizeof(__half) * ldsh * M, st), "memset");
+  f32cm_to_f16rm_kernel<<<256, 256, 0, st>>>(M, K, Y, ldy, (__half*)yh.p, kp);
+  f32cm_to_f16rm_kernel<<<256, 256, 0, st>>>(M, K, Z, ldz, (__half*)zh.p, kp);
+  GemmTcLaunch gs{};
+  gs.A0 = (__half*)yh.p;
+  gs.A1 = (__half*)zh.p;
+  gs.B0 = (__half*)zh.p;
+  gs.B1 = (__half*)yh.p;
+  gs.K = K;
+  gs.a_rows = gs.b_rows = M;
+  gs.ld_a = gs.ld_b = kp;
+  gs.arow0 = gs.brow0 = 0;
+  gs.Mrows = gs.Ncols = M;
+  gs.C = C;
+  gs.ldc = ldc;
+  gs.shadow = (__half*)sh.p;
+  gs.ld_shadow = ldsh;
+  gs.num_sms = h->nsm;
+  SBR_CK(launch_syr2k_tc(gs, st), "syr2k_tc");
+  if (S) f16_to_f32_kernel<<<256, 256, 0, st>>>(M, (int)M, (__half*)sh.p, ldsh, false, S, lds);
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
+
+int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
+                        const float* X, int64_t ldx, float* Z, int64_t ldz) {
+  if (!h) return -1;
+  if (M < 1) return -2;
+  if (K < 1) return -3;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t kp = (K + 7) / 8 * 8;
+  DevBuf yh(sizeof(__half) * M * kp), gh(sizeof(__half) * K * kp), zh(sizeof(__half) * M * kp);
+  if (!yh.p || !gh.p || !zh.p) return SBR_ERR_NOMEM;
+  f32cm_to_f16rm_kernel<<<256, 256, 0, st>>>(M, K, Y, ldy, (__half*)yh.p, kp);
+  f32cm_to_f16rm_kernel<<<256, 256, 0, st>>>(K, K, G, ldg, (__half*)gh.p, kp);
+  GemmTcLaunch gz{};
+  gz.A0 = gz.A1 = (__half*)yh.p;
+  gz.B0 = gz.B1 = (__half*)gh.p;
+  gz.K = K;
+  gz.a_rows = M;
+  gz.ld_a = kp;
+  gz.b_rows = K;
+  gz.ld_b = kp;
+  gz.Mrows = M;
+  gz.Ncols = K;
+  gz.X = X;
+  gz.ldx = ldx;
+  gz.Zh = (__half*)zh.p;
+  gz.ldz = kp;
+  gz.num_sms = h->nsm;
+  SBR_CK(launch_zform_tc(gz, st), "zform_tc");
+  f16_to_f32_kernel<<<256, 256, 0, st>>>(M, K, (__half*)zh.p, kp, true, Z, ldz);
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
 
 }  // extern "C"
