@@ -44,12 +44,16 @@ SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
   }
 }
 
+constexpr int G_EPI_WARPS = 8;  // two warps per TMEM lane quarter, each half of the 256 columns
+constexpr int G_THREADS = 128 + 32 * G_EPI_WARPS;
+
 template <int MODE>
-__global__ void __launch_bounds__(256, 1)
+__global__ void __launch_bounds__(G_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap mapA0, const __grid_constant__ CUtensorMap mapA1,
                    const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
                    int nhalves, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles, float* C,
-                   int64_t ldc, __half* shadow, int64_t ldsh, const float* X, int64_t ldx, __half* Zh, int64_t ldz) {
+                   int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, const float* __restrict__ X, int64_t ldx,
+                   __half* __restrict__ Zh, int64_t ldz) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint64_t* bars = (uint64_t*)(smem + G_OFF_BAR);
@@ -61,7 +65,7 @@ __global__ void __launch_bounds__(256, 1)
   const int warp = warp_id(), lane = lane_id();
   if (threadIdx.x == 0) {
     for (int i = 0; i < G_NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 128); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 32 * G_EPI_WARPS); }
     mbar_fence_init();
   }
   if (warp == 0 && lane == 0) {
@@ -117,8 +121,10 @@ __global__ void __launch_bounds__(256, 1)
         if (++ab == 2) { ab = 0; aph ^= 1; }
       }
     }
-  } else if (warp >= 4) {  // ---------------- epilogue
-    const int q = warp - 4;
+  } else if (warp >= 4) {  // ---------------- epilogue (8 warps)
+    const int e = warp - 4;
+    const int q = e & 3;                    // TMEM lane quarter (warp % 4)
+    const int chalf = e >> 2;               // which 128 of the 256 accumulator columns
     const int rit = q * 32 + lane;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     int ab = 0; uint32_t aph = 0;
@@ -128,33 +134,36 @@ __global__ void __launch_bounds__(256, 1)
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();
       const int64_t row = (int64_t)I * G_BM + rit;
+      const int64_t rmax = (int64_t)I * G_BM + G_BM - 1;  // last row of the tile
 #pragma unroll 1
-      for (int cc = 0; cc < G_BN / 32; ++cc) {
+      for (int cc = chalf * 4; cc < chalf * 4 + 4; ++cc) {
         const int64_t col0 = (int64_t)Jc * G_BN + cc * 32;
-        if (MODE == 0 && col0 > (int64_t)I * G_BM + G_BM - 1) break;  // chunk entirely above the diagonal
+        if (MODE == 0 && col0 > rmax) break;  // chunk entirely above the diagonal (warp-uniform)
         if (col0 >= Ncols) break;
         float v[32];
         tmem_ld32(tmem + ab * G_BN + cc * 32 + lane_off, v);
         if (row >= Mrows) continue;
         if (MODE == 0) {
+          float* cp = C + row + col0 * ldc;
+          float old[32];
+#pragma unroll
+          for (int c = 0; c < 32; ++c) old[c] = (col0 + c <= row) ? __ldcs(cp + c * ldc) : 0.f;   // all loads first
 #pragma unroll
           for (int c = 0; c < 32; ++c) {
             const int64_t col = col0 + c;
             if (col <= row) {
-              float* cp = C + row + col * ldc;
-              const float nv = *cp - v[c];
-              *cp = nv;
+              const float nv = old[c] - v[c];
+              __stcs(cp + c * ldc, nv);
               shadow[row + col * ldsh] = __float2half_rn(col == row ? 0.5f * nv : nv);
             }
           }
         } else {
+          float xv[32];
+#pragma unroll
+          for (int c = 0; c < 32; ++c) xv[c] = (col0 + c < Ncols) ? __ldcs(X + row + (col0 + c) * ldx) : 0.f;
           __align__(16) __half z[32];
 #pragma unroll
-          for (int c = 0; c < 32; ++c) {
-            const int64_t col = col0 + c;
-            const float xv = (col < Ncols) ? X[row + col * ldx] : 0.f;
-            z[c] = __float2half_rn(fmaf(-0.5f, v[c], xv));
-          }
+          for (int c = 0; c < 32; ++c) z[c] = __float2half_rn(fmaf(-0.5f, v[c], xv[c]));
           __half* zp = Zh + row * ldz + col0;
           if (col0 + 32 <= Ncols) {
 #pragma unroll
@@ -209,7 +218,7 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   }
   if (ntiles == 0) return cudaSuccess;
   const int grid = std::min(ntiles, p.num_sms);
-  kern<<<grid, 256, G_SMEM, st>>>(mA0, mA1, mB0, mB1, kpb, MODE == 0 ? 2 : 1, (int)p.arow0, (int)p.brow0, p.Mrows,
+  kern<<<grid, G_THREADS, G_SMEM, st>>>(mA0, mA1, mB0, mB1, kpb, MODE == 0 ? 2 : 1, (int)p.arow0, (int)p.brow0, p.Mrows,
                                   p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx, p.Zh, p.ldz);
   return cudaGetLastError();
 }

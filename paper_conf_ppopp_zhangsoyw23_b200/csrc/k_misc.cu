@@ -148,4 +148,57 @@ cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, i
   return cudaGetLastError();
 }
 
+__global__ void f32cm_to_f16rm_kernel2(int64_t rows, int cols, const float* src, int64_t lds, __half* dst,
+                                       int64_t ldd) {
+  // thread per (row, 8-column group): coalesced-enough reads along rows, 16-byte row writes
+  const int groups = (cols + 7) / 8;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < rows * groups;
+       e += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = e % rows;
+    const int g = (int)(e / rows);
+    __align__(16) __half v[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const int c = g * 8 + i;
+      v[i] = __float2half_rn(c < cols ? src[r + (int64_t)c * lds] : 0.f);
+    }
+    if (g * 8 + 8 <= cols && ((r * ldd + g * 8) & 7) == 0) {
+      *reinterpret_cast<uint4*>(dst + r * ldd + g * 8) = *reinterpret_cast<const uint4*>(v);
+    } else {
+      for (int i = 0; i < 8 && g * 8 + i < cols; ++i) dst[r * ldd + g * 8 + i] = v[i];
+    }
+  }
+}
+
+cudaError_t f32cm_to_f16rm(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd,
+                           cudaStream_t st) {
+  if (rows <= 0 || cols <= 0) return cudaSuccess;
+  const int64_t work = rows * ((cols + 7) / 8);
+  f32cm_to_f16rm_kernel2<<<(unsigned)std::min<int64_t>((work + 255) / 256, 1184), 256, 0, st>>>(rows, cols, src, lds,
+                                                                                               dst, ldd);
+  return cudaGetLastError();
+}
+
+// B operand of the lazy update: row n = [ Y(c+n, 0:k) | 0 .. | P(0:k, n)^T ] with the second part
+// starting at column 64*ceil(k/64) (see SkinnyNN).
+__global__ void build_lazy_b_kernel(int k, int b, const __half* Yh, int64_t ldyh, int64_t c, const float* P,
+                                    __half* Bl, int64_t ldbl) {
+  const int kp = (k + 63) / 64 * 64;
+  const int n = blockIdx.y;
+  for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < kp + k; j += gridDim.x * blockDim.x) {
+    __half v;
+    if (j < k) v = Yh[(c + n) * ldyh + j];
+    else if (j < kp) v = __float2half_rn(0.f);
+    else v = __float2half_rn(P[(j - kp) + (int64_t)n * k]);
+    Bl[n * ldbl + j] = v;
+  }
+}
+
+cudaError_t build_lazy_b(int k, int b, const __half* Yh, int64_t ldyh, int64_t c, const float* P, __half* Bl,
+                         int64_t ldbl, cudaStream_t st) {
+  const int kp = (k + 63) / 64 * 64;
+  build_lazy_b_kernel<<<dim3((kp + k + 255) / 256, b), 256, 0, st>>>(k, b, Yh, ldyh, c, P, Bl, ldbl);
+  return cudaGetLastError();
+}
+
 }  // namespace sbr

@@ -51,6 +51,15 @@ cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_
                     const float* B, int64_t ldb, bool transB, float beta, const float* C, int64_t ldc,
                     float* D, int64_t ldd, cudaStream_t st);
 
+// ---- small split-K SIMT kernels (k_small.cu); D is zeroed and accumulated atomically ----
+// D = alpha * A op(B) + beta * op(C); op(B) = B^T (B stored n x K) if transB; op(C) = C^T if transC
+cudaError_t small_gemm(int m, int n, int K, float alpha, const float* A, int64_t lda, const float* B, int64_t ldb,
+                       bool transB, float beta, const float* C, int64_t ldc, bool transC, float* D, int64_t ldd,
+                       cudaStream_t st);
+// D[b x b] = A^T B over `rows` rows
+cudaError_t tn_small(int64_t rows, int b, const float* A, int64_t lda, const float* B, int64_t ldb, float* D,
+                     int64_t ldd, cudaStream_t st);
+
 // ---- misc ----
 cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaStream_t st);
 cudaError_t check_finite(int64_t n, const float* A, int64_t lda, unsigned* flag, cudaStream_t st);
@@ -106,7 +115,37 @@ struct GemmTcLaunch {
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st);
 
+// skinny tcgen05 GEMMs (k_skinny_tc.cu)
+struct SkinnyNN {                 // D[rows x b] = C - [A0 | A1] B^T
+  const __half *A0, *A1;          // row-major fp16, K0 / K1 columns used, a_rows x lda
+  int64_t K0, K1, a_rows, lda, arow0;
+  const __half* B;                // b x ldb row-major: cols [0,K0) | zero pad to 64*ceil(K0/64) | [.., +K1)
+  int64_t ldb;
+  int64_t rows;
+  int b;
+  const float* C; int64_t ldc;    // column-major fp32 (may alias D)
+  float* D; int64_t ldd;
+  __half* Hcm; int64_t ldhc;      // optional fp16 column-major copy of D
+  __half* Hrm; int64_t ldhr;      // optional fp16 row-major copy of D
+};
+cudaError_t launch_skinny_nn(const SkinnyNN& p, cudaStream_t st);
+struct SkinnyTN {                 // D0 += A0[rows]^T B[rows], D1 += A1[rows]^T B[rows] (fp32 reductions)
+  const __half *A0, *A1;          // row-major fp16 (a_rows x lda), K1 columns; A1 may be NULL
+  int64_t K1, a_rows, lda;
+  const __half* B;                // column-major fp16 (b_rows x b), ld ldb
+  int64_t b_rows, ldb;
+  int64_t row0, rows;             // reduction rows [row0, row0+rows)
+  int b;
+  float *D0, *D1; int64_t ldd;    // K1 x b, column-major, pre-zeroed
+  int num_sms;
+};
+cudaError_t launch_skinny_tn(const SkinnyTN& p, cudaStream_t st);
+
 // fp16 conversions
+cudaError_t f32cm_to_f16rm(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd,
+                           cudaStream_t st);
+cudaError_t build_lazy_b(int k, int b, const __half* Yh, int64_t ldyh, int64_t c, const float* P, __half* Bl,
+                         int64_t ldbl, cudaStream_t st);
 cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int64_t ldsh, cudaStream_t st);
 cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
                        int64_t ldd, cudaStream_t st);

@@ -58,8 +58,10 @@ struct sbr_ctx {
         *Pb = nullptr, *Gb = nullptr;
   float *pv = nullptr, *ptau = nullptr, *pr = nullptr, *pq = nullptr, *pmisc = nullptr;
   unsigned* flag = nullptr;
-  __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr;
-  int64_t ldwh = 0, ldsh = 0, ldk = 0;
+  __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr, *Xh = nullptr, *Wrh = nullptr,
+         *Bl = nullptr, *Gh = nullptr;
+  float* Hb = nullptr;
+  int64_t ldwh = 0, ldsh = 0, ldk = 0, ldbl = 0;
   int panel_ctas = 0;
   // host-buffer (e2e) device copies
   void* e2e = nullptr;
@@ -152,7 +154,9 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   const int64_t ldk = (nb + 7) / 8 * 8;
   const size_t oSh = take((size_t)ldsh * n / 2 + 8), oYh = take((size_t)n * ldk / 2 + 8),
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
-               oWtXh = take((size_t)nb * ldk / 2 + 8);
+               oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
+               oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
+               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64);
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
   if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
@@ -190,6 +194,12 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->Zh = (__half*)(base + oZh);
   h->Wh = (__half*)(base + oWh);
   h->WtXh = (__half*)(base + oWtXh);
+  h->Xh = (__half*)(base + oXh);
+  h->Wrh = (__half*)(base + oWrh);
+  h->Bl = (__half*)(base + oBl);
+  h->Gh = (__half*)(base + oGh);
+  h->Hb = (float*)(base + oHb);
+  h->ldbl = 2 * ldk + 128;
   h->ldwh = ldwh;
   h->ldsh = ldsh;
   h->ldk = ldk;
@@ -263,15 +273,40 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       if (t >= 1) {  // ---- a5: lazy update of panel t's columns (Alg.1 l.8-10)
         const int64_t c = tb - b;  // OA column of the panel's first column
         const int64_t rows = M - c;
-        Scope sc(h, SBR_K_LAZY, 4.0 * rows * (2.0 * k + 2 * b), 4.0 * rows * k * b);
-        SBR_CK(lazy_small_p(k, b, h->Xb + c, ldn, h->WtX, nb, h->Yb + c, ldn, h->Pb, st), "lazy_p");
-        SBR_CK(mirror_lower_block(b, A + g + g * lda, lda, st), "mirror");
         float* Ablk = A + g + g * lda;
-        SBR_CK(gemm_nn(rows, b, k, -1.f, h->Xb + c, ldn, h->Yb + c, ldn, true, 1.f, Ablk, lda, Ablk, lda, st),
-               "lazy X Yc^T");
-        SBR_CK(gemm_nn(rows, b, k, -1.f, h->Yb + c, ldn, h->Pb, k, false, 1.f, Ablk, lda, Ablk, lda, st),
-               "lazy Y P");
-        h->launches += 4;
+        if (tc16) {  // GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
+          Scope sc(h, SBR_K_LAZY, 2.0 * rows * 2.0 * k + 8.0 * rows * b, 4.0 * rows * k * b);
+          SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Yb + c, ldn, true, 1.f, h->Xb + c, ldn, true, h->Pb, k, st), "lazy_p");
+          SBR_CK(build_lazy_b(k, b, h->Yh, h->ldk, c, h->Pb, h->Bl, h->ldbl, st), "lazy_b");
+          SBR_CK(mirror_lower_block(b, Ablk, lda, st), "mirror");
+          SkinnyNN q{};
+          q.A0 = h->Xh;
+          q.A1 = h->Yh;
+          q.K0 = k;
+          q.K1 = k;
+          q.a_rows = M;
+          q.lda = h->ldk;
+          q.arow0 = c;
+          q.B = h->Bl;
+          q.ldb = h->ldbl;
+          q.rows = rows;
+          q.b = b;
+          q.C = Ablk;
+          q.ldc = lda;
+          q.D = Ablk;
+          q.ldd = lda;
+          SBR_CK(launch_skinny_nn(q, st), "lazy_nn");
+          h->launches += 4;
+        } else {
+          Scope sc(h, SBR_K_LAZY, 4.0 * rows * (2.0 * k + 2 * b), 4.0 * rows * k * b);
+          SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Yb + c, ldn, true, 1.f, h->Xb + c, ldn, true, h->Pb, k, st), "lazy_p");
+          SBR_CK(mirror_lower_block(b, Ablk, lda, st), "mirror");
+          SBR_CK(gemm_nn(rows, b, k, -1.f, h->Xb + c, ldn, h->Yb + c, ldn, true, 1.f, Ablk, lda, Ablk, lda, st),
+                 "lazy X Yc^T");
+          SBR_CK(gemm_nn(rows, b, k, -1.f, h->Yb + c, ldn, h->Pb, k, false, 1.f, Ablk, lda, Ablk, lda, st),
+                 "lazy Y P");
+          h->launches += 4;
+        }
       }
       {  // ---- a1/a2: TSQR + reconstruction
         Scope sc(h, SBR_K_PANEL, 4.0 * m * b * 4, 4.0 * m * b * b * 2);
@@ -296,7 +331,66 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
         h->launches += 1;
       }
-      if (t >= 1) {  // ---- a3: W merge
+      float* Wt = Wb + tb * ldwb;  // this panel's W columns (W_t^0 from the panel, then W_t)
+      if (tc16) {
+        // ---- a3 on tcgen05: G = Y^T W0, H = X^T W0 (one pass over Y, X); W^T X_t = H - (W^T X) G;
+        //      W_t = W0 - W G, written as fp32 + fp16 (column-major for the pass, row-major for later merges)
+        Scope sc(h, SBR_K_WMERGE, t >= 1 ? (2.0 * (M - tb) * 2.0 * k + 2.0 * M * k + 12.0 * M * b) : 6.0 * M * b,
+                 t >= 1 ? 2.0 * (2.0 * (M - tb) + M) * k * b : 0.0);
+        const int bn = pass_bn(b);
+        SBR_CK(to_half_cm(M, b, bn, Wt, ldwb, h->Wh, h->ldwh, st), "W0 -> fp16");
+        if (t >= 1) {
+          SBR_CK(zero_matrix(k, b, h->Gb, k, st), "zero G");
+          SBR_CK(zero_matrix(k, b, h->Hb, k, st), "zero H");
+          SkinnyTN q{};
+          q.A0 = h->Yh;
+          q.A1 = h->Xh;
+          q.K1 = k;
+          q.a_rows = M;
+          q.lda = h->ldk;
+          q.B = h->Wh;
+          q.b_rows = M;
+          q.ldb = h->ldwh;
+          q.row0 = tb;
+          q.rows = M - tb;
+          q.b = b;
+          q.D0 = h->Gb;
+          q.D1 = h->Hb;
+          q.ldd = k;
+          q.num_sms = h->nsm;
+          SBR_CK(launch_skinny_tn(q, st), "Y^T W0, X^T W0");
+          // W^T X_t (rows < k) = H - (W^T X) G  (symmetry of OA: W_{<t}^T OA W_t = X_{<t}^T W_t)
+          SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Gb, k, false, 1.f, h->Hb, k, false, h->WtX + tb * nb, nb, st),
+                 "WtX col");
+          SBR_CK(mirror_wtx(k, b, h->WtX, nb, st), "mirror wtx");
+          SBR_CK(to_half_cm(k, b, b, h->Gb, k, h->Gh, k, st), "G -> fp16");
+          SkinnyNN mq{};
+          mq.A0 = h->Wrh;
+          mq.A1 = nullptr;
+          mq.K0 = k;
+          mq.K1 = 0;
+          mq.a_rows = M;
+          mq.lda = h->ldk;
+          mq.arow0 = 0;
+          mq.B = h->Gh;
+          mq.ldb = k;
+          mq.rows = M;
+          mq.b = b;
+          mq.C = Wt;
+          mq.ldc = ldwb;
+          mq.D = Wt;
+          mq.ldd = ldwb;
+          mq.Hcm = h->Wh;
+          mq.ldhc = h->ldwh;
+          mq.Hrm = h->Wrh + tb;
+          mq.ldhr = h->ldk;
+          SBR_CK(launch_skinny_nn(mq, st), "W merge");
+          h->launches += 6;
+        } else {
+          SBR_CK(f32cm_to_f16rm(M, b, Wt, ldwb, h->Wrh, h->ldk, st), "W -> fp16 rm");
+          h->launches += 2;
+        }
+      } else if (t >= 1) {  // ---- a3 (SIMT fp32): W merge
         Scope sc(h, SBR_K_WMERGE, 4.0 * (M - tb) * (k + b) + 4.0 * M * (k + 2 * b), 2.0 * (2.0 * M - tb) * k * b);
         SBR_CK(zero_matrix(k, b, h->Gb, k, st), "zero G");
         SBR_CK(gemm_tn(M - tb, k, b, 1.f, h->Yb + tb, ldn, Wb + tb + tb * ldwb, ldwb, h->Gb, k, st), "Y^T W0");
@@ -307,8 +401,6 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       }
       if (tc16) {  // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA)
         Scope sc(h, SBR_K_PASS, 1.0 * M * M + 6.0 * M * b, 2.0 * M * M * b);
-        const int bn = pass_bn(b);
-        SBR_CK(to_half_cm(M, b, bn, Wb + tb * ldwb, ldwb, h->Wh, h->ldwh, st), "W -> fp16");
         SBR_CK(zero_matrix(M, b, h->Xb + tb * ldn, ldn, st), "zero X");
         PassLaunch pl{};
         pl.shadow = h->Sh;
@@ -331,7 +423,12 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
                "pass");
         h->launches += 1;
       }
-      {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
+      if (tc16) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b)
+        Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
+        SBR_CK(f32cm_to_f16rm(M, b, h->Xb + tb * ldn, ldn, h->Xh + tb, h->ldk, st), "X -> fp16");
+        SBR_CK(tn_small(M, b, Wt, ldwb, h->Xb + tb * ldn, ldn, h->WtX + tb + tb * nb, nb, st), "Wt^T Xt");
+        h->launches += 2;
+      } else {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
         Scope sc(h, SBR_K_WMERGE, 4.0 * M * (k + 2 * b), 2.0 * M * (k + b) * b);
         SBR_CK(zero_matrix(k + b, b, h->WtX + tb * nb, nb, st), "zero wtx");
         SBR_CK(gemm_tn(M, k + b, b, 1.f, Wb, ldwb, h->Xb + tb * ldn, ldn, h->WtX + tb * nb, nb, st), "W^T X");
