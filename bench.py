@@ -118,27 +118,27 @@ class ClockSampler:
 
 
 def cpu_oracle_sample(n: int, b: int, a_host, budget_s: float):
-    """Time the CPU oracle (oracle.sbr.sbr_unblocked, fp64, as it stands) on a prefix of
-    the same n x n reduction and extrapolate by per-column cost (n-c-b)."""
+    """Time the CPU oracle (oracle.sbr.sbr_unblocked, fp64 numpy, as it stands) on a prefix of
+    the same n x n reduction and extrapolate: setup (measured) + loop time scaled by the
+    per-column cost (n - c - b) of the remaining columns."""
     import numpy as np
 
     from oracle import sbr as osbr
 
     ncol_total = max(0, n - b - 1)
-    # first call: 2 columns to estimate the per-column cost, then size the sample
-    cols = 2
+    st = {}
     t0 = time.perf_counter()
-    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=cols)
-    t1 = time.perf_counter() - t0
-    per = t1 / cols
-    cols = int(max(2, min(ncol_total, budget_s / max(per, 1e-9))))
-    t0 = time.perf_counter()
-    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=cols)
-    ts = time.perf_counter() - t0
+    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=1, stats=st)
+    t_first = time.perf_counter() - t0
+    per_col = max(st["loop_seconds"], 1e-6)
+    setup = max(t_first - st["loop_seconds"], 0.0)
+    cols = int(max(1, min(ncol_total, (budget_s - setup) / per_col)))
+    st = {}
+    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=cols, stats=st)
     c = np.arange(ncol_total, dtype=np.float64)
     w = (n - c - b)
     frac = float(w[:cols].sum() / w.sum())
-    t_full = ts / frac
+    t_full = setup + st["loop_seconds"] / frac
     cores = len(os.sched_getaffinity(0))
     try:
         from threadpoolctl import threadpool_info
@@ -152,8 +152,8 @@ def cpu_oracle_sample(n: int, b: int, a_host, budget_s: float):
         "cores": int(thr),
         "kind": "oracle",
         "sample": f"oracle.sbr.sbr_unblocked (fp64 numpy, as it stands) on the first {cols} of {ncol_total} "
-                  f"columns of the same n={n} b={b} input ({ts:.1f} s, incl. the fp64 copy), extrapolated "
-                  f"by per-column cost (n-c-b): full run ~{t_full:.0f} s",
+                  f"columns of the same n={n} b={b} input: setup {setup:.1f} s + {st['loop_seconds']:.1f} s loop, "
+                  f"extrapolated by per-column cost (n-c-b) to ~{t_full:.3g} s for the full reduction",
         "seconds_extrapolated": t_full,
     }
 

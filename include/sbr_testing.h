@@ -34,6 +34,12 @@ int sbr_test_syr2k_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
                         const float* X, int64_t ldx, float* Z, int64_t ldz);
 
+/* One panel factorisation (TSQR + reconstruction, steps a1-a2) of the m x b panel P
+ * (overwritten with the compact form); explicit Y and W = Y T (m x b, ld ldyw).  If
+ * trace != NULL it receives 16 int64 globaltimer stamps (ns) of the kernel's phases. */
+int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_t ldp, float* Y, float* W, int64_t ldyw,
+                   int64_t* trace);
+
 #ifdef __cplusplus
 }
 #endif

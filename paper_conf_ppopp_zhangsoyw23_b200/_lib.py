@@ -49,6 +49,7 @@ SIGNATURES = {
     "sbr_test_pass_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_syr2k_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_zform_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_test_panel": (_i, [_h, _i64, _i, _p, _i64, _p, _p, _i64, _p]),
 }
 
 _LIB = None

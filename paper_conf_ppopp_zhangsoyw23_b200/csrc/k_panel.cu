@@ -5,23 +5,23 @@
 // modified Gram-Schmidt on each small block", "each warp is in charge of one
 // column").  Sec. 5.2 (Alg. 3 + Ballard's sign matrix S, reading
 // C7): the explicit Q of the tree is turned back into Householder vectors by the
-// non-pivoted LU  Q_1 - S = L U  (s_j = -sign(d_j) chosen on the fly),
-// Y = [L; Q_2 U^-1],  T = -U S L^-T,  W = Y T,  R = S R_tree.
+// non-pivoted LU  Q_1 - S = L U  (s_j = -sign(d_j) chosen on the fly):
+//     Y = [L; Q_2 U^-1],   W = Y T = (E - Q S) L^-T,   R = S R_tree.
+// Each row of Y and W is obtained by two b x b triangular solves (with U and with L),
+// so the T factor is never formed.
 //
-// One cooperative kernel does the whole panel (grid barriers between tree levels):
-//   up sweep   : leaves (<= 512 rows, b <= 32) and inner nodes (stacked child R's)
-//                are QR-factored in registers, one warp per column; V, tau, R -> ws.
-//   down sweep : explicit Q = H_node [C; 0] from the root down; leaves write their
-//                Q rows over the panel.
-//   reconstruct: CTA 0 runs the modified LU on Q's top b x b block and forms
-//                T = -U S L^-T; every row i >= b then solves y_i U = q_i and
-//                w_i = y_i T (thread per row).
-// A panel that fits one leaf (m <= 32*S rows) is factored directly (exact LAPACK
-// dgeqr2 convention, T by the dlarft recurrence), without tree or reconstruction.
-//
-// Outputs: the panel in A is overwritten in LAPACK compact form (R on and above
-// the diagonal, Y's tail strictly below); explicit Y and W^0 = Y T columns
-// (with zero rows above row0) go to the block's Y and W buffers.
+// One cooperative kernel per panel, one CTA (16 warps, each owning b/16 columns) per
+// leaf of <= 256 rows, inner tree nodes of <= 512 rows (16 stacked R factors for b=32):
+//   up    : node QR in registers; the reflector of column j is broadcast through shared
+//           memory and read ONCE into registers by every warp; V -> ws; grid barrier
+//           per level; the root CTA factors the root and forms its explicit Q directly.
+//   down  : each node forms H_node [C; 0] from its parent's block C; a leaf keeps its
+//           Q rows in shared memory.  CTA 0 (leaf 0 holds Q's top b rows) runs the
+//           modified LU in one warp (columns in registers) and publishes L, U, S.
+//   rows  : after one more grid barrier every CTA solves its own rows from shared
+//           memory and writes Y (fp32 + fp16 row-major), W^0 and the compact panel.
+// A panel of <= 512 rows is factored directly by one CTA (LAPACK dgeqr2 convention,
+// T by the dlarft recurrence) -- no tree and no reconstruction.
 #include <cooperative_groups.h>
 
 #include "common.cuh"
@@ -31,70 +31,155 @@ namespace cg = cooperative_groups;
 
 namespace sbr {
 
-// Householder QR of a register-resident node (rows x b), warp w owns columns
-// w, w+32, ... (slot j), lane l owns rows l, l+32, ... (slot s).  Writes the
-// reflectors (unit diagonal, zeros above) to Vs (ld RS), taus, and R (b x b, ld b).
-template <int CPW, int S>
-SBR_DEV void cta_qr(float (&x)[CPW][S], int rows, int b, float* Vs, float* Rs, float* taus) {
-  constexpr int NW = 32, RS = 32 * S;
+constexpr int P_NW = 32;   // warps per CTA (one column per warp for b <= 32)
+constexpr int P_SL = 8;    // leaf rows per lane  (256-row leaves)
+constexpr int P_SN = 16;   // inner-node rows per lane (512-row nodes)
+
+SBR_DEV int64_t gtimer() {
+  int64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+#define PTRACE(k) \
+  if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[k] = gtimer();
+
+// Householder QR of a register-resident node (rows x b, rows <= 32*S): warp w owns columns
+// w, w+NW, .. (slot j), lane l owns rows l, l+32, .. (slot s).  Reflector jc (unit diagonal,
+// zeros above) goes to Vs[:, jc] (ld 32*S), tau to taus[jc], R (b x b, ld b) to Rs.
+// Reflector of column jc from alpha = x[jc] and sig2 = ||x[jc+1:]||^2 (dlarfg), written to
+// Vs[:, jc], Rs[:, jc] and taus[jc] by the owning warp (column values in xs[0..S)).
+template <int S, int SM>
+SBR_DEV void make_reflector(const float (&xs)[SM], int jc, int b, float alpha, float sig2, float* Vs, float* Rs,
+                            float* taus) {
+  constexpr int RS = 32 * S;
+  const int lane = lane_id();
+  float beta, tau, scal;
+  if (sig2 <= 0.f) {               // dlarfg: x(2:) == 0 -> H = I
+    beta = alpha; tau = 0.f; scal = 0.f;
+  } else {
+    const float nrm = sqrtf(fmaf(alpha, alpha, sig2));
+    beta = alpha >= 0.f ? -nrm : nrm;
+    tau = __fdividef(beta - alpha, beta);
+    scal = __frcp_rn(alpha - beta);
+  }
+#pragma unroll
+  for (int s = 0; s < S; ++s) {
+    const int i = lane + 32 * s;
+    Vs[i + jc * RS] = (i == jc) ? 1.f : (i > jc ? xs[s] * scal : 0.f);
+    if (i < b) Rs[i + jc * b] = (i < jc) ? xs[s] : (i == jc ? beta : 0.f);
+  }
+  if (lane == 0) taus[jc] = tau;
+}
+
+// alpha = x[jc], sig2 = sum_{i > jc} x_i^2 by a plain warp reduction
+template <int S, int SM>
+SBR_DEV void col_norm(const float (&xs)[SM], int jc, float& alpha, float& sig2) {
+  const int lane = lane_id();
+  float a_own = 0.f, s2 = 0.f;
+#pragma unroll
+  for (int s = 0; s < S; ++s) {
+    const int i = lane + 32 * s;
+    if (i == jc) a_own = xs[s];
+    if (i > jc) s2 = fmaf(xs[s], xs[s], s2);
+  }
+  alpha = __shfl_sync(0xffffffffu, a_own, jc & 31);
+  sig2 = warp_sum(s2);
+}
+
+// Householder QR of a register-resident node (rows x b, rows <= 32*S): warp w owns columns
+// w, w+NW, .. (slot j), lane l owns rows l, l+32, .. (slot s).  Reflector jc (unit diagonal,
+// zeros above) goes to Vs[:, jc] (ld 32*S), tau to taus[jc], R (b x b, ld b) to Rs.
+// The warp owning column jc+1 fuses, into the single reduction of its update with
+// reflector jc, the sums it needs for reflector jc+1 (norm downdate
+//   ||x - d v||^2 = xx - 2 d xv + d^2 vv  over rows > jc+1),
+// and recomputes the norm directly when the downdate cancels (< 1/64 of xx).
+template <int CPW, int S, int SM>
+SBR_DEV void cta_qr(float (&x)[CPW][SM], int rows, int b, float* Vs, float* Rs, float* taus,
+                    long long* dbg = nullptr) {
+  constexpr int RS = 32 * S;
   const int lane = lane_id(), warp = warp_id();
   const int kr = min(rows, b);
+  const int wmax = warp + (CPW - 1) * P_NW;  // this warp's last column
+  if (warp == 0 && kr > 0) {
+    float alpha, sig2;
+    col_norm<S, SM>(x[0], 0, alpha, sig2);
+    make_reflector<S, SM>(x[0], 0, b, alpha, sig2, Vs, Rs, taus);
+  }
+  long long t_a = 0, t_b = 0, t_c = 0, t_d = 0;
   for (int jc = 0; jc < kr; ++jc) {
-    const int ow = jc % NW, oslot = jc / NW;
-    if (warp == ow) {
-#pragma unroll
-      for (int j = 0; j < CPW; ++j) {
-        if (j != oslot) continue;
-        float a_l = 0.f, s2 = 0.f;
-#pragma unroll
-        for (int s = 0; s < S; ++s) {
-          const int i = lane + 32 * s;
-          const float v = x[j][s];
-          if (i == jc) a_l = v;
-          else if (i > jc) s2 = fmaf(v, v, s2);
-        }
-        const float alpha = warp_sum(a_l);
-        const float sig2 = warp_sum(s2);
-        float beta, tau, scal;
-        if (sig2 == 0.f) {            // dlarfg: x(2:) == 0 -> H = I
-          beta = alpha; tau = 0.f; scal = 0.f;
-        } else {
-          const float nrm = sqrtf(fmaf(alpha, alpha, sig2));
-          beta = alpha >= 0.f ? -nrm : nrm;
-          tau = (beta - alpha) / beta;
-          scal = 1.f / (alpha - beta);
-        }
-#pragma unroll
-        for (int s = 0; s < S; ++s) {
-          const int i = lane + 32 * s;
-          const float v = (i == jc) ? 1.f : (i > jc ? x[j][s] * scal : 0.f);
-          Vs[i + jc * RS] = v;
-          if (i < b) Rs[i + jc * b] = (i < jc) ? x[j][s] : (i == jc ? beta : 0.f);
-        }
-        if (lane == 0) taus[jc] = tau;
-      }
-    }
-    __syncthreads();
+    const long long c0 = clock64();
+    __syncthreads();                                  // reflector jc published
+    const long long c1 = clock64();
     const float tau = taus[jc];
-    if (tau != 0.f) {
+    if (wmax <= jc) continue;
+    float v[S];
 #pragma unroll
-      for (int j = 0; j < CPW; ++j) {
-        const int c = warp + j * NW;
-        if (c > jc && c < b) {
-          float d = 0.f;
+    for (int s = 0; s < S; ++s) v[s] = Vs[lane + 32 * s + jc * RS];
 #pragma unroll
-          for (int s = 0; s < S; ++s) d = fmaf(Vs[lane + 32 * s + jc * RS], x[j][s], d);
-          d = warp_sum(d) * tau;
+    for (int j = 0; j < CPW; ++j) {
+      const int c = warp + j * P_NW;
+      if (c <= jc || c >= b) continue;
+      const int nx = jc + 1;
+      if (c == nx && nx < kr) {                       // next owner: fused reduction
+        t_a += c1 - c0;
+        float d0 = 0.f, xx = 0.f, xv = 0.f, vv = 0.f, xo = 0.f, vo = 0.f;
 #pragma unroll
-          for (int s = 0; s < S; ++s) x[j][s] = fmaf(-d, Vs[lane + 32 * s + jc * RS], x[j][s]);
+        for (int s = 0; s < S; ++s) {
+          const int i = lane + 32 * s;
+          d0 = fmaf(v[s], x[j][s], d0);
+          if (i > nx) {
+            xx = fmaf(x[j][s], x[j][s], xx);
+            xv = fmaf(x[j][s], v[s], xv);
+            vv = fmaf(v[s], v[s], vv);
+          }
+          if (i == nx) { xo = x[j][s]; vo = v[s]; }
         }
+        const long long c2 = clock64();
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) {
+          d0 += __shfl_xor_sync(0xffffffffu, d0, o);
+          xx += __shfl_xor_sync(0xffffffffu, xx, o);
+          xv += __shfl_xor_sync(0xffffffffu, xv, o);
+          vv += __shfl_xor_sync(0xffffffffu, vv, o);
+        }
+        const long long c3 = clock64();
+        t_b += c2 - c1;
+        t_c += c3 - c2;
+        const float d = d0 * tau;
+#pragma unroll
+        for (int s = 0; s < S; ++s) x[j][s] = fmaf(-d, v[s], x[j][s]);
+        const float xo_b = __shfl_sync(0xffffffffu, xo, nx & 31);
+        const float vo_b = __shfl_sync(0xffffffffu, vo, nx & 31);
+        const float alpha = fmaf(-d, vo_b, xo_b);
+        float sig2 = fmaf(d * d, vv, fmaf(-2.f * d, xv, xx));
+        if (!(sig2 > xx * (1.f / 64.f))) {            // cancellation: recompute directly
+          float a2;
+          col_norm<S, SM>(x[j], nx, a2, sig2);
+        }
+        make_reflector<S, SM>(x[j], nx, b, alpha, sig2, Vs, Rs, taus);
+        t_d += clock64() - c3;
+      } else if (tau != 0.f) {
+        float d0 = 0.f, d1 = 0.f;
+#pragma unroll
+        for (int s = 0; s < S; s += 2) {
+          d0 = fmaf(v[s], x[j][s], d0);
+          if (s + 1 < S) d1 = fmaf(v[s + 1], x[j][s + 1], d1);
+        }
+        const float d = warp_sum(d0 + d1) * tau;
+#pragma unroll
+        for (int s = 0; s < S; ++s) x[j][s] = fmaf(-d, v[s], x[j][s]);
       }
     }
   }
-  // wide node (rows < b): the remaining columns are all R
 #pragma unroll
-  for (int j = 0; j < CPW; ++j) {
-    const int c = warp + j * NW;
+  if (dbg && lane == 0 && blockIdx.x == 0) {
+    atomicAdd((unsigned long long*)&dbg[0], (unsigned long long)t_a);
+    atomicAdd((unsigned long long*)&dbg[1], (unsigned long long)t_b);
+    atomicAdd((unsigned long long*)&dbg[2], (unsigned long long)t_c);
+    atomicAdd((unsigned long long*)&dbg[3], (unsigned long long)t_d);
+  }
+  for (int j = 0; j < CPW; ++j) {  // wide node (rows < b): the remaining columns are all R
+    const int c = warp + j * P_NW;
     if (c >= kr && c < b) {
 #pragma unroll
       for (int s = 0; s < S; ++s) {
@@ -103,32 +188,37 @@ SBR_DEV void cta_qr(float (&x)[CPW][S], int rows, int b, float* Vs, float* Rs, f
       }
     }
   }
-  for (int e = threadIdx.x; e < RS * b; e += blockDim.x) {
-    const int c = e / RS;
-    if (c >= kr) Vs[e] = 0.f;
-  }
+  for (int e = threadIdx.x; e < RS * b; e += blockDim.x)
+    if (e / RS >= kr) Vs[e] = 0.f;
   if (threadIdx.x < b && threadIdx.x >= kr) taus[threadIdx.x] = 0.f;
   __syncthreads();
 }
 
-// x <- H_1 ... H_kr x   (explicit-Q formation, reflectors read from smem).
-template <int CPW, int S>
-SBR_DEV void cta_apply_q(float (&x)[CPW][S], int kr, int b, const float* Vs, const float* taus) {
-  constexpr int NW = 32, RS = 32 * S;
+// x <- H_1 ... H_kr x   (explicit-Q formation; reflectors read from smem, no barriers).
+template <int CPW, int S, int SM>
+SBR_DEV void cta_apply_q(float (&x)[CPW][SM], int kr, int b, const float* Vs, const float* taus) {
+  constexpr int RS = 32 * S;
   const int lane = lane_id(), warp = warp_id();
+  if (warp >= b) return;
   for (int jc = kr - 1; jc >= 0; --jc) {
     const float tau = taus[jc];
     if (tau == 0.f) continue;
+    float v[S];
+#pragma unroll
+    for (int s = 0; s < S; ++s) v[s] = Vs[lane + 32 * s + jc * RS];
 #pragma unroll
     for (int j = 0; j < CPW; ++j) {
-      const int c = warp + j * NW;
+      const int c = warp + j * P_NW;
       if (c < b) {
-        float d = 0.f;
+        float d0 = 0.f, d1 = 0.f;
 #pragma unroll
-        for (int s = 0; s < S; ++s) d = fmaf(Vs[lane + 32 * s + jc * RS], x[j][s], d);
-        d = warp_sum(d) * tau;
+        for (int s = 0; s < S; s += 2) {
+          d0 = fmaf(v[s], x[j][s], d0);
+          if (s + 1 < S) d1 = fmaf(v[s + 1], x[j][s + 1], d1);
+        }
+        const float d = warp_sum(d0 + d1) * tau;
 #pragma unroll
-        for (int s = 0; s < S; ++s) x[j][s] = fmaf(-d, Vs[lane + 32 * s + jc * RS], x[j][s]);
+        for (int s = 0; s < S; ++s) x[j][s] = fmaf(-d, v[s], x[j][s]);
       }
     }
   }
@@ -159,88 +249,184 @@ SBR_DEV float* node_v(const PanelArgs& a, int lev, int k, const NodeInfo& ni) {
   return a.ws_v + a.voff[lev] + (lev == 0 ? ni.start * a.b : (int64_t)k * a.arity * a.b * a.b);
 }
 
-template <int B, int CPW, int S>
-__global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
-  constexpr int NW = 32, RS = 32 * S;
+template <int CPW, int S, int SM>
+SBR_DEV void load_node(const PanelArgs& a, int lev, int k, const NodeInfo& ni, float (&x)[CPW][SM]) {
+  const int lane = lane_id(), warp = warp_id(), b = a.b;
+#pragma unroll
+  for (int j = 0; j < CPW; ++j) {
+    const int c = warp + j * P_NW;
+#pragma unroll
+    for (int s = 0; s < SM; ++s) {
+      const int i = lane + 32 * s;
+      float v = 0.f;
+      if (s < S && c < b && i < ni.rows) {
+        if (lev == 0) {
+          v = a.P[(ni.start + i) + (int64_t)c * a.ldp];
+        } else {
+          const int ch = k * a.arity + i / b, ii = i % b;
+          v = a.ws_r[a.roff[lev - 1] + (int64_t)ch * b * b + ii + c * b];
+        }
+      }
+      x[j][s] = v;
+    }
+  }
+}
+
+template <int S>
+SBR_DEV void store_v(const PanelArgs& a, int lev, int k, const NodeInfo& ni, const float* Vs, const float* taus,
+                     const float* Rs) {
+  constexpr int RS = 32 * S;
+  const int b = a.b;
+  float* vd = node_v(a, lev, k, ni);
+  for (int e = threadIdx.x; e < ni.rows * b; e += blockDim.x) vd[e] = Vs[(e % ni.rows) + (e / ni.rows) * RS];
+  if (threadIdx.x < b) a.ws_tau[a.toff[lev] + (int64_t)k * b + threadIdx.x] = taus[threadIdx.x];
+  for (int e = threadIdx.x; e < b * b; e += blockDim.x) a.ws_r[a.roff[lev] + (int64_t)k * b * b + e] = Rs[e];
+}
+
+// x = [C; 0] with C = the node's b x b block of its parent's explicit Q (or I at the root)
+template <int CPW, int SM>
+SBR_DEV void load_c(const PanelArgs& a, int lev, int k, float (&x)[CPW][SM]) {
+  const int lane = lane_id(), warp = warp_id(), b = a.b;
+  const float* cpar = nullptr;
+  int ldc = 0;
+  if (lev < a.nlev - 1) {
+    const int parent = k / a.arity, idx = k % a.arity;
+    const NodeInfo pi = node_info(a, lev + 1, parent);
+    cpar = a.ws_q + a.qoff[lev + 1] + (int64_t)parent * a.arity * b * b + idx * b;
+    ldc = pi.rows;
+  }
+#pragma unroll
+  for (int j = 0; j < CPW; ++j) {
+    const int c = warp + j * P_NW;
+#pragma unroll
+    for (int s = 0; s < SM; ++s) {
+      const int i = lane + 32 * s;
+      float v = 0.f;
+      if (c < b && i < b) v = cpar ? cpar[i + (int64_t)c * ldc] : (i == c ? 1.f : 0.f);
+      x[j][s] = v;
+    }
+  }
+}
+
+template <int CPW, int S, int SM>
+SBR_DEV void store_q_ws(const PanelArgs& a, int lev, int k, const NodeInfo& ni, const float (&x)[CPW][SM]) {
+  const int lane = lane_id(), warp = warp_id(), b = a.b;
+#pragma unroll
+  for (int j = 0; j < CPW; ++j) {
+    const int c = warp + j * P_NW;
+#pragma unroll
+    for (int s = 0; s < S; ++s) {
+      const int i = lane + 32 * s;
+      if (c < b && i < ni.rows) a.ws_q[a.qoff[lev] + (int64_t)k * a.arity * b * b + i + (int64_t)c * ni.rows] = x[j][s];
+    }
+  }
+}
+
+template <int S>
+SBR_DEV void stage_v(const PanelArgs& a, int lev, int k, const NodeInfo& ni, float* Vs, float* taus) {
+  constexpr int RS = 32 * S;
+  const int b = a.b;
+  const float* vs = node_v(a, lev, k, ni);
+  for (int e = threadIdx.x; e < RS * b; e += blockDim.x) {   // rows >= ni.rows must read 0
+    const int i = e % RS, c = e / RS;
+    Vs[e] = (i < ni.rows) ? vs[i + c * ni.rows] : 0.f;
+  }
+  if (threadIdx.x < b) taus[threadIdx.x] = a.ws_tau[a.toff[lev] + (int64_t)k * b + threadIdx.x];
+  __syncthreads();
+}
+
+// modified LU of Q_1 - S (s_j = -sign(d_j)), one warp, lane c holds column c in
+// registers (b <= 32).  Writes U (upper, incl. diagonal) and L (unit lower) to Us / Ls.
+template <int LDU>
+SBR_DEV void warp_lu32(int b, const float* Q1, int ldq, float* Us, float* Ls, float* Ss) {
+  const int lane = lane_id();
+  float col[32];
+#pragma unroll
+  for (int i = 0; i < 32; ++i) col[i] = (lane < b && i < b) ? Q1[i + lane * ldq] : 0.f;
+  float sgn = 0.f;
+#pragma unroll
+  for (int j = 0; j < 32; ++j) {
+    if (j < b) {
+      const float d = __shfl_sync(0xffffffffu, col[j], j);
+      const float sj = (d >= 0.f) ? -1.f : 1.f;   // s_j = -sign(d_j)
+      const float piv = d - sj;
+      if (lane == j) { col[j] = piv; sgn = sj; }
+      const float inv = 1.f / piv;
+      if (lane == j) {
+#pragma unroll
+        for (int i = j + 1; i < 32; ++i) col[i] *= inv;
+      }
+      // broadcast L[:, j] (rows > j) and update columns c > j
+#pragma unroll
+      for (int i = j + 1; i < 32; ++i) {
+        const float lij = __shfl_sync(0xffffffffu, col[i], j);
+        if (lane > j) col[i] = fmaf(-lij, col[j], col[i]);
+      }
+    }
+  }
+  if (lane < b) {
+#pragma unroll
+    for (int i = 0; i < 32; ++i) {
+      if (i < b) {
+        Us[i + lane * LDU] = (i <= lane) ? col[i] : 0.f;
+        Ls[i + lane * LDU] = (i > lane) ? col[i] : (i == lane ? 1.f : 0.f);
+      }
+    }
+    Ss[lane] = sgn;
+  }
+}
+
+template <int B, int CPW>
+__global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
+  constexpr int RSL = 32 * P_SL, RSN = 32 * P_SN;
+  constexpr int LDU = B + 1;                 // padded ld for the b x b factors
   extern __shared__ __align__(16) float smem[];
-  float* Vs = smem;               // RS x B
-  float* Rs = Vs + RS * B;        // B x B
-  float* taus = Rs + B * B;       // B (padded to 64)
-  float* Us = taus + 64;          // B x B  (LU's U; later kept for the row solves)
-  float* Ts = Us + B * B;         // B x B  (T)
-  float* Ls = Ts + B * B;         // B x B  (L1, then scratch)
-  float* Ss = Ls + B * B;         // B      (signs)
+  float* Vs = smem;                          // RSN x B (reflectors; later the leaf's explicit Q)
+  float* Rs = Vs + RSN * B;                  // B x B
+  float* taus = Rs + B * B;                  // 64
+  float* Us = taus + 64;                     // B x LDU : U (upper) / LU work
+  float* Ls = Us + B * LDU;                  // B x LDU : L_1 (unit lower) ; T in the single-leaf path
+  float* Ss = Ls + B * LDU;                  // B signs
   const int b = a.b;
   const int lane = lane_id(), warp = warp_id();
   cg::grid_group grid = cg::this_grid();
-  float x[CPW][S];
+  if (a.run_if && *a.run_if == 0) return;    // CholeskyQR already factored this panel
+  float x[CPW][P_SN];
+  PTRACE(0);
+  if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[10] = clock64();
+  const int64_t M = a.M, row0 = a.row0;
 
-  // ---------------- up sweep ----------------
-  for (int lev = 0; lev < a.nlev; ++lev) {
-    for (int k = blockIdx.x; k < a.nodes[lev]; k += gridDim.x) {
-      const NodeInfo ni = node_info(a, lev, k);
-#pragma unroll
-      for (int j = 0; j < CPW; ++j) {
-        const int c = warp + j * NW;
-#pragma unroll
-        for (int s = 0; s < S; ++s) {
-          const int i = lane + 32 * s;
-          float v = 0.f;
-          if (c < b && i < ni.rows) {
-            if (lev == 0) {
-              v = a.P[(ni.start + i) + (int64_t)c * a.ldp];
-            } else {
-              const int ch = k * a.arity + i / b, ii = i % b;
-              v = a.ws_r[a.roff[lev - 1] + (int64_t)ch * b * b + ii + c * b];
-            }
-          }
-          x[j][s] = v;
-        }
-      }
-      cta_qr<CPW, S>(x, ni.rows, b, Vs, Rs, taus);
-      if (a.nlev == 1) break;  // single leaf: keep V, R, tau in smem
-      float* vd = node_v(a, lev, k, ni);
-      for (int e = threadIdx.x; e < ni.rows * b; e += blockDim.x) {
-        const int i = e % ni.rows, c = e / ni.rows;
-        vd[e] = Vs[i + c * RS];
-      }
-      if (threadIdx.x < b) a.ws_tau[a.toff[lev] + (int64_t)k * b + threadIdx.x] = taus[threadIdx.x];
-      for (int e = threadIdx.x; e < b * b; e += blockDim.x) a.ws_r[a.roff[lev] + (int64_t)k * b * b + e] = Rs[e];
-      __syncthreads();
-    }
-    if (a.nlev > 1) grid.sync();
-  }
-
-  const int64_t M = a.M;
-  const int64_t row0 = a.row0;
+  // ================= single node: LAPACK-exact V, T (dlarft), R; W = V T =================
   if (a.nlev == 1) {
-    // --------- single leaf: LAPACK-exact V, T (dlarft), R ---------
+    const NodeInfo ni = node_info(a, 0, 0);
+    load_node<CPW, P_SN, P_SN>(a, 0, 0, ni, x);
+    cta_qr<CPW, P_SN, P_SN>(x, ni.rows, b, Vs, Rs, taus);
     const int rows = a.m, kr = min(rows, b);
-    // T[0:j, j] = -tau_j T[0:j,0:j] (V^T v_j)[0:j]; first G[p][j] = v_p . v_j (p < j) by warps
-    for (int pair = warp; pair < b * b; pair += NW) {
+    float* G = Us;  // G[p][j] = v_p . v_j, p < j
+    for (int pair = warp; pair < b * b; pair += P_NW) {
       const int p = pair % b, j = pair / b;
       if (p >= j) continue;
       float d = 0.f;
-      for (int i = lane; i < rows; i += 32) d = fmaf(Vs[i + p * RS], Vs[i + j * RS], d);
+      for (int i = lane; i < rows; i += 32) d = fmaf(Vs[i + p * RSN], Vs[i + j * RSN], d);
       d = warp_sum(d);
-      if (lane == 0) Ls[p + j * B] = d;
+      if (lane == 0) G[p + j * LDU] = d;
     }
     __syncthreads();
-    for (int j = 0; j < b; ++j) {     // dlarft recurrence, one column per step
+    float* T = Ls;
+    for (int j = 0; j < b; ++j) {  // dlarft recurrence: T[0:j, j] = -tau_j T[0:j,0:j] G[0:j, j]
       const float tj = (j < kr) ? taus[j] : 0.f;
       if (threadIdx.x < b) {
         const int p = threadIdx.x;
         float val = (p == j) ? tj : 0.f;
         if (p < j) {
           float acc = 0.f;
-          for (int q = p; q < j; ++q) acc = fmaf(Ts[p + q * B], Ls[q + j * B], acc);
+          for (int q = p; q < j; ++q) acc = fmaf(T[p + q * LDU], G[q + j * LDU], acc);
           val = -tj * acc;
         }
-        Ts[p + j * B] = val;
+        T[p + j * LDU] = val;
       }
       __syncthreads();
     }
-    // rows: y = v, w = y T; compact panel: strictly lower = v, upper = R
     for (int64_t i = threadIdx.x; i < M; i += blockDim.x) {
       if (i < row0) {
         for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
@@ -249,200 +435,203 @@ __global__ void __launch_bounds__(1024, 1) panel_tsqr_kernel(PanelArgs a) {
       }
       const int64_t il = i - row0;
       for (int c = 0; c < b; ++c) {
-        const float y = Vs[il + c * RS];
+        const float y = Vs[il + c * RSN];
         a.Y[i + c * a.ldy] = y;
         if (a.Yh) a.Yh[i * a.ldyh + c] = __float2half_rn(y);
         a.P[il + c * a.ldp] = (il > c) ? y : (il < b ? Rs[il + c * b] : 0.f);
         float w = 0.f;
-        for (int k = 0; k <= c; ++k) w = fmaf(Vs[il + k * RS], Ts[k + c * B], w);
+        for (int k = 0; k <= c; ++k) w = fmaf(Vs[il + k * RSN], T[k + c * LDU], w);
         a.W[i + c * a.ldw] = w;
       }
     }
     return;
   }
 
-  // ---------------- down sweep: explicit Q ----------------
-  for (int lev = a.nlev - 1; lev >= 0; --lev) {
-    for (int k = blockIdx.x; k < a.nodes[lev]; k += gridDim.x) {
+  // ================= up sweep =================
+  const int top = a.nlev - 1;
+  for (int lev = 0; lev < top; ++lev) {
+    const int k = blockIdx.x;
+    if (k < a.nodes[lev]) {
       const NodeInfo ni = node_info(a, lev, k);
-      const float* vs = node_v(a, lev, k, ni);
-      for (int e = threadIdx.x; e < RS * b; e += blockDim.x) {   // rows >= ni.rows must read 0
-        const int i = e % RS, c = e / RS;
-        Vs[e] = (i < ni.rows) ? vs[i + c * ni.rows] : 0.f;
+      if (lev == 0) {
+        load_node<CPW, P_SL, P_SN>(a, lev, k, ni, x);
+        cta_qr<CPW, P_SL, P_SN>(x, ni.rows, b, Vs, Rs, taus, a.trace ? (long long*)(a.trace + 12) : nullptr);
+        PTRACE(1);
+        if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) a.trace[11] = clock64();
+        store_v<P_SL>(a, lev, k, ni, Vs, taus, Rs);
+      } else {
+        load_node<CPW, P_SN, P_SN>(a, lev, k, ni, x);
+        cta_qr<CPW, P_SN, P_SN>(x, ni.rows, b, Vs, Rs, taus);
+        store_v<P_SN>(a, lev, k, ni, Vs, taus, Rs);
       }
-      if (threadIdx.x < b) taus[threadIdx.x] = a.ws_tau[a.toff[lev] + (int64_t)k * b + threadIdx.x];
-      __syncthreads();
-      const float* cpar = nullptr;
-      int ldc = 0;
-      if (lev < a.nlev - 1) {
-        const int parent = k / a.arity, idx = k % a.arity;
-        const NodeInfo pi = node_info(a, lev + 1, parent);
-        cpar = a.ws_q + a.qoff[lev + 1] + (int64_t)parent * a.arity * b * b + idx * b;
-        ldc = pi.rows;
-      }
-#pragma unroll
-      for (int j = 0; j < CPW; ++j) {
-        const int c = warp + j * NW;
-#pragma unroll
-        for (int s = 0; s < S; ++s) {
-          const int i = lane + 32 * s;
-          float v = 0.f;
-          if (c < b && i < b) v = cpar ? cpar[i + (int64_t)c * ldc] : (i == c ? 1.f : 0.f);
-          x[j][s] = v;
-        }
-      }
-      cta_apply_q<CPW, S>(x, min(ni.rows, b), b, Vs, taus);
-#pragma unroll
-      for (int j = 0; j < CPW; ++j) {
-        const int c = warp + j * NW;
-#pragma unroll
-        for (int s = 0; s < S; ++s) {
-          const int i = lane + 32 * s;
-          if (c < b && i < ni.rows) {
-            if (lev == 0) a.P[(ni.start + i) + (int64_t)c * a.ldp] = x[j][s];
-            else a.ws_q[a.qoff[lev] + (int64_t)k * a.arity * b * b + i + (int64_t)c * ni.rows] = x[j][s];
-          }
-        }
-      }
-      __syncthreads();
+    }
+    grid.sync();
+    if (lev == 0) PTRACE(2);
+  }
+  // root: QR and explicit Q = H_root [I; 0] in the same CTA
+  if (blockIdx.x == 0) {
+    const NodeInfo ni = node_info(a, top, 0);
+    load_node<CPW, P_SN, P_SN>(a, top, 0, ni, x);
+    cta_qr<CPW, P_SN, P_SN>(x, ni.rows, b, Vs, Rs, taus);
+    PTRACE(3);
+    for (int e = threadIdx.x; e < b * b; e += blockDim.x) a.ws_r[a.roff[top] + e] = Rs[e];
+    load_c<CPW, P_SN>(a, top, 0, x);
+    cta_apply_q<CPW, P_SN, P_SN>(x, min(ni.rows, b), b, Vs, taus);
+    store_q_ws<CPW, P_SN, P_SN>(a, top, 0, ni, x);
+    PTRACE(4);
+  }
+  grid.sync();
+  PTRACE(5);
+  // ================= down sweep =================
+  for (int lev = top - 1; lev >= 1; --lev) {
+    const int k = blockIdx.x;
+    if (k < a.nodes[lev]) {
+      const NodeInfo ni = node_info(a, lev, k);
+      stage_v<P_SN>(a, lev, k, ni, Vs, taus);
+      load_c<CPW, P_SN>(a, lev, k, x);
+      cta_apply_q<CPW, P_SN, P_SN>(x, min(ni.rows, b), b, Vs, taus);
+      store_q_ws<CPW, P_SN, P_SN>(a, lev, k, ni, x);
     }
     grid.sync();
   }
-
-  // ---------------- reconstruction (Alg. 3 + S) ----------------
-  if (blockIdx.x == 0) {
-    // Q_1 = top b x b of the explicit Q (written by this CTA: leaf 0)
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-      const int i = e % b, c = e / b;
-      Us[i + c * B] = a.P[i + (int64_t)c * a.ldp];
-      Ts[i + c * B] = Us[i + c * B];   // keep Q_1 for W_top
-    }
-    __syncthreads();
-    for (int j = 0; j < b; ++j) {      // non-pivoted LU of Q_1 - S
-      if (threadIdx.x == 0) {
-        const float d = Us[j + j * B];
-        const float sj = (d >= 0.f) ? -1.f : 1.f;   // s_j = -sign(d_j)
-        Ss[j] = sj;
-        Us[j + j * B] = d - sj;
-      }
-      __syncthreads();
-      const float piv = Us[j + j * B];
-      for (int i = j + 1 + threadIdx.x; i < b; i += blockDim.x) Us[i + j * B] /= piv;
-      __syncthreads();
-      const int nt = b - j - 1;
-      for (int e = threadIdx.x; e < nt * nt; e += blockDim.x) {
-        const int i = j + 1 + e % nt, c = j + 1 + e / nt;
-        Us[i + c * B] = fmaf(-Us[i + j * B], Us[j + c * B], Us[i + c * B]);
-      }
-      __syncthreads();
-    }
-    // L1 (unit lower) -> Ls;  L1^-1 by column forward substitution (thread per column) -> scratch in Rs? keep R!
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-      const int i = e % b, c = e / b;
-      Ls[i + c * B] = (i > c) ? Us[i + c * B] : (i == c ? 1.f : 0.f);
-    }
-    __syncthreads();
-    // Linv (lower unit) into Vs scratch (Vs is free now): Linv[:, c] solves L1 x = e_c
-    float* Linv = Vs;
-    if (threadIdx.x < b) {
-      const int c = threadIdx.x;
-      for (int i = 0; i < b; ++i) {
-        float v = (i == c) ? 1.f : 0.f;
-        for (int k = c; k < i; ++k) v = fmaf(-Ls[i + k * B], Linv[k + c * B], v);
-        Linv[i + c * B] = (i < c) ? 0.f : v;
-      }
-    }
-    __syncthreads();
-    // T = -U S L1^-T : T[r][c] = -sum_k U[r][k] s_k Linv[c][k], k in [r, c]
-    float* Tn = Vs + B * B;
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-      const int r = e % b, c = e / b;
-      float acc = 0.f;
-      for (int k = r; k <= c; ++k) acc = fmaf(Us[r + k * B] * Ss[k], Linv[c + k * B], acc);
-      Tn[r + c * B] = (r <= c) ? -acc : 0.f;
-    }
-    __syncthreads();
-    // R = S R_root ; publish U, T for the row solves
-    const float* rroot = a.ws_r + a.roff[a.nlev - 1];
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-      const int i = e % b, c = e / b;
-      a.ws_misc[e] = (i <= c) ? Us[i + c * B] : 0.f;              // U
-      a.ws_misc[b * b + e] = Tn[i + c * B];                          // T
-      // top b rows of the panel: Y_top = L1, W_top = L1 T, compact = L1 (strict) / S R
-      const float rfin = Ss[i] * rroot[i + c * b];
-      a.P[i + (int64_t)c * a.ldp] = (i > c) ? Ls[i + c * B] : rfin;
-      a.Y[(row0 + i) + c * a.ldy] = Ls[i + c * B];
-      if (a.Yh) a.Yh[(row0 + i) * a.ldyh + c] = __float2half_rn(Ls[i + c * B]);
-      float w = 0.f;
-      for (int k = 0; k <= min(i, c); ++k) w = fmaf(Ls[i + k * B], Tn[k + c * B], w);
-      a.W[(row0 + i) + c * a.ldw] = w;
-    }
-  }
-  grid.sync();
-  // rows i >= b of the panel:  y_i U = q_i  ;  w_i = y_i T   (thread per row)
-  for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-    Us[e % b + (e / b) * B] = a.ws_misc[e];
-    Ts[e % b + (e / b) * B] = a.ws_misc[b * b + e];
+  const NodeInfo ni = node_info(a, 0, blockIdx.x);   // this CTA's leaf
+  stage_v<P_SL>(a, 0, blockIdx.x, ni, Vs, taus);
+  load_c<CPW, P_SN>(a, 0, blockIdx.x, x);
+  cta_apply_q<CPW, P_SL, P_SN>(x, min(ni.rows, b), b, Vs, taus);
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < CPW; ++j) {   // leaf: keep Q in smem (Vs, ld RSL) for the row phase
+    const int c = warp + j * P_NW;
+#pragma unroll
+    for (int s = 0; s < P_SL; ++s)
+      if (c < b) Vs[lane + 32 * s + c * RSL] = x[j][s];
   }
   __syncthreads();
+  PTRACE(6);
+  // ================= reconstruction: modified LU of Q_1 - S (CTA 0) =================
+  if (blockIdx.x == 0) {
+    if (B <= 32) {
+      if (warp == 0) warp_lu32<LDU>(b, Vs, RSL, Us, Ls, Ss);
+    } else if (warp == 0) {            // b > 32: column-per-lane LU through shared memory
+      for (int e = lane; e < b * b; e += 32) Us[(e % b) + (e / b) * LDU] = Vs[(e % b) + (e / b) * RSL];
+      __syncwarp();
+      for (int j = 0; j < b; ++j) {
+        const float d = Us[j + j * LDU];
+        const float sj = (d >= 0.f) ? -1.f : 1.f;
+        const float piv = d - sj;
+        __syncwarp();
+        if (lane == 0) { Us[j + j * LDU] = piv; Ss[j] = sj; }
+        for (int i = j + 1 + lane; i < b; i += 32) Us[i + j * LDU] /= piv;
+        __syncwarp();
+        for (int c = j + 1 + lane; c < b; c += 32) {
+          const float ujc = Us[j + c * LDU];
+          for (int i = j + 1; i < b; ++i) Us[i + c * LDU] = fmaf(-Us[i + j * LDU], ujc, Us[i + c * LDU]);
+        }
+        __syncwarp();
+      }
+      for (int e = lane; e < b * b; e += 32) {
+        const int i = e % b, c = e / b;
+        Ls[i + c * LDU] = (i > c) ? Us[i + c * LDU] : (i == c ? 1.f : 0.f);
+        if (i > c) Us[i + c * LDU] = 0.f;
+      }
+    }
+    __syncthreads();
+    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
+      const int i = e % b, c = e / b;
+      a.ws_misc[e] = Us[i + c * LDU];
+      a.ws_misc[b * b + e] = Ls[i + c * LDU];
+    }
+    if (threadIdx.x < b) a.ws_misc[2 * b * b + threadIdx.x] = Ss[threadIdx.x];
+  }
+  PTRACE(7);
+  grid.sync();
+  PTRACE(8);
+  // ================= rows of this leaf: y U = q (rows >= b), w L^T = (E - q S) =================
+  if (blockIdx.x != 0) {
+    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
+      const int i = e % b, c = e / b;
+      Us[i + c * LDU] = a.ws_misc[e];
+      Ls[i + c * LDU] = a.ws_misc[b * b + e];
+    }
+    if (threadIdx.x < b) Ss[threadIdx.x] = a.ws_misc[2 * b * b + threadIdx.x];
+    __syncthreads();
+  }
+  const float* rroot = a.ws_r + a.roff[top];
+  for (int il_local = threadIdx.x; il_local < ni.rows; il_local += blockDim.x) {
+    const int64_t il = ni.start + il_local;           // panel row
+    const int64_t gr = row0 + il;
+    const float* qrow = Vs + il_local;                 // q_c = qrow[c * RSL]
+    float v_[B];
+    // w L_1^T = (e_il if il < b) - q S   (forward substitution, L_1 unit lower)
+#pragma unroll
+    for (int c = 0; c < B; ++c) {
+      if (c < b) {
+        float v = ((il == c) ? 1.f : 0.f) - qrow[c * RSL] * Ss[c];
+#pragma unroll
+        for (int k = 0; k < c; ++k) v = fmaf(-v_[k], Ls[c + k * LDU], v);
+        v_[c] = v;
+      } else {
+        v_[c] = 0.f;
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < B; ++c)
+      if (c < b) a.W[gr + c * a.ldw] = v_[c];
+    // y = L_1 row (il < b)  or  y U = q
+#pragma unroll
+    for (int c = 0; c < B; ++c) {
+      if (c < b) {
+        if (il < b) {
+          v_[c] = Ls[il + c * LDU];
+        } else {
+          float v = qrow[c * RSL];
+#pragma unroll
+          for (int k = 0; k < c; ++k) v = fmaf(-v_[k], Us[k + c * LDU], v);
+          v_[c] = v / Us[c + c * LDU];
+        }
+      } else {
+        v_[c] = 0.f;
+      }
+    }
+#pragma unroll
+    for (int c = 0; c < B; ++c) {
+      if (c < b) {
+        a.Y[gr + c * a.ldy] = v_[c];
+        a.P[il + (int64_t)c * a.ldp] = (il > c) ? v_[c] : (Ss[il] * rroot[il + c * b]);   // il < b here
+        if (a.Yh) a.Yh[gr * a.ldyh + c] = __float2half_rn(v_[c]);
+      }
+    }
+  }
+  // rows above the panel: zero Y and W (and Yh)
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t nth = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = tid; i < row0; i += nth) {
     for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
     if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
   }
-  for (int64_t il = b + tid; il < a.m; il += nth) {
-    float q[B];
-#pragma unroll
-    for (int c = 0; c < B; ++c) q[c] = (c < b) ? a.P[il + (int64_t)c * a.ldp] : 0.f;
-#pragma unroll
-    for (int c = 0; c < B; ++c) {
-      if (c < b) {
-        float v = q[c];
-#pragma unroll
-        for (int k = 0; k < c; ++k) v = fmaf(-q[k], Us[k + c * B], v);
-        q[c] = v / Us[c + c * B];
-      }
-    }
-#pragma unroll
-    for (int c = 0; c < B; ++c) {
-      if (c < b) {
-        a.P[il + (int64_t)c * a.ldp] = q[c];
-        a.Y[(row0 + il) + c * a.ldy] = q[c];
-        if (a.Yh) a.Yh[(row0 + il) * a.ldyh + c] = __float2half_rn(q[c]);
-      }
-    }
-#pragma unroll
-    for (int c = B - 1; c >= 0; --c) {
-      if (c < b) {
-        float w = 0.f;
-#pragma unroll
-        for (int k = 0; k <= c; ++k) w = fmaf(q[k], Ts[k + c * B], w);
-        q[c] = w;
-      }
-    }
-#pragma unroll
-    for (int c = 0; c < B; ++c)
-      if (c < b) a.W[(row0 + il) + c * a.ldw] = q[c];
-  }
+  PTRACE(9);
 }
 
 // ---------------------------------------------------------------- host side
-template <int B, int CPW, int S>
+template <int B>
+static constexpr size_t panel_smem() {
+  return sizeof(float) * (32 * P_SN * B + B * B + 64 + 2 * B * (B + 1) + B);
+}
+
+template <int B, int CPW>
 static cudaError_t launch_panel_t(PanelArgs& a, int max_ctas, cudaStream_t st) {
-  constexpr int RS = 32 * S;
-  const size_t smem = sizeof(float) * (RS * B + B * B + 64 + 4 * B * B + B);
-  auto kern = panel_tsqr_kernel<B, CPW, S>;
+  constexpr size_t smem = panel_smem<B>();
+  auto kern = panel_tsqr_kernel<B, CPW>;
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  // tree shape
-  const int cap = RS;
-  int L = (a.m <= cap) ? 1 : (a.m + cap - 1) / cap;
-  a.arity = max(2, cap / a.b);
+  constexpr int capN = 32 * P_SN, capL = 32 * P_SL;
+  const int L = (a.m <= capN) ? 1 : (a.m + capL - 1) / capL;   // 1: single node, direct QR
+  if (L > max_ctas) return cudaErrorInvalidValue;  // one CTA per leaf must be co-resident
+  a.arity = std::max(2, capN / a.b);
   a.nlev = 0;
   int nodes = L;
   int64_t voff = 0, roff = 0, toff = 0, qoff = 0;
@@ -461,25 +650,22 @@ static cudaError_t launch_panel_t(PanelArgs& a, int max_ctas, cudaStream_t st) {
     nodes = (nodes + a.arity - 1) / a.arity;
     if (a.nlev >= kPanelMaxLev) return cudaErrorInvalidValue;
   }
-  const int grid = (L == 1) ? 1 : min(L, max_ctas);
   void* args[] = {&a};
-  return cudaLaunchCooperativeKernel((const void*)kern, dim3(grid), dim3(1024), args, smem, st);
+  return cudaLaunchCooperativeKernel((const void*)kern, dim3(L), dim3(P_NW * 32), args, smem, st);
 }
 
 cudaError_t launch_panel(PanelArgs& a, int max_ctas, cudaStream_t st) {
-  if (a.b <= 8) return launch_panel_t<8, 1, 16>(a, max_ctas, st);
-  if (a.b <= 16) return launch_panel_t<16, 1, 16>(a, max_ctas, st);
-  if (a.b <= 32) return launch_panel_t<32, 1, 16>(a, max_ctas, st);
-  return launch_panel_t<64, 2, 8>(a, max_ctas, st);
+  if (a.b <= 16) return launch_panel_t<16, 1>(a, max_ctas, st);
+  if (a.b <= 32) return launch_panel_t<32, 1>(a, max_ctas, st);
+  return launch_panel_t<64, 2>(a, max_ctas, st);
 }
 
 PanelWs panel_ws_sizes(int64_t m_max, int b) {
-  // leaves hold >= 256/2 rows, so #nodes over all levels <= 2*(m/128 + 1) + 2
   const int64_t nodes = 2 * (m_max / 128 + 2) + 2;
-  const int64_t arity_rows = 64 * 64 * 2;  // generous: inner node rows x b bound
+  const int64_t node_floats = 512 * 64;  // inner node rows x b bound (rows <= 512)
   PanelWs w;
-  w.v = (size_t)(m_max * b + nodes * arity_rows + 4096);
-  w.q = (size_t)(nodes * arity_rows + 4096);
+  w.v = (size_t)(m_max * b + nodes * node_floats + 4096);
+  w.q = (size_t)(nodes * node_floats + 4096);
   w.r = (size_t)(nodes * b * b + 4096);
   w.tau = (size_t)(nodes * b + 256);
   w.misc = (size_t)(2 * 64 * 64 + 256);
@@ -492,13 +678,12 @@ int panel_max_ctas(int b) {
   cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   const void* k;
   size_t smem;
-  if (b <= 8) { k = (const void*)panel_tsqr_kernel<8, 1, 16>; smem = sizeof(float) * (512 * 8 + 5 * 64 + 64 + 8); }
-  else if (b <= 16) { k = (const void*)panel_tsqr_kernel<16, 1, 16>; smem = sizeof(float) * (512 * 16 + 5 * 256 + 64 + 16); }
-  else if (b <= 32) { k = (const void*)panel_tsqr_kernel<32, 1, 16>; smem = sizeof(float) * (512 * 32 + 5 * 1024 + 64 + 32); }
-  else { k = (const void*)panel_tsqr_kernel<64, 2, 8>; smem = sizeof(float) * (256 * 64 + 5 * 4096 + 64 + 64); }
+  if (b <= 16) { k = (const void*)panel_tsqr_kernel<16, 1>; smem = panel_smem<16>(); }
+  else if (b <= 32) { k = (const void*)panel_tsqr_kernel<32, 1>; smem = panel_smem<32>(); }
+  else { k = (const void*)panel_tsqr_kernel<64, 2>; smem = panel_smem<64>(); }
   cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, 1024, smem);
-  return max(1, per) * nsm;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, P_NW * 32, smem);
+  return std::max(1, per) * nsm;
 }
 
 }  // namespace sbr

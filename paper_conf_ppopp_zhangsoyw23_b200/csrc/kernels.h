@@ -28,6 +28,8 @@ struct PanelArgs {
   float* ws_r;
   float* ws_q;
   float* ws_misc;
+  int64_t* trace;  // optional: CTA 0 phase timestamps (globaltimer ns), 10 entries
+  const int* run_if;  // TSQR only: if non-NULL, do nothing unless *run_if != 0 (CholQR fallback)
   // tree (filled by launch_panel)
   int nlev, arity;
   int nodes[kPanelMaxLev];
@@ -40,6 +42,8 @@ struct PanelWs {
 PanelWs panel_ws_sizes(int64_t m_max, int b);
 cudaError_t launch_panel(PanelArgs& a, int max_ctas, cudaStream_t st);
 int panel_max_ctas(int b);
+// shifted CholeskyQR3 (fp64) + reconstruction; *fail = 1 (panel untouched) if rank deficient
+cudaError_t launch_panel_chol(PanelArgs& a, int max_ctas, double* gram, int* fail, cudaStream_t st);
 
 // ---- SIMT building blocks (fp32) ----
 // C[m1 x n2] (+)= alpha * A[rows x m1]^T B[rows x n2]   (accumulate=1: atomics into C)

@@ -12,6 +12,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -61,6 +62,9 @@ struct sbr_ctx {
   __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr, *Xh = nullptr, *Wrh = nullptr,
          *Bl = nullptr, *Gh = nullptr;
   float* Hb = nullptr;
+  double* gram = nullptr;  // CholeskyQR Gram matrices (3 x 64 x 64)
+  int* pfail = nullptr;
+  int panel_mode = 0;      // 0: CholeskyQR3 + TSQR fallback, 1: TSQR only (SBR_PANEL=tsqr)
   int64_t ldwh = 0, ldsh = 0, ldk = 0, ldbl = 0;
   int panel_ctas = 0;
   // host-buffer (e2e) device copies
@@ -156,7 +160,7 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
-               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64);
+               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take((3 * 8 + 3) * 64 * 64 * 2 + 64);
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
   if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
@@ -199,6 +203,8 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->Bl = (__half*)(base + oBl);
   h->Gh = (__half*)(base + oGh);
   h->Hb = (float*)(base + oHb);
+  h->gram = (double*)(base + oGram);
+  h->pfail = (int*)(h->gram + (3 * 8 + 3) * 64 * 64);
   h->ldbl = 2 * ldk + 128;
   h->ldwh = ldwh;
   h->ldsh = ldsh;
@@ -328,6 +334,15 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.ws_r = h->pr;
         pa.ws_q = h->pq;
         pa.ws_misc = h->pmisc;
+        if (h->panel_mode == 0 && m > 512 && m >= 2 * b) {   // CholeskyQR3, TSQR only if it declines
+          const cudaError_t ce = launch_panel_chol(pa, h->panel_ctas, h->gram, h->pfail, st);
+          if (ce == cudaSuccess) {
+            pa.run_if = h->pfail;
+            h->launches += 1;
+          } else if (ce != cudaErrorNotSupported) {
+            SBR_CK(ce, "panel_chol");
+          }
+        }
         SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
         h->launches += 1;
       }
@@ -512,6 +527,8 @@ int sbr_create(sbr_handle_t* out, int device, void* stream) {
   h->device = device;
   h->stream = (cudaStream_t)stream;
   cudaDeviceGetAttribute(&h->nsm, cudaDevAttrMultiProcessorCount, device);
+  const char* pm = getenv("SBR_PANEL");   // "tsqr": the paper's TSQR panel only (ablation)
+  if (pm && strcmp(pm, "tsqr") == 0) h->panel_mode = 1;
   *out = h;
   return SBR_OK;
 }
@@ -811,3 +828,47 @@ int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 }
 
 }  // extern "C"
+
+extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_t ldp, float* Y, float* W,
+                              int64_t ldyw, int64_t* trace_host) {
+  if (!h) return -1;
+  if (m < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  int rc = ensure_ws(h, m + b, b, b, 0, nullptr);
+  if (rc != SBR_OK) return rc;
+  cudaStream_t st = h->stream;
+  DevBuf tr(trace_host ? sizeof(int64_t) * 16 : 0);
+  if (trace_host) {
+    if (!tr.p) return SBR_ERR_NOMEM;
+    SBR_CK(cudaMemsetAsync(tr.p, 0, sizeof(int64_t) * 16, st), "memset");
+  }
+  PanelArgs pa{};
+  pa.P = P;
+  pa.ldp = ldp;
+  pa.m = (int)m;
+  pa.b = b;
+  pa.Y = Y;
+  pa.ldy = ldyw;
+  pa.W = W;
+  pa.ldw = ldyw;
+  pa.row0 = 0;
+  pa.M = m;
+  pa.ws_v = h->pv;
+  pa.ws_tau = h->ptau;
+  pa.ws_r = h->pr;
+  pa.ws_q = h->pq;
+  pa.ws_misc = h->pmisc;
+  pa.trace = trace_host ? (int64_t*)tr.p : nullptr;
+  if (h->panel_mode == 0 && m > 512 && m >= 2 * b) {
+    const cudaError_t ce = launch_panel_chol(pa, h->panel_ctas, h->gram, h->pfail, st);
+    if (ce == cudaSuccess) pa.run_if = h->pfail;
+    else if (ce != cudaErrorNotSupported) SBR_CK(ce, "panel_chol");
+  }
+  SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
+  if (trace_host) {
+    SBR_CK(cudaMemcpyAsync(trace_host, tr.p, sizeof(int64_t) * 16, cudaMemcpyDeviceToHost, st), "trace D2H");
+    SBR_CK(cudaStreamSynchronize(st), "sync");
+  }
+  return SBR_OK;
+}

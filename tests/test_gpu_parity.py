@@ -115,5 +115,9 @@ def test_reduce_host_matches_device():
     pinned = torch.from_numpy(a_host.copy()).pin_memory()
     ab_host, _ = h.reduce_host(pinned, b, nb, mode="fp16")
     torch.cuda.synchronize()
-    # same kernels; float atomics make the summation order (not the math) differ
-    np.testing.assert_allclose(ab_host.numpy(), ab_dev.cpu().numpy(), atol=1e-4, rtol=0)
+    # Same kernels, but fp32 reductions (atomics) sum in a different order, and SBR is
+    # backward- not forward-stable: compare the spectra of the two bands, not entries.
+    lam_h = np.linalg.eigvalsh(sbr.band_to_dense(ab_host.double()).numpy())
+    lam_d = np.linalg.eigvalsh(sbr.band_to_dense(ab_dev.double().cpu()).numpy())
+    assert np.max(np.abs(lam_h - lam_d)) <= 1e-3 * np.max(np.abs(lam_d))
+    assert np.all(np.isfinite(ab_host.numpy()))
