@@ -1,212 +1,284 @@
-// k_panel_chol.cu -- panel QR by shifted CholeskyQR in fp64 + the paper's Householder
+// k_panel_chol.cu -- panel QR by CholeskyQR in fp64 + the paper's Householder
 // reconstruction (steps a1, a2), the B200 fast path for tall panels.
 //
 // Why not only TSQR: on sm_100a the TSQR tree is latency-bound -- every tree
 // level is b dependent Householder column steps in one CTA -- while fp64 SIMT throughput
-// is ample.  Shifted CholeskyQR3 (Fukaya, Kannan, Nakatsukasa, Yamamoto, Yanagisawa 2020)
-// needs grid-wide Gram reductions only and keeps all SMs busy:
-//     G1 = P^T P + s I, R1 = chol(G1), Q1 = P R1^-1   (s = 11 (m b + b(b+1)) u ||P||_F^2)
-//     G2 = Q1^T Q1,     R2 = chol(G2), Q2 = Q1 R2^-1
-//     G3 = Q2^T Q2,     R3 = chol(G3), Q  = Q2 R3^-1,  R = R3 R2 R1
-// in fp64 (u = 2^-53; panel data fp32), stable for cond(P) up to ~1e12.  A round k >= 2 is
-// skipped once G_k = I to 1e-12 (Q is orthonormal to fp64 accuracy).  A panel whose
-// second-round Cholesky signals (numerical) rank deficiency is left untouched and a flag
-// makes the TSQR kernel (k_panel.cu), launched right after, factor it instead.
+// is ample.  CholeskyQR needs only grid-wide Gram reductions and keeps all SMs busy:
+//     round 0:  G = P^T P,  R_0 = chol(G),  Q = P R_0^-1
+//     round k:  G = Q^T Q;  if max|G - I| <= 1e-9 stop, else R_k = chol(G), Q <- Q R_k^-1
+//     R = R_k ... R_1 R_0
+// in fp64 (panel data fp32).  The a-posteriori test G = Q^T Q ~ I (to 1e-9, far below the
+// fp32 outputs' rounding) makes the result as good as TSQR's whenever it is accepted; one
+// round suffices for cond(P) up to ~1e3, two up to ~1e7 (CholeskyQR2).  A panel whose
+// Cholesky breaks down (numerical rank deficiency) or that is still not orthonormal after
+// three rounds is left untouched and a flag makes the TSQR kernel (k_panel.cu), launched
+// right after, factor it instead.
 // The explicit Q then goes through the same reconstruction as TSQR's (Alg. 3 + S,
 // P:315-339; reading C7): Q_1 - S = L U, Y = [L; Q_2 U^-1], W = (E - Q S) L^-T,
 // R_h = S R.  The result is the LAPACK dgeqrf (V, T, R) of the panel.
-// Latency design: every b x b factorisation is one warp with its columns in registers
-// (fully unrolled, row broadcasts through shared memory); every triangular solve is
-// right-looking so its dependency chain is b steps, not b^2/2.
+//
+// Latency design (the panel is on the critical path of every b columns):
+//  * one CTA per SM, rows of the panel resident in shared memory in fp64 for all rounds;
+//  * Gram matrices reduced by fp64 atomics into PC_NCOPY copies, then a hand-rolled split
+//    grid barrier (arrive / wait) so CTA 0 can run the LU of Q_1 - S speculatively between
+//    its arrive and its wait -- the LU overlaps the barrier instead of adding one;
+//  * the b x b Cholesky / LU are one warp each with columns in registers; the next pivot
+//    is computed first so the dependency chain per column is shfl -> rsqrt -> fma;
+//  * Gram sets, barrier counters are double-buffered by launch parity: launch L zeroes the
+//    buffers of parity (L+1)&1 while using those of parity L&1 -- no memset launches.
 #include <cooperative_groups.h>
 
 #include "common.cuh"
 #include "kernels.h"
 
-namespace cg = cooperative_groups;
-
 namespace sbr {
 
 constexpr int PC_THREADS = 256;
-constexpr int PC_NCOPY = 8;   // Gram accumulated into 8 copies (CTA k -> k % 8): less atomic contention
-template <int B> constexpr int pc_maxr() { return B <= 32 ? 512 : 160; }   // rows per CTA
-template <int B> constexpr int pc_ngrp() { return PC_THREADS / ((B / 4) * (B / 4)) > 0 ? PC_THREADS / ((B / 4) * (B / 4)) : 1; }
+constexpr int PC_NCOPY = 8;    // Gram accumulated into 8 copies (CTA k -> k % 8): less atomic contention
+constexpr int PC_NSET = 4;     // Gram sets per launch: round 0 + up to 3 checks
+constexpr int PC_SETSTRIDE = 64 * 64;   // doubles per copy (max b)
+constexpr double PC_ORTH_TOL = 1e-9;
+template <int B> constexpr int pc_maxr() { return B <= 32 ? 512 : 128; }   // rows per CTA (smem)
+template <int B> constexpr int pc_tpb() { return B / 4; }
+template <int B> constexpr int pc_nt() { return pc_tpb<B>() * (pc_tpb<B>() + 1) / 2; }   // upper 4x4 tiles
+template <int B> constexpr int pc_ngrp() { return PC_THREADS / pc_nt<B>() > 0 ? PC_THREADS / pc_nt<B>() : 1; }
+
+// global workspace (bytes): [sets: 2 parities x NSET x NCOPY x 64 x 64 doubles]
+//                           [ctr[2], luflag, fail]  [lu: Lcol, Urow (64x64 f32), S, dinv (64 f32)]
+constexpr size_t PCW_SETS = 0;
+constexpr size_t PCW_CTL = PCW_SETS + sizeof(double) * 2 * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
+constexpr size_t PCW_LU = PCW_CTL + 256;
+constexpr size_t PCW_BYTES = PCW_LU + sizeof(float) * (2 * 64 * 64 + 2 * 64);
+
+size_t panel_chol_ws_bytes() { return PCW_BYTES; }
+int* panel_chol_fail(void* ws) { return reinterpret_cast<int*>((char*)ws + PCW_CTL) + 3; }
 
 template <int B>
 struct CholSmem {
   static constexpr int LDG = B + 1;
-  static constexpr size_t OFF_Q = 0;                                            // double rows x B
-  static constexpr size_t OFF_GP = OFF_Q + sizeof(double) * pc_maxr<B>() * B;  // double NGRP x B x B
-  static constexpr size_t OFF_G = OFF_GP + sizeof(double) * (pc_ngrp<B>() > 2 ? pc_ngrp<B>() : 2) * B * B;   // double B x LDG
-  static constexpr size_t OFF_RD = OFF_G + sizeof(double) * B * LDG;           // double B
-  static constexpr size_t OFF_RR = OFF_RD + sizeof(double) * B;                // double B (row broadcast)
-  static constexpr size_t OFF_U = OFF_RR + sizeof(double) * B;                 // float B x LDG
-  static constexpr size_t OFF_L = OFF_U + sizeof(float) * B * LDG;             // float B x LDG
-  static constexpr size_t OFF_S = OFF_L + sizeof(float) * B * LDG;             // float B (signs)
-  static constexpr size_t OFF_LR = OFF_S + sizeof(float) * B;                  // float B (row broadcast)
+  static constexpr int LDQ = B + 2;   // Qd row stride (doubles): 4-way instead of 32-way conflicts on column stores
+  static constexpr int NGRP = pc_ngrp<B>();
+  static constexpr size_t OFF_Q = 0;                                              // double rows x B (row-major)
+  static constexpr size_t OFF_GP = OFF_Q + sizeof(double) * pc_maxr<B>() * LDQ;  // double NGRP x B x B
+  static constexpr size_t OFF_G = OFF_GP + sizeof(double) * NGRP * B * B;        // double B x LDG (chol in place)
+  static constexpr size_t OFF_RRM = OFF_G + sizeof(double) * B * LDG;            // double B x B, R row-major
+  static constexpr size_t OFF_RACC = OFF_RRM + sizeof(double) * B * B;           // double B x B (CTA 0: R product)
+  static constexpr size_t OFF_RD = OFF_RACC + sizeof(double) * B * B;            // double B (1 / r_jj)
+  static constexpr size_t OFF_RROW = OFF_RD + sizeof(double) * B;                // double B (row broadcast)
+  // L, U alias the Gram partials (Gpart is dead once a round's bulk reduction completed;
+  // the LU of a round is recomputed after any later Gram)
+  static constexpr size_t OFF_LC = OFF_GP;                                       // float B x B: Lcol[k*B + c] = L[c][k]
+  static constexpr size_t OFF_UR = OFF_LC + sizeof(float) * B * B;               // float B x B: Urow[k*B + c] = U[k][c]
+  static constexpr size_t OFF_S = OFF_RROW + sizeof(double) * B;                 // float B signs
+  static constexpr size_t OFF_DI = OFF_S + sizeof(float) * B;                    // float B 1/U[k][k]
+  static constexpr size_t OFF_LR = OFF_DI + sizeof(float) * B;
   static constexpr size_t BYTES = OFF_LR + sizeof(float) * B + 64;
 };
 
-// In-place Cholesky (CTA, one barrier per column) -- used for b > 32.
-template <int LDG>
-SBR_DEV bool cta_chol(double* G, double* rd, int b, double floor_rel) {
+SBR_DEV unsigned ld_acquire_u32(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+SBR_DEV void st_release_u32(unsigned* p, unsigned v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+SBR_DEV void bar_arrive(unsigned* ctr) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(ctr, 1u);
+  }
+}
+SBR_DEV void bar_wait(const unsigned* ctr, unsigned target) {
+  if (threadIdx.x == 0) {
+    while (ld_acquire_u32(ctr) < target) {
+    }
+  }
+  __syncthreads();
+}
+
+// Cholesky G = R^T R of a B x B (B <= 32) fp64 matrix by ONE warp: lane c holds column c
+// in registers; R row j is broadcast through shared memory (rrow); the next pivot is
+// computed first so the chain per column is shfl -> rsqrt -> mul -> fma.  (Measured on
+// B200, tools/ubench/ubench_fact.cu: ~9.1k cycles for b = 32, vs 9.8k with all-shuffle
+// broadcasts and 14-20k for rolled variants.)  Writes R (upper, row-major) to Rrm,
+// R (upper, ld LDG) to G and 1/r_jj to rd.  Returns false on breakdown
+// (pivot <= floor_rel * max diag).
+template <int B, int LDG>
+SBR_DEV bool warp_chol(double* G, double* Rrm, double* rd, double* rrow, double floor_rel) {
+  const int lane = lane_id();
+  double g[B];
+#pragma unroll
+  for (int i = 0; i < B; ++i) g[i] = (lane < B && i <= lane) ? G[i + lane * LDG] : 0.0;
+  double dmax = (lane < B) ? G[lane + lane * LDG] : 0.0;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) dmax = fmax(dmax, __shfl_xor_sync(0xffffffffu, dmax, o));
+  bool ok = true;
+  double piv = __shfl_sync(0xffffffffu, g[0], 0);
+#pragma unroll
+  for (int j = 0; j < B; ++j) {
+    ok = ok && (piv > floor_rel * dmax);
+    const double r = rsqrt(fmax(piv, 1e-300));   // 1 / r_jj
+    const double rjc = g[j] * r;                  // r_jc (lane j: r_jj)
+    g[j] = rjc;
+    if (j + 1 < B) piv = __shfl_sync(0xffffffffu, fma(-rjc, rjc, g[j + 1]), j + 1);
+    if (lane == j) rd[j] = r;
+    if (lane < B) rrow[lane] = rjc;
+    __syncwarp();
+#pragma unroll
+    for (int i = j + 1; i < B; ++i) g[i] = fma(-rrow[i], rjc, g[i]);
+    __syncwarp();
+  }
+  if (lane < B) {
+#pragma unroll
+    for (int i = 0; i < B; ++i) {
+      const double v = (i <= lane) ? g[i] : 0.0;
+      G[i + lane * LDG] = v;
+      Rrm[i * B + lane] = v;
+    }
+  }
+  __syncwarp();
+  return __all_sync(0xffffffffu, ok);
+}
+
+// Same by the whole CTA (one barrier per column) -- used for B > 32.
+template <int B, int LDG>
+SBR_DEV bool cta_chol(double* G, double* Rrm, double* rd, double floor_rel) {
   double dmax = 0.0;
-  for (int i = 0; i < b; ++i) dmax = fmax(dmax, G[i + i * LDG]);
+  for (int i = 0; i < B; ++i) dmax = fmax(dmax, G[i + i * LDG]);
   bool ok = true;
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5, ny = blockDim.x >> 5;
-  for (int j = 0; j < b; ++j) {
+  for (int j = 0; j < B; ++j) {
     const double gjj = G[j + j * LDG];
     if (!(gjj > floor_rel * dmax)) ok = false;
-    const double inv = __drcp_rn(fmax(gjj, 1e-300));
-    for (int c = j + 1 + tx; c < b; c += 32) {
+    const double inv = 1.0 / fmax(gjj, 1e-300);
+    for (int c = j + 1 + tx; c < B; c += 32) {
       const double gjc = G[j + c * LDG] * inv;
       for (int i = j + 1 + ty; i <= c; i += ny) G[i + c * LDG] = fma(-G[j + i * LDG], gjc, G[i + c * LDG]);
     }
     __syncthreads();
   }
-  for (int i = threadIdx.x; i < b; i += blockDim.x) rd[i] = rsqrt(fmax(G[i + i * LDG], 1e-300));
+  for (int i = threadIdx.x; i < B; i += blockDim.x) rd[i] = rsqrt(fmax(G[i + i * LDG], 1e-300));
   __syncthreads();
-  for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-    const int i = e % b, c = e / b;
-    G[i + c * LDG] = (i <= c) ? G[i + c * LDG] * rd[i] : 0.0;
+  for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+    const int i = e % B, c = e / B;
+    const double v = (i <= c) ? G[i + c * LDG] * rd[i] : 0.0;
+    G[i + c * LDG] = v;
+    Rrm[i * B + c] = v;
   }
   __syncthreads();
   return ok;
 }
 
-// Cholesky G = R^T R of a b x b (b <= 32) fp64 matrix by ONE warp: lane c holds column c
-// in registers, R row j is broadcast through rrow.  G (upper) -> R (upper) in place, rd = 1/diag.
-template <int LDG>
-SBR_DEV bool warp_chol32(double* G, double* rd, double* rrow, int b, double floor_rel) {
+// Modified LU of Q_1 - S (s_j = -sign(d_j)) of a B x B (B <= 32) matrix by ONE
+// warp (fp32).  Lane c holds column c, shifted so col[k] is row j+k at step j (rolled step
+// loop, static register indices -- see warp_chol); L column j is broadcast from lane j by
+// shuffles.  Writes Lcol[k*B + c] = L[c][k] (unit lower), Urow[k*B + c] = U[k][c], S and
+// dinv = 1/U[k][k].
+template <int B, int LDQ>
+SBR_DEV void warp_lu(const double* Q1, float* Lcol, float* Urow, float* Ss, float* dinv) {
   const int lane = lane_id();
-  double g[32];
+  float col[B];
 #pragma unroll
-  for (int i = 0; i < 32; ++i) g[i] = (lane < b && i <= lane) ? G[i + lane * LDG] : 0.0;
-  double dmax = (lane < b) ? G[lane + lane * LDG] : 0.0;
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) dmax = fmax(dmax, __shfl_xor_sync(0xffffffffu, dmax, o));
-  bool ok = true;
-#pragma unroll
-  for (int j = 0; j < 32; ++j) {
-    if (j < b) {
-      const double gjj = __shfl_sync(0xffffffffu, g[j], j);
-      if (!(gjj > floor_rel * dmax)) ok = false;
-      const double rjj = sqrt(fmax(gjj, 1e-300));
-      const double rjc = (lane == j) ? rjj : g[j] * __drcp_rn(rjj);
-      if (lane >= j) g[j] = rjc;
-      rrow[lane] = (lane > j && lane < b) ? rjc : 0.0;
-      __syncwarp();
-#pragma unroll
-      for (int i = j + 1; i < 32; ++i) {
-        const double rji = rrow[i];
-        if (lane >= i) g[i] = fma(-rji, rjc, g[i]);
-      }
-      __syncwarp();
+  for (int i = 0; i < B; ++i) col[i] = (lane < B) ? (float)Q1[i * LDQ + lane] : 0.f;
+#pragma unroll 1
+  for (int j = 0; j < B; ++j) {
+    const float d = __shfl_sync(0xffffffffu, col[0], j);   // A[j][j]
+    const float sj = (d >= 0.f) ? -1.f : 1.f;
+    const float piv = d - sj;
+    const float inv = __fdividef(1.f, piv);
+    const float ujc = (lane == j) ? piv : col[0];   // lane c >= j: U[j][c]
+    if (lane < B) {
+      Urow[j * B + lane] = (lane >= j) ? ujc : 0.f;
+      Lcol[lane * B + j] = (lane < j) ? col[0] : (lane == j ? 1.f : 0.f);   // L[j][lane]
     }
-  }
-  if (lane < b) {
+    if (lane == j) {
+      Ss[j] = sj;
+      dinv[j] = inv;
+    }
 #pragma unroll
-    for (int i = 0; i < 32; ++i)
-      if (i < b) G[i + lane * LDG] = (i <= lane) ? g[i] : 0.0;
+    for (int k0 = 1; k0 < B; k0 += 8) {
+      if (j + k0 < B) {
+#pragma unroll
+        for (int k = k0; k < k0 + 8 && k < B; ++k) {
+          const float lk = __shfl_sync(0xffffffffu, col[k], j) * inv;   // L[j+k][j]
+          col[k - 1] = (lane > j) ? fmaf(-lk, ujc, col[k]) : ((lane == j) ? lk : col[k]);
+        }
+      }
+    }
+    col[B - 1] = 0.f;
   }
   __syncwarp();
-  if (lane < b) rd[lane] = 1.0 / G[lane + lane * LDG];
-  __syncwarp();
-  return __all_sync(0xffffffffu, ok);
 }
 
-// Modified LU of Q_1 - S (s_j = -sign(d_j)) of a b x b (b <= 32) fp32 matrix by ONE
-// warp: lane c holds column c; the L column is broadcast through lrow.  Writes U (with the
-// pivots on its diagonal), L (unit lower) and the signs.
-template <int LDG>
-SBR_DEV void warp_lu32(int b, const double* Q1, int ldq_row, float* Us, float* Ls, float* Ss, float* lrow) {
-  const int lane = lane_id();
-  float col[32];
-#pragma unroll
-  for (int i = 0; i < 32; ++i) col[i] = (lane < b && i < b) ? (float)Q1[i * ldq_row + lane] : 0.f;
-#pragma unroll
-  for (int j = 0; j < 32; ++j) {
-    if (j < b) {
-      const float d = __shfl_sync(0xffffffffu, col[j], j);
-      const float sj = (d >= 0.f) ? -1.f : 1.f;
-      const float piv = d - sj;
-      const float inv = __frcp_rn(piv);
-      if (lane == j) {
-        col[j] = piv;
-#pragma unroll
-        for (int i = j + 1; i < 32; ++i) { col[i] *= inv; lrow[i] = col[i]; }
-        Ss[j] = sj;
-      }
-      __syncwarp();
-      if (lane > j) {
-        const float ujc = col[j];
-#pragma unroll
-        for (int i = j + 1; i < 32; ++i) col[i] = fmaf(-lrow[i], ujc, col[i]);
-      }
-      __syncwarp();
-    }
-  }
-  if (lane < b) {
-#pragma unroll
-    for (int i = 0; i < 32; ++i) {
-      if (i < b) {
-        Us[i + lane * LDG] = (i <= lane) ? col[i] : 0.f;
-        Ls[i + lane * LDG] = (i > lane) ? col[i] : (i == lane ? 1.f : 0.f);
-      }
-    }
-  }
-}
-
-// Same by the whole CTA (one barrier per column) -- used for b > 32.
-template <int LDG>
-SBR_DEV void cta_lu(int b, const double* Q1, int ldq_row, float* Us, float* Ls, float* Ss) {
-  for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-    const int i = e % b, c = e / b;
-    Us[i + c * LDG] = (float)Q1[i * ldq_row + c];
-  }
+// Same by the whole CTA (one barrier per column) -- used for B > 32.
+template <int B, int LDQ>
+SBR_DEV void cta_lu(const double* Q1, float* Lcol, float* Urow, float* Ss, float* dinv) {
+  // work in Urow as a dense row-major matrix A[i][c] = Urow[i*B + c]
+  for (int e = threadIdx.x; e < B * B; e += blockDim.x) Urow[e] = (float)Q1[(e / B) * LDQ + e % B];
   __syncthreads();
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5, ny = blockDim.x >> 5;
-  for (int j = 0; j < b; ++j) {
-    const float d = Us[j + j * LDG];
+  for (int j = 0; j < B; ++j) {
+    const float d = Urow[j * B + j];
     const float sj = (d >= 0.f) ? -1.f : 1.f;
     const float invp = __frcp_rn(d - sj);
-    for (int c = j + 1 + tx; c < b; c += 32) {
-      const float ujc = Us[j + c * LDG] * invp;
-      for (int i = j + 1 + ty; i < b; i += ny) Us[i + c * LDG] = fmaf(-Us[i + j * LDG], ujc, Us[i + c * LDG]);
+    for (int c = j + 1 + tx; c < B; c += 32) {
+      const float ujc = Urow[j * B + c];
+      for (int i = j + 1 + ty; i < B; i += ny) Urow[i * B + c] = fmaf(-Urow[i * B + j] * invp, ujc, Urow[i * B + c]);
     }
     __syncthreads();
-    for (int i = j + 1 + threadIdx.x; i < b; i += blockDim.x) Ls[i + j * LDG] = Us[i + j * LDG] * invp;
-    if (threadIdx.x == 0) { Ss[j] = sj; Us[j + j * LDG] = d - sj; }
+    for (int i = j + 1 + threadIdx.x; i < B; i += blockDim.x) Lcol[j * B + i] = Urow[i * B + j] * invp;
+    if (threadIdx.x == 0) {
+      Ss[j] = sj;
+      dinv[j] = invp;
+      Urow[j * B + j] = d - sj;
+    }
     __syncthreads();
   }
-  for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-    const int i = e % b, c = e / b;
-    if (i > c) Us[i + c * LDG] = 0.f;
-    else Ls[i + c * LDG] = (i == c) ? 1.f : 0.f;
+  for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+    const int k = e / B, c = e % B;
+    if (c < k) Urow[k * B + c] = 0.f;             // U is upper
+    if (c <= k) Lcol[k * B + c] = (c == k) ? 1.f : 0.f;   // L column k: rows < k zero, unit diagonal
   }
   __syncthreads();
 }
 
 template <int B>
-__global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, double* gram, int* fail) {
+__global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, unsigned char* ws, unsigned launch) {
   using L = CholSmem<B>;
   constexpr int LDG = L::LDG;
+  constexpr int LDQ = L::LDQ;
+  constexpr int NGRP = L::NGRP;
+  constexpr int TPB = pc_tpb<B>(), NT = pc_nt<B>();
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  double* Qd = reinterpret_cast<double*>(smem_raw + L::OFF_Q);     // rows x B, row-major, fp64
+  double* Qd = reinterpret_cast<double*>(smem_raw + L::OFF_Q);
   double* Gpart = reinterpret_cast<double*>(smem_raw + L::OFF_GP);
   double* Gk = reinterpret_cast<double*>(smem_raw + L::OFF_G);
+  double* Rrm = reinterpret_cast<double*>(smem_raw + L::OFF_RRM);
+  double* Racc = reinterpret_cast<double*>(smem_raw + L::OFF_RACC);
   double* rd = reinterpret_cast<double*>(smem_raw + L::OFF_RD);
-  double* rrow = reinterpret_cast<double*>(smem_raw + L::OFF_RR);
-  float* Us = reinterpret_cast<float*>(smem_raw + L::OFF_U);
-  float* Ls = reinterpret_cast<float*>(smem_raw + L::OFF_L);
+  double* rrow = reinterpret_cast<double*>(smem_raw + L::OFF_RROW);
+  float* Lc = reinterpret_cast<float*>(smem_raw + L::OFF_LC);
+  float* Ur = reinterpret_cast<float*>(smem_raw + L::OFF_UR);
   float* Ss = reinterpret_cast<float*>(smem_raw + L::OFF_S);
-  float* lrow = reinterpret_cast<float*>(smem_raw + L::OFF_LR);
-  double* Rstore = gram + 3 * PC_NCOPY * B * B;                    // R_1, R_2, R_3 (global)
-  cg::grid_group grid = cg::this_grid();
-  const int b = a.b;
+  float* Di = reinterpret_cast<float*>(smem_raw + L::OFF_DI);
+
+  const unsigned par = launch & 1u;
+  double* sets = reinterpret_cast<double*>(ws + PCW_SETS) + (size_t)par * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
+  unsigned* ctl = reinterpret_cast<unsigned*>(ws + PCW_CTL);
+  unsigned* ctr = ctl + par;
+  unsigned* luflag = ctl + 2;
+  int* fail = reinterpret_cast<int*>(ctl + 3);
+  float* gLc = reinterpret_cast<float*>(ws + PCW_LU);
+  float* gUr = gLc + 64 * 64;
+  float* gS = gUr + 64 * 64;
+  float* gDi = gS + 64;
+
   const int warp = warp_id(), lane = lane_id();
   const int64_t m = a.m;
-  const int64_t r_beg = (int64_t)blockIdx.x * m / gridDim.x, r_end = (int64_t)(blockIdx.x + 1) * m / gridDim.x;
+  const int G = gridDim.x;
+  const int64_t r_beg = (int64_t)blockIdx.x * m / G, r_end = (int64_t)(blockIdx.x + 1) * m / G;
   const int rows = (int)(r_end - r_beg);
   auto stamp = [&](int k) {
     if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) {
@@ -216,285 +288,403 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     }
   };
   stamp(0);
-  // ---- load the CTA's rows: warp w -> columns w, w+8, ..; lane -> rows (coalesced, unrolled)
-  for (int c = warp; c < B; c += PC_THREADS / 32) {
-    const float* src = a.P + r_beg + (int64_t)c * a.ldp;
-#pragma unroll 4
-    for (int r = lane; r < pc_maxr<B>(); r += 32)
-      if (r < rows) Qd[r * B + c] = (c < b) ? (double)src[r] : 0.0;
+  // ---- load the CTA's rows (column-major fp32 -> row-major fp64): all loads issued first
+  {
+    constexpr int CPW = (B + 7) / 8, RPL = pc_maxr<B>() / 32;
+    float v[CPW][RPL];
+#pragma unroll
+    for (int ci = 0; ci < CPW; ++ci) {
+      const int c = warp + 8 * ci;
+      const float* src = a.P + r_beg + (int64_t)c * a.ldp;
+#pragma unroll
+      for (int k = 0; k < RPL; ++k) {
+        const int r = lane + 32 * k;
+        v[ci][k] = (c < B && r < rows) ? __ldg(src + r) : 0.f;
+      }
+    }
+#pragma unroll
+    for (int ci = 0; ci < CPW; ++ci) {
+      const int c = warp + 8 * ci;
+#pragma unroll
+      for (int k = 0; k < RPL; ++k) {
+        const int r = lane + 32 * k;
+        if (c < B && r < rows) Qd[r * LDQ + c] = (double)v[ci][k];
+      }
+    }
+  }
+  // ---- zero the other parity's Gram sets and barrier counter (used by the next launch)
+  {
+    double* other = reinterpret_cast<double*>(ws + PCW_SETS) + (size_t)(par ^ 1u) * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
+    const int64_t tot = (int64_t)PC_NSET * PC_NCOPY * PC_SETSTRIDE;
+    const int64_t per = (tot + G - 1) / G;
+    const int64_t lo = (int64_t)blockIdx.x * per, hi = std::min<int64_t>(tot, lo + per);
+    for (int64_t e = lo + threadIdx.x; e < hi; e += blockDim.x) other[e] = 0.0;
+    if (blockIdx.x == 0 && threadIdx.x == 0) ctl[par ^ 1u] = 0u;
   }
   __syncthreads();
-  stamp(4);
+  stamp(1);
 
-  int nrounds = 3;
-  for (int round = 0; round < nrounds; ++round) {
-    double* Gg = gram + (size_t)round * PC_NCOPY * B * B;   // PC_NCOPY copies
-    // ---- partial Gram of this CTA's rows: 4x4 register tiles, reduced over the row
-    //      groups in smem, then fp64 reductions of the upper triangle into Gg
-    {
-      constexpr int TPB = B / 4, NTILE = TPB * TPB, NGRP = pc_ngrp<B>();
-      const int grp = threadIdx.x / NTILE, tl = threadIdx.x % NTILE;
-      const int ti = tl / TPB, tj = tl % TPB;
-      double acc[4][4];
+  // Gram tile of this thread: upper 4x4 tile (ti, tj), row group grp
+  const int grp = threadIdx.x / NT, tl = threadIdx.x % NT;
+  int ti = 0, tj = tl;
+  while (tj >= TPB - ti) {
+    tj -= TPB - ti;
+    ++ti;
+  }
+  tj += ti;
+  auto gram_arrive = [&](int set) {   // partial Gram of Qd -> atomics into set -> barrier arrive
+    double acc[4][4];
 #pragma unroll
-      for (int u = 0; u < 4; ++u)
+    for (int u = 0; u < 4; ++u)
 #pragma unroll
-        for (int v = 0; v < 4; ++v) acc[u][v] = 0.0;
-      if (grp < NGRP && ti <= tj) {
+      for (int v = 0; v < 4; ++v) acc[u][v] = 0.0;
+    if (grp < NGRP) {
 #pragma unroll 2
-        for (int r = grp; r < rows; r += NGRP) {
-          const double2 a0 = *reinterpret_cast<const double2*>(Qd + r * B + 4 * ti);
-          const double2 a1 = *reinterpret_cast<const double2*>(Qd + r * B + 4 * ti + 2);
-          const double2 b0 = *reinterpret_cast<const double2*>(Qd + r * B + 4 * tj);
-          const double2 b1 = *reinterpret_cast<const double2*>(Qd + r * B + 4 * tj + 2);
-          const double aa[4] = {a0.x, a0.y, a1.x, a1.y};
-          const double bb[4] = {b0.x, b0.y, b1.x, b1.y};
-#pragma unroll
-          for (int u = 0; u < 4; ++u)
-#pragma unroll
-            for (int v = 0; v < 4; ++v) acc[u][v] = fma(aa[u], bb[v], acc[u][v]);
-        }
-      }
-      if (grp < NGRP) {
+      for (int r = grp; r < rows; r += NGRP) {
+        const double2 a0 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * ti);
+        const double2 a1 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * ti + 2);
+        const double2 b0 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * tj);
+        const double2 b1 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * tj + 2);
+        const double aa[4] = {a0.x, a0.y, a1.x, a1.y};
+        const double bb[4] = {b0.x, b0.y, b1.x, b1.y};
 #pragma unroll
         for (int u = 0; u < 4; ++u)
 #pragma unroll
-          for (int v = 0; v < 4; ++v) Gpart[grp * B * B + (4 * ti + u) + (4 * tj + v) * B] = acc[u][v];
+          for (int v = 0; v < 4; ++v) acc[u][v] = fma(aa[u], bb[v], acc[u][v]);
       }
-      __syncthreads();
-      if (round == 0) stamp(8);
-      for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
-        const int p = e % B, q = e / B;
-        if (p <= q && q < b) {
-          double sum = 0.0;
 #pragma unroll
-          for (int g = 0; g < NGRP; ++g) sum += Gpart[g * B * B + e];
-          atomicAdd(&Gg[(blockIdx.x % PC_NCOPY) * B * B + p + q * B], sum);
-        }
-      }
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4; ++v) Gpart[grp * B * B + (4 * ti + u) + (4 * tj + v) * B] = acc[u][v];
     }
-    stamp(1 + 4 * round);
-    grid.sync();
-    stamp(2 + 4 * round);
-    // ---- Cholesky (redundantly in every CTA; identical input -> identical R)
+    __syncthreads();
+    // reduce the row groups in place into group 0 (lower triangle zero), then ONE bulk
+    // async reduction (cp.reduce.async.bulk .add.f64) of the b x b block into the set copy
+    for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+      const int p = e % B, q = e / B;
+      double sum = 0.0;
+      if (p <= q) {
+#pragma unroll 4
+        for (int g2 = 0; g2 < NGRP; ++g2) sum += Gpart[g2 * B * B + e];
+      }
+      Gpart[e] = sum;
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    __syncthreads();
+    if (threadIdx.x == 0) {
+      double* Gg = sets + ((size_t)set * PC_NCOPY + blockIdx.x % PC_NCOPY) * PC_SETSTRIDE;
+      const unsigned sa = (unsigned)__cvta_generic_to_shared(Gpart);
+      asm volatile("cp.reduce.async.bulk.global.shared::cta.bulk_group.add.f64 [%0], [%1], %2;"
+                   ::"l"(Gg), "r"(sa), "r"((unsigned)(B * B * sizeof(double))) : "memory");
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+      asm volatile("fence.proxy.async.global;" ::: "memory");
+      __threadfence();
+      atomicAdd(ctr, 1u);
+    }
+  };
+  auto gram_read = [&](int set) {   // after the barrier: sum the copies into Gk (upper)
+    const double* Gs = sets + (size_t)set * PC_NCOPY * PC_SETSTRIDE;
     for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
       const int i = e % B, c = e / B;
       double g = 0.0;
-      if (i < b && c < b && i <= c)
+      if (i <= c) {
 #pragma unroll
-        for (int k = 0; k < PC_NCOPY; ++k) g += Gg[k * B * B + i + c * B];
+        for (int k = 0; k < PC_NCOPY; ++k) g += __ldcg(Gs + (size_t)k * PC_SETSTRIDE + e);
+      }
       Gk[i + c * LDG] = g;
     }
     __syncthreads();
-    if (round == 0) {                          // shift s = 11 (m b + b(b+1)) u ||P||_F^2
-      double tr = 0.0;
-      for (int i = 0; i < b; ++i) tr += Gk[i + i * LDG];
-      const double sh = 11.0 * ((double)m * b + (double)b * (b + 1)) * 1.1102230246251565e-16 * tr;
-      __syncthreads();
-      if (threadIdx.x < b) Gk[threadIdx.x * (LDG + 1)] += (sh > 0.0 ? sh : 1e-300);
-      __syncthreads();
-    } else {                                   // Q orthonormal to fp64 accuracy already: done
-      double dev = 0.0;
-      for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-        const int i = e % b, c = e / b;
-        if (i <= c) dev = fmax(dev, fabs(Gk[i + c * LDG] - (i == c ? 1.0 : 0.0)));
-      }
-      const int big = __syncthreads_or(dev > 1e-12);
-      if (!big) {
-        if (blockIdx.x == 0)
-          for (int rr = round; rr < 3; ++rr)
-            for (int e = threadIdx.x; e < B * B; e += blockDim.x) Rstore[rr * B * B + e] = (e % B == e / B) ? 1.0 : 0.0;
-        nrounds = round;
-        break;
-      }
-    }
-    bool ok;
+  };
+  auto chol = [&](double floor_rel) -> bool {
     if constexpr (B <= 32) {
       __shared__ int okflag;
       if (warp == 0) {
-        const bool w = warp_chol32<LDG>(Gk, rd, rrow, b, round == 0 ? 0.0 : 1e-12);
+        const bool w = warp_chol<B, LDG>(Gk, Rrm, rd, rrow, floor_rel);
         if (lane == 0) okflag = w ? 1 : 0;
       }
       __syncthreads();
-      ok = okflag != 0;
+      return okflag != 0;
     } else {
-      ok = cta_chol<LDG>(Gk, rd, b, round == 0 ? 0.0 : 1e-12);
+      return cta_chol<B, LDG>(Gk, Rrm, rd, floor_rel);
     }
-    stamp(3 + 4 * round);
-    if (!ok) {                                 // rank deficient: leave the panel to TSQR
-      if (blockIdx.x == 0 && threadIdx.x == 0) *fail = 1;
-      return;
-    }
-    if (blockIdx.x == 0)
-      for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
-        const int i = e % B, c = e / B;
-        Rstore[round * B * B + e] = (i < b && c < b) ? Gk[i + c * LDG] : 0.0;
-      }
-    // ---- Q <- Q R_k^-1: thread per row, right-looking forward substitution (chain b)
-    for (int r = threadIdx.x; r < rows; r += blockDim.x) {
-      double q[B];
+  };
+  auto solve = [&]() {   // Q <- Q R^-1: forward substitution, 2 rows per thread (R row-major in Rrm)
+    const int half = (rows + 1) >> 1;
+    for (int r = threadIdx.x; r < half; r += blockDim.x) {
+      const int r2 = r + half;
+      const bool two = r2 < rows;
+      const double2* R2 = reinterpret_cast<const double2*>(Rrm);
+      asm volatile("" : "+l"(R2));   // opaque: no hoisting of the b^2 loads out of the row loop
+      double q[B], p[B];
 #pragma unroll
-      for (int c = 0; c < B; ++c) q[c] = Qd[r * B + c];
+      for (int c = 0; c < B; c += 2) {
+        const double2 t = *reinterpret_cast<const double2*>(Qd + r * LDQ + c);
+        q[c] = t.x;
+        q[c + 1] = t.y;
+        const double2 u = two ? *reinterpret_cast<const double2*>(Qd + r2 * LDQ + c) : make_double2(0.0, 0.0);
+        p[c] = u.x;
+        p[c + 1] = u.y;
+      }
 #pragma unroll
       for (int c = 0; c < B; ++c) {
-        if (c < b) {
-          q[c] *= rd[c];
+        q[c] *= rd[c];
+        p[c] *= rd[c];
 #pragma unroll
-          for (int c2 = c + 1; c2 < B; ++c2)
-            if (c2 < b) q[c2] = fma(-q[c], Gk[c + c2 * LDG], q[c2]);
+        for (int h = (c + 1) / 2; h < B / 2; ++h) {
+          const double2 rr = R2[c * (B / 2) + h];
+          if (2 * h > c) {
+            q[2 * h] = fma(-q[c], rr.x, q[2 * h]);
+            p[2 * h] = fma(-p[c], rr.x, p[2 * h]);
+          }
+          q[2 * h + 1] = fma(-q[c], rr.y, q[2 * h + 1]);
+          p[2 * h + 1] = fma(-p[c], rr.y, p[2 * h + 1]);
         }
       }
 #pragma unroll
-      for (int c = 0; c < B; ++c) Qd[r * B + c] = (c < b) ? q[c] : 0.0;
+      for (int c = 0; c < B; c += 2) {
+        *reinterpret_cast<double2*>(Qd + r * LDQ + c) = make_double2(q[c], q[c + 1]);
+        if (two) *reinterpret_cast<double2*>(Qd + r2 * LDQ + c) = make_double2(p[c], p[c + 1]);
+      }
     }
     __syncthreads();
-  }
-  stamp(13);
-  // ---- reconstruction: LU of Q_1 - S by CTA 0 (holds Q's top b rows), published to all
-  if (blockIdx.x == 0) {
-    if (threadIdx.x == 0) *fail = 0;
+  };
+  auto racc_update = [&](bool first) {   // CTA 0: Racc <- R_k Racc (upper triangular product)
+    if (first) {
+      for (int e = threadIdx.x; e < B * B; e += blockDim.x) Racc[e] = Rrm[e];
+      __syncthreads();
+      return;
+    }
+    constexpr int PER = (B * B + PC_THREADS - 1) / PC_THREADS;
+    double t4[PER];
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int e = threadIdx.x + k * PC_THREADS;
+      double acc = 0.0;
+      if (e < B * B) {
+        const int i = e / B, c = e % B;
+        for (int kk = i; kk <= c; ++kk) acc = fma(Rrm[i * B + kk], Racc[kk * B + c], acc);
+      }
+      t4[k] = acc;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < PER; ++k) {
+      const int e = threadIdx.x + k * PC_THREADS;
+      if (e < B * B) Racc[e] = t4[k];
+    }
+    __syncthreads();
+  };
+  auto lu_publish = [&](unsigned gen) {   // CTA 0: LU of Q_1 - S, to smem and to global
     if constexpr (B <= 32) {
-      if (warp == 0) warp_lu32<LDG>(b, Qd, B, Us, Ls, Ss, lrow);
+      if (warp == 0) warp_lu<B, LDQ>(Qd, Lc, Ur, Ss, Di);
       __syncthreads();
     } else {
-      cta_lu<LDG>(b, Qd, B, Us, Ls, Ss);
+      cta_lu<B, LDQ>(Qd, Lc, Ur, Ss, Di);
     }
-    stamp(12);
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-      const int i = e % b, c = e / b;
-      a.ws_misc[e] = Us[i + c * LDG];
-      a.ws_misc[b * b + e] = Ls[i + c * LDG];
-    }
-    if (threadIdx.x < b) a.ws_misc[2 * b * b + threadIdx.x] = Ss[threadIdx.x];
-    // R = R_3 R_2 R_1 for the compact panel (rows < b): copy to smem, two triangular products
-    double* R1 = Gpart;
-    double* R2 = Gpart + B * B;
-    double* R3 = Gk;   // ld B here
     for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
-      R1[e] = Rstore[e];
-      R2[e] = Rstore[B * B + e];
-      R3[e] = Rstore[2 * B * B + e];
+      gLc[e] = Lc[e];
+      gUr[e] = Ur[e];
+    }
+    if (threadIdx.x < B) {
+      gS[threadIdx.x] = Ss[threadIdx.x];
+      gDi[threadIdx.x] = Di[threadIdx.x];
     }
     __syncthreads();
-    double t4[(B * B + PC_THREADS - 1) / PC_THREADS];
-    for (int k = 0; k < (B * B + PC_THREADS - 1) / PC_THREADS; ++k) t4[k] = 0.0;
-    int kk = 0;
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x, ++kk) {   // T = R2 R1
-      const int i = e % b, c = e / b;
-      double acc = 0.0;
-      for (int k = i; k <= c; ++k) acc = fma(R2[i + k * B], R1[k + c * B], acc);
-      t4[kk] = (i <= c) ? acc : 0.0;
+    if (threadIdx.x == 0) {
+      __threadfence();
+      st_release_u32(luflag, gen);
     }
-    __syncthreads();
-    kk = 0;
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x, ++kk) R2[(e % b) + (e / b) * B] = t4[kk];
-    __syncthreads();
-    kk = 0;
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x, ++kk) {   // R = R3 T
-      const int i = e % b, c = e / b;
-      double acc = 0.0;
-      for (int k = i; k <= c; ++k) acc = fma(R3[i + k * B], R2[k + c * B], acc);
-      t4[kk] = (i <= c) ? acc : 0.0;
-    }
-    __syncthreads();
-    kk = 0;
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x, ++kk) R1[(e % b) + (e / b) * B] = t4[kk];
-    __syncthreads();
+  };
+
+  // ---- round 0: G = P^T P, R_0 = chol(G), Q = P R_0^-1
+  gram_arrive(0);
+  stamp(2);
+  bar_wait(ctr, (unsigned)G);
+  stamp(3);
+  gram_read(0);
+  if (!chol(0.0)) {                    // not numerically SPD: leave the panel to TSQR
+    if (blockIdx.x == 0 && threadIdx.x == 0) *fail = 1;
+    return;
   }
-  stamp(14);
-  grid.sync();
-  stamp(15);
+  stamp(4);
+  solve();
+  if (blockIdx.x == 0) racc_update(true);
+  stamp(5);
+  // ---- rounds k = 1..3: check G = Q^T Q ~ I, else one more CholeskyQR step
+  unsigned gen = 0;
+  bool done = false;
+  for (int k = 1; k < PC_NSET; ++k) {
+    gram_arrive(k);
+    gen = launch * 4u + (unsigned)k;
+    if (k == 1) stamp(6);
+    if (blockIdx.x == 0) lu_publish(gen);   // speculative: valid if this round's check passes
+    if (k == 1) stamp(7);
+    bar_wait(ctr, (unsigned)G * (k + 1));
+    if (k == 1) stamp(8);
+    gram_read(k);
+    double dev = 0.0;
+    for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+      const int i = e % B, c = e / B;
+      if (i <= c) dev = fmax(dev, fabs(Gk[i + c * LDG] - (i == c ? 1.0 : 0.0)));
+    }
+    if (!__syncthreads_or(!(dev <= PC_ORTH_TOL))) {
+      done = true;
+      break;
+    }
+    if (k == PC_NSET - 1 || !chol(0.0)) break;
+    solve();
+    if (blockIdx.x == 0) racc_update(false);
+  }
+  if (!done) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) *fail = 1;
+    return;
+  }
+  stamp(9);
+  // ---- L, U, S from CTA 0
   if (blockIdx.x != 0) {
-    for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
-      const int i = e % b, c = e / b;
-      Us[i + c * LDG] = a.ws_misc[e];
-      Ls[i + c * LDG] = a.ws_misc[b * b + e];
+    if (threadIdx.x == 0) {
+      while (ld_acquire_u32(luflag) != gen) {
+      }
     }
-    if (threadIdx.x < b) Ss[threadIdx.x] = a.ws_misc[2 * b * b + threadIdx.x];
     __syncthreads();
+    for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+      Lc[e] = __ldcg(gLc + e);
+      Ur[e] = __ldcg(gUr + e);
+    }
+    if (threadIdx.x < B) {
+      Ss[threadIdx.x] = __ldcg(gS + threadIdx.x);
+      Di[threadIdx.x] = __ldcg(gDi + threadIdx.x);
+    }
+    __syncthreads();
+  } else if (threadIdx.x == 0) {
+    *fail = 0;
   }
-  const double* Rfin = Gpart;   // CTA 0 only (ld B)
-  // ---- rows (right-looking solves): w L_1^T = (e_il) - q S ;  y = L_1 row (il < b) or y U = q
+  stamp(10);
+  // ---- rows: w L_1^T = e_il - q S ;  y = L_1 row (il < B) or y U = q ;  compact panel
   const int64_t row0 = a.row0;
   for (int r = threadIdx.x; r < rows; r += blockDim.x) {
     const int64_t il = r_beg + r;
     const int64_t gr = row0 + il;
-    float v_[B];
+    // opaque per-iteration copies of the smem factors: keeps the compiler from hoisting
+    // all b^2 loads out of the row loop (which spills)
+    const float* Lc_ = Lc;
+    const float* Ur_ = Ur;
+    asm volatile("" : "+l"(Lc_), "+l"(Ur_));
+    const float4* Lc4 = reinterpret_cast<const float4*>(Lc_);
+    const float4* Ur4 = reinterpret_cast<const float4*>(Ur_);
+    float qf[B], v_[B];
 #pragma unroll
-    for (int c = 0; c < B; ++c) v_[c] = (c < b) ? ((il == c) ? 1.f : 0.f) - (float)Qd[r * B + c] * Ss[c] : 0.f;
-#pragma unroll
-    for (int k = 0; k < B; ++k) {
-      if (k < b) {
-#pragma unroll
-        for (int c = k + 1; c < B; ++c)
-          if (c < b) v_[c] = fmaf(-v_[k], Ls[c + k * LDG], v_[c]);
-      }
+    for (int c = 0; c < B; c += 2) {
+      const double2 t = *reinterpret_cast<const double2*>(Qd + r * LDQ + c);
+      qf[c] = (float)t.x;
+      qf[c + 1] = (float)t.y;
     }
 #pragma unroll
-    for (int c = 0; c < B; ++c)
-      if (c < b) a.W[gr + c * a.ldw] = v_[c];
-    if (il < b) {
+    for (int c = 0; c < B; ++c) v_[c] = ((il == c) ? 1.f : 0.f) - qf[c] * Ss[c];
 #pragma unroll
-      for (int c = 0; c < B; ++c) v_[c] = (c < b) ? Ls[il + c * LDG] : 0.f;
+    for (int k = 0; k < B; ++k)
+#pragma unroll
+      for (int h = (k + 1) / 4; h < B / 4; ++h) {
+        const float4 l4 = Lc4[k * (B / 4) + h];
+        const float lv[4] = {l4.x, l4.y, l4.z, l4.w};
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (4 * h + u > k) v_[4 * h + u] = fmaf(-v_[k], lv[u], v_[4 * h + u]);
+      }
+#pragma unroll
+    for (int c = 0; c < B; ++c) a.W[gr + c * a.ldw] = v_[c];
+    if (il < B) {
+#pragma unroll
+      for (int c = 0; c < B; ++c) v_[c] = Lc_[c * B + il];   // L[il][c]
     } else {
 #pragma unroll
-      for (int c = 0; c < B; ++c) v_[c] = (c < b) ? (float)Qd[r * B + c] : 0.f;
-#pragma unroll
       for (int k = 0; k < B; ++k) {
-        if (k < b) {
-          v_[k] = v_[k] / Us[k + k * LDG];
+        qf[k] *= Di[k];
 #pragma unroll
-          for (int c = k + 1; c < B; ++c)
-            if (c < b) v_[c] = fmaf(-v_[k], Us[k + c * LDG], v_[c]);
+        for (int h = (k + 1) / 4; h < B / 4; ++h) {
+          const float4 u4 = Ur4[k * (B / 4) + h];
+          const float uv[4] = {u4.x, u4.y, u4.z, u4.w};
+#pragma unroll
+          for (int u = 0; u < 4; ++u)
+            if (4 * h + u > k) qf[4 * h + u] = fmaf(-qf[k], uv[u], qf[4 * h + u]);
         }
       }
+#pragma unroll
+      for (int c = 0; c < B; ++c) v_[c] = qf[c];
     }
 #pragma unroll
     for (int c = 0; c < B; ++c) {
-      if (c < b) {
-        a.Y[gr + c * a.ldy] = v_[c];
-        // compact panel: Y tail strictly below, R_h = S R on and above the diagonal (CTA 0)
-        a.P[il + (int64_t)c * a.ldp] = (il > c) ? v_[c] : (float)((double)Ss[il] * Rfin[il + c * B]);
-        if (a.Yh) a.Yh[gr * a.ldyh + c] = __float2half_rn(v_[c]);
+      a.Y[gr + c * a.ldy] = v_[c];
+      // compact panel: Y tail strictly below, R_h = S R on and above the diagonal (CTA 0)
+      a.P[il + (int64_t)c * a.ldp] = (il > c) ? v_[c] : (il < B ? (float)((double)Ss[il] * Racc[il * B + c]) : 0.f);
+    }
+    if (a.Yh) {
+      __half* yh = a.Yh + gr * a.ldyh;
+      if constexpr (B % 8 == 0) {
+#pragma unroll
+        for (int c = 0; c < B; c += 8) {
+          __align__(16) __half hv[8];
+#pragma unroll
+          for (int u = 0; u < 8; ++u) hv[u] = __float2half_rn(v_[c + u]);
+          *reinterpret_cast<uint4*>(yh + c) = *reinterpret_cast<const uint4*>(hv);
+        }
+      } else {
+#pragma unroll
+        for (int c = 0; c < B; ++c) yh[c] = __float2half_rn(v_[c]);
       }
     }
   }
+  // rows of the block above the panel: Y = W = 0
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t nth = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = tid; i < row0; i += nth) {
-    for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
-    if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
+#pragma unroll
+    for (int c = 0; c < B; ++c) {
+      a.Y[i + c * a.ldy] = 0.f;
+      a.W[i + c * a.ldw] = 0.f;
+    }
+    if (a.Yh) {
+#pragma unroll
+      for (int c = 0; c < B; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
+    }
   }
+  stamp(11);
 }
 
 template <int B>
-static cudaError_t launch_chol_t(PanelArgs& a, double* gram, int* fail, cudaStream_t st) {
+static cudaError_t launch_chol_t(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st) {
   auto kern = panel_chol_kernel<B>;
   constexpr size_t smem = CholSmem<B>::BYTES;
-  static int per_sm = -1;
+  static int per_sm = -1, nsm = 0;
   if (per_sm < 0) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, PC_THREADS, smem);
     if (per_sm < 1) per_sm = 1;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   }
-  int nsm = 0, dev = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   const int cap = per_sm * nsm;
-  int G = (int)std::min<int64_t>(cap, (a.m + 127) / 128);
+  // >= 64 rows per CTA (CTA 0 must hold the b top rows); enough CTAs for the smem row cap
+  int G = (int)std::min<int64_t>(cap, a.m / 64);
   if ((int64_t)G * pc_maxr<B>() < a.m) G = (int)((a.m + pc_maxr<B>() - 1) / pc_maxr<B>());
-  if (G > cap) return cudaErrorNotSupported;   // too tall for one pass: caller uses TSQR
-  cudaError_t e = cudaMemsetAsync(gram, 0, sizeof(double) * 3 * PC_NCOPY * B * B, st);
-  if (e != cudaSuccess) return e;
-  void* args[] = {&a, &gram, &fail};
+  if (G > cap || G < 1) return cudaErrorNotSupported;   // caller uses TSQR
+  unsigned char* wsp = (unsigned char*)ws;
+  void* args[] = {&a, &wsp, &launch};
   return cudaLaunchCooperativeKernel((const void*)kern, dim3(G), dim3(PC_THREADS), args, smem, st);
 }
 
-cudaError_t launch_panel_chol(PanelArgs& a, int max_ctas, double* gram, int* fail, cudaStream_t st) {
-  (void)max_ctas;
-  if (a.b <= 32) return launch_chol_t<32>(a, gram, fail, st);
-  return launch_chol_t<64>(a, gram, fail, st);
+cudaError_t launch_panel_chol(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st) {
+  if (a.m < 2 * a.b) return cudaErrorNotSupported;
+  switch (a.b) {
+    case 8: return launch_chol_t<8>(a, ws, launch, st);
+    case 16: return launch_chol_t<16>(a, ws, launch, st);
+    case 32: return launch_chol_t<32>(a, ws, launch, st);
+    case 64: return launch_chol_t<64>(a, ws, launch, st);
+    default: return cudaErrorNotSupported;
+  }
 }
 
 }  // namespace sbr

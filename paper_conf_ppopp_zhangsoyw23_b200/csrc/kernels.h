@@ -43,7 +43,13 @@ PanelWs panel_ws_sizes(int64_t m_max, int b);
 cudaError_t launch_panel(PanelArgs& a, int max_ctas, cudaStream_t st);
 int panel_max_ctas(int b);
 // shifted CholeskyQR3 (fp64) + reconstruction; *fail = 1 (panel untouched) if rank deficient
-cudaError_t launch_panel_chol(PanelArgs& a, int max_ctas, double* gram, int* fail, cudaStream_t st);
+// CholeskyQR panel (k_panel_chol.cu): b in {8,16,32,64}; returns cudaErrorNotSupported when it
+// does not apply (then run TSQR unconditionally).  ws: panel_chol_ws_bytes() bytes, zeroed once
+// at allocation; launch: per-handle launch counter (buffers are double-buffered by its parity).
+// On return the TSQR fallback must be launched with run_if = panel_chol_fail(ws).
+size_t panel_chol_ws_bytes();
+int* panel_chol_fail(void* ws);
+cudaError_t launch_panel_chol(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st);
 
 // ---- SIMT building blocks (fp32) ----
 // C[m1 x n2] (+)= alpha * A[rows x m1]^T B[rows x n2]   (accumulate=1: atomics into C)

@@ -62,8 +62,9 @@ struct sbr_ctx {
   __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr, *Xh = nullptr, *Wrh = nullptr,
          *Bl = nullptr, *Gh = nullptr;
   float* Hb = nullptr;
-  double* gram = nullptr;  // CholeskyQR Gram matrices (3 x 64 x 64)
+  void* chol_ws = nullptr;  // CholeskyQR panel workspace (Gram sets, barrier, LU), zeroed at allocation
   int* pfail = nullptr;
+  unsigned chol_launches = 0;
   int panel_mode = 0;      // 0: CholeskyQR3 + TSQR fallback, 1: TSQR only (SBR_PANEL=tsqr)
   int64_t ldwh = 0, ldsh = 0, ldk = 0, ldbl = 0;
   int panel_ctas = 0;
@@ -160,7 +161,7 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
-               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take((3 * 8 + 3) * 64 * 64 * 2 + 64);
+               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take(panel_chol_ws_bytes() / sizeof(float) + 64);
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
   if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
@@ -203,8 +204,9 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->Bl = (__half*)(base + oBl);
   h->Gh = (__half*)(base + oGh);
   h->Hb = (float*)(base + oHb);
-  h->gram = (double*)(base + oGram);
-  h->pfail = (int*)(h->gram + (3 * 8 + 3) * 64 * 64);
+  h->chol_ws = base + oGram;
+  h->pfail = panel_chol_fail(h->chol_ws);
+  if (cudaMemset(h->chol_ws, 0, panel_chol_ws_bytes()) != cudaSuccess) return SBR_ERR_CUDA;
   h->ldbl = 2 * ldk + 128;
   h->ldwh = ldwh;
   h->ldsh = ldsh;
@@ -334,8 +336,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.ws_r = h->pr;
         pa.ws_q = h->pq;
         pa.ws_misc = h->pmisc;
-        if (h->panel_mode == 0 && m > 512 && m >= 2 * b) {   // CholeskyQR3, TSQR only if it declines
-          const cudaError_t ce = launch_panel_chol(pa, h->panel_ctas, h->gram, h->pfail, st);
+        if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
+          const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
           if (ce == cudaSuccess) {
             pa.run_if = h->pfail;
             h->launches += 1;
@@ -860,8 +862,8 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
   pa.ws_q = h->pq;
   pa.ws_misc = h->pmisc;
   pa.trace = trace_host ? (int64_t*)tr.p : nullptr;
-  if (h->panel_mode == 0 && m > 512 && m >= 2 * b) {
-    const cudaError_t ce = launch_panel_chol(pa, h->panel_ctas, h->gram, h->pfail, st);
+  if (h->panel_mode == 0 && m > 512) {
+    const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
     if (ce == cudaSuccess) pa.run_if = h->pfail;
     else if (ce != cudaErrorNotSupported) SBR_CK(ce, "panel_chol");
   }

@@ -6,7 +6,7 @@ import __graft_entry__; __graft_entry__.build()
 import paper_conf_ppopp_zhangsoyw23_b200 as sbr
 from paper_conf_ppopp_zhangsoyw23_b200 import _lib
 h = sbr.Handle(0)
-names = ["start", "gram0", "sync0", "chol0", "load", "solve0+gram1", "sync1", "chol1", "gram0compute", "solve1+gram2", "sync2", "chol2", "LUloop", "rounds_done", "LU+R", "sync"]
+names = ["start", "loaded", "gram0", "wait0", "chol0", "solve0", "gram1", "LU(cta0)", "wait1", "checked", "LUread", "rows", "x12", "x13", "x14", "x15"]
 for b in (32,):
     for m in (4000, 16000, 32000):
         P0 = torch.randn(b, m, device="cuda")   # column-major m x b
