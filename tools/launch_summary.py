@@ -11,7 +11,7 @@ for r in rows:
     name = d["Kernel Name"].split("(")[0]
     v = float(d["Metric Value"].replace(",", ""))
     unit = d.get("Metric Unit", "nsecond")
-    v = v / 1e3 if unit == "nsecond" else (v if unit == "usecond" else v * 1e3)
+    v = v / 1e3 if unit in ("ns", "nsecond") else (v if unit in ("us", "usecond") else v * 1e3)
     tot[name] += v; cnt[name] += 1
 T = sum(tot.values())
 print(f"total {T/1e3:.2f} ms over {sum(cnt.values())} launches")
