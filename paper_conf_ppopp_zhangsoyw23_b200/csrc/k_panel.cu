@@ -431,6 +431,8 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
       if (i < row0) {
         for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
         if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
+        if (a.Wh) for (int c = 0; c < b; ++c) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
+        if (a.Wrh) for (int c = 0; c < b; ++c) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
         continue;
       }
       const int64_t il = i - row0;
@@ -442,6 +444,8 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
         float w = 0.f;
         for (int k = 0; k <= c; ++k) w = fmaf(Vs[il + k * RSN], T[k + c * LDU], w);
         a.W[i + c * a.ldw] = w;
+        if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(w);
+        if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(w);
       }
     }
     return;
@@ -576,7 +580,11 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
     }
 #pragma unroll
     for (int c = 0; c < B; ++c)
-      if (c < b) a.W[gr + c * a.ldw] = v_[c];
+      if (c < b) {
+        a.W[gr + c * a.ldw] = v_[c];
+        if (a.Wh) a.Wh[gr + c * a.ldwh] = __float2half_rn(v_[c]);
+        if (a.Wrh) a.Wrh[gr * a.ldwrh + c] = __float2half_rn(v_[c]);
+      }
     // y = L_1 row (il < b)  or  y U = q
 #pragma unroll
     for (int c = 0; c < B; ++c) {
@@ -608,6 +616,8 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
   for (int64_t i = tid; i < row0; i += nth) {
     for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
     if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
+    if (a.Wh) for (int c = 0; c < b; ++c) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
+    if (a.Wrh) for (int c = 0; c < b; ++c) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
   }
   PTRACE(9);
 }

@@ -594,6 +594,14 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       }
 #pragma unroll
     for (int c = 0; c < B; ++c) a.W[gr + c * a.ldw] = v_[c];
+    if (a.Wh) {
+#pragma unroll
+      for (int c = 0; c < B; ++c) a.Wh[gr + c * a.ldwh] = __float2half_rn(v_[c]);
+    }
+    if (a.Wrh) {
+#pragma unroll
+      for (int c = 0; c < B; ++c) a.Wrh[gr * a.ldwrh + c] = __float2half_rn(v_[c]);
+    }
     if (il < B) {
 #pragma unroll
       for (int c = 0; c < B; ++c) v_[c] = Lc_[c * B + il];   // L[il][c]
@@ -643,6 +651,8 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     for (int c = 0; c < B; ++c) {
       a.Y[i + c * a.ldy] = 0.f;
       a.W[i + c * a.ldw] = 0.f;
+      if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
+      if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
     }
     if (a.Yh) {
 #pragma unroll

@@ -32,7 +32,8 @@ struct NnCfg {
 template <int BN>
 __global__ void __launch_bounds__(256, 1)
     skinny_nn_kernel(const __grid_constant__ CUtensorMap mapA0, const __grid_constant__ CUtensorMap mapA1,
-                     const __grid_constant__ CUtensorMap mapB, int kc0, int kct, int arow0, int64_t rows, int b,
+                     const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kc0,
+                     int kct, int arow0, int brow0, int64_t rows, int b,
                      const float* Cin, int64_t ldc, float* Dout, int64_t ldd, __half* __restrict__ Hcm, int64_t ldhc,
                      __half* __restrict__ Hrm, int64_t ldhr) {
   using Cfg = NnCfg<BN>;
@@ -64,7 +65,7 @@ __global__ void __launch_bounds__(256, 1)
       const bool second = kc >= kc0;
       const int kin = (second ? kc - kc0 : kc) * 64;
       tma_load_2d(sa, second ? &mapA1 : &mapA0, &full[st], kin, arow0 + tile * 128);
-      tma_load_2d(sa + Cfg::SA, &mapB, &full[st], kc * 64, 0);
+      tma_load_2d(sa + Cfg::SA, second ? &mapB1 : &mapB0, &full[st], kin, second ? 0 : brow0);
       if (++st == Cfg::NS) { st = 0; ph ^= 1; }
     }
   } else if (warp == 1 && lane == 0) {
@@ -131,19 +132,21 @@ static cudaError_t launch_nn_t(const SkinnyNN& p, cudaStream_t st) {
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  CUtensorMap mA0, mA1, mB;
+  CUtensorMap mA0, mA1, mB0, mB1;
   cudaError_t e;
   const int64_t K0 = std::max<int64_t>(p.K0, 1), K1 = std::max<int64_t>(p.K1, 1);
   if ((e = make_tmap_2d(&mA0, p.A0, true, K0, p.a_rows, p.lda, 64, 128)) != cudaSuccess) return e;
   if ((e = make_tmap_2d(&mA1, p.A1 ? p.A1 : p.A0, true, K1, p.a_rows, p.lda, 64, 128)) != cudaSuccess) return e;
-  const int kc0 = (int)((p.K0 + 63) / 64);
-  if ((e = make_tmap_2d(&mB, p.B, true, std::max<int64_t>(kc0 * 64 + p.K1, 1), p.b, p.ldb, 64, BN)) != cudaSuccess)
+  if ((e = make_tmap_2d(&mB0, p.B0, true, K0, p.b0_rows, p.ldb0, 64, BN)) != cudaSuccess) return e;
+  if ((e = make_tmap_2d(&mB1, p.B1 ? p.B1 : p.B0, true, K1, p.B1 ? p.b : p.b0_rows, p.B1 ? p.ldb1 : p.ldb0, 64, BN)) !=
+      cudaSuccess)
     return e;
+  const int kc0 = (int)((p.K0 + 63) / 64);
   const int kct = kc0 + (int)((p.K1 + 63) / 64);
   const int grid = (int)((p.rows + 127) / 128);
   if (grid == 0) return cudaSuccess;
-  kern<<<grid, 256, Cfg::SMEM, st>>>(mA0, mA1, mB, kc0, kct, (int)p.arow0, p.rows, p.b, p.C, p.ldc, p.D, p.ldd, p.Hcm,
-                                     p.ldhc, p.Hrm, p.ldhr);
+  kern<<<grid, 256, Cfg::SMEM, st>>>(mA0, mA1, mB0, mB1, kc0, kct, (int)p.arow0, (int)p.brow0, p.rows, p.b, p.C,
+                                     p.ldc, p.D, p.ldd, p.Hcm, p.ldhc, p.Hrm, p.ldhr);
   return cudaGetLastError();
 }
 
@@ -244,7 +247,7 @@ __global__ void __launch_bounds__(256, 1)
           if (j < K1) {
 #pragma unroll
             for (int c = 0; c < 32; ++c)
-              if (c0 + c < b) atomicAdd(&D[j + (int64_t)(c0 + c) * ldd], v[c]);
+              if (c0 + c < b) atomicAdd(&D[(int64_t)j * ldd + (c0 + c)], v[c]);
           }
         }
       }

@@ -21,6 +21,10 @@ struct PanelArgs {
   int64_t ldw;
   __half* Yh;     // optional fp16 row-major copy of Y (row r, column c at Yh[r*ldyh + c])
   int64_t ldyh;
+  __half* Wh;     // optional fp16 column-major copy of W^0 (Wh[r + c*ldwh]), rows 0 .. M-1
+  int64_t ldwh;
+  __half* Wrh;    // optional fp16 row-major copy of W^0 (Wrh[r*ldwrh + c]), rows 0 .. M-1
+  int64_t ldwrh;
   int64_t row0, M;
   // workspace
   float* ws_v;
@@ -126,11 +130,13 @@ cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st);
 
 // skinny tcgen05 GEMMs (k_skinny_tc.cu)
-struct SkinnyNN {                 // D[rows x b] = C - [A0 | A1] B^T
+struct SkinnyNN {                 // D[rows x b] = C - [A0 | A1] [B0 | B1]^T
   const __half *A0, *A1;          // row-major fp16, K0 / K1 columns used, a_rows x lda
   int64_t K0, K1, a_rows, lda, arow0;
-  const __half* B;                // b x ldb row-major: cols [0,K0) | zero pad to 64*ceil(K0/64) | [.., +K1)
-  int64_t ldb;
+  const __half* B0;               // row-major fp16 (K-major), rows brow0 .. brow0+b-1 of b0_rows, K0 columns
+  int64_t ldb0, b0_rows, brow0;
+  const __half* B1;               // row-major fp16 b x K1 (may be NULL if K1 == 0)
+  int64_t ldb1;
   int64_t rows;
   int b;
   const float* C; int64_t ldc;    // column-major fp32 (may alias D)
@@ -146,10 +152,31 @@ struct SkinnyTN {                 // D0 += A0[rows]^T B[rows], D1 += A1[rows]^T 
   int64_t b_rows, ldb;
   int64_t row0, rows;             // reduction rows [row0, row0+rows)
   int b;
-  float *D0, *D1; int64_t ldd;    // K1 x b, column-major, pre-zeroed
+  float *D0, *D1; int64_t ldd;    // K1 x b, ROW-major (D[j*ldd + c]), pre-zeroed
   int num_sms;
 };
 cudaError_t launch_skinny_tn(const SkinnyTN& p, cudaStream_t st);
+
+// per-panel chain helpers (k_chain.cu)
+// kxb: D[q, p] = C(q, p) - sum_r WtX[q + r*ldwx] B(r, p),  q < k, p < b, r < k.
+//   LAZY  (a5): B(r,p) = Y[(c+p) + r*ldy], C(q,p) = X[(c+p) + q*ldx]  -> Ph[p*ldph + q] = fp16(D)  (P^T)
+//               also mirrors the b x b diagonal block of the master at Adiag.
+//   MERGE (a3): B(r,p) = G[r*b + p],       C(q,p) = H[q*b + p]      -> WtX[q + (k+p)*ldwx] = D and its
+//               mirror WtX[(k+p) + q*ldwx]; also Gh[r + p*ldgh] = fp16(G(r, p)).
+struct KxbArgs {
+  int mode;                       // 0 = LAZY, 1 = MERGE
+  int k, b;
+  float* WtX; int64_t ldwx;
+  const float* Y; int64_t ldy; const float* X; int64_t ldx; int64_t c;   // LAZY
+  __half* Ph; int64_t ldph;
+  float* Adiag; int64_t lda;
+  const float* G; const float* H;                                        // MERGE
+  __half* Gh; int64_t ldgh;
+};
+cudaError_t launch_kxb(const KxbArgs& a, cudaStream_t st);
+// after the pass: Xh[r*ldxh + p] = fp16(X[r + p*ldx]) and WtXtt[i + j*ldw] += sum_r W[r,i] X[r,j]
+cudaError_t launch_postpass(int64_t M, int b, const float* X, int64_t ldx, const float* W, int64_t ldw, __half* Xh,
+                            int64_t ldxh, float* WtXtt, int64_t ldwtx, cudaStream_t st);
 
 // fp16 conversions
 cudaError_t f32cm_to_f16rm(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd,

@@ -62,6 +62,8 @@ struct sbr_ctx {
   __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr, *Xh = nullptr, *Wrh = nullptr,
          *Bl = nullptr, *Gh = nullptr;
   float* Hb = nullptr;
+  float* GH = nullptr;     // per-block G_t / H_t (row-major k x b each, panel t at offset t*nb*b), zeroed per block
+  __half* Ph = nullptr;    // fp16 P^T (b x k, row-major) of the lazy update
   void* chol_ws = nullptr;  // CholeskyQR panel workspace (Gram sets, barrier, LU), zeroed at allocation
   int* pfail = nullptr;
   unsigned chol_launches = 0;
@@ -161,7 +163,8 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
-               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take(panel_chol_ws_bytes() / sizeof(float) + 64);
+               oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take(panel_chol_ws_bytes() / sizeof(float) + 64),
+               oGH = take((size_t)2 * nb * nb), oPh = take((size_t)64 * ldk / 2 + 8);
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
   if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
@@ -205,6 +208,8 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->Gh = (__half*)(base + oGh);
   h->Hb = (float*)(base + oHb);
   h->chol_ws = base + oGram;
+  h->GH = (float*)(base + oGH);
+  h->Ph = (__half*)(base + oPh);
   h->pfail = panel_chol_fail(h->chol_ws);
   if (cudaMemset(h->chol_ws, 0, panel_chol_ws_bytes()) != cudaSuccess) return SBR_ERR_CUDA;
   h->ldbl = 2 * ldk + 128;
@@ -260,6 +265,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, st), "shadow_init");
     h->launches += (n + 65534) / 65535;
   }
+  if (tc16) {  // fp16 W copies: pad columns (b < BN) must read as zero in the pass
+    SBR_CK(cudaMemsetAsync(h->Wh, 0, sizeof(__half) * h->ldwh * 64, st), "zero Wh");
+  }
   for (int64_t c0 = 0; c0 < ncols; c0 += nb) {
     const int64_t r0 = c0 + b, M = n - r0;
     const int kJ = (int)std::min<int64_t>(nb, ncols - c0);
@@ -273,20 +281,42 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
                                cudaMemcpyDeviceToDevice, st),
              "strip copy");
     }
+    if (tc16) {  // block start: X (accumulated by the passes), W^T X (diagonal blocks accumulated), G/H
+      Scope sc(h, SBR_K_OTHER, 4.0 * M * p * b + 4.0 * nb * nb * 3, 0);
+      SBR_CK(zero_matrix(M, (int64_t)p * b, h->Xb, ldn, st), "zero X");
+      SBR_CK(cudaMemsetAsync(h->WtX, 0, sizeof(float) * nb * nb, st), "zero WtX");
+      SBR_CK(cudaMemsetAsync(h->GH, 0, sizeof(float) * 2 * nb * nb, st), "zero G/H");
+    }
     for (int t = 0; t < p; ++t) {
       const int64_t g = c0 + (int64_t)t * b;
       const int64_t tb = (int64_t)t * b;
       const int64_t m = M - tb;
       const int k = t * b;
+      float* Wt = Wb + tb * ldwb;  // this panel's W columns (W_t^0 from the panel, then W_t)
+      float* Gt = h->GH + (size_t)t * nb * b;
+      float* Ht = h->GH + (size_t)nb * nb + (size_t)t * nb * b;
       if (t >= 1) {  // ---- a5: lazy update of panel t's columns (Alg.1 l.8-10)
         const int64_t c = tb - b;  // OA column of the panel's first column
         const int64_t rows = M - c;
         float* Ablk = A + g + g * lda;
-        if (tc16) {  // GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
+        if (tc16) {  // P = W^T R (SIMT), then GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
           Scope sc(h, SBR_K_LAZY, 2.0 * rows * 2.0 * k + 8.0 * rows * b, 4.0 * rows * k * b);
-          SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Yb + c, ldn, true, 1.f, h->Xb + c, ldn, true, h->Pb, k, st), "lazy_p");
-          SBR_CK(build_lazy_b(k, b, h->Yh, h->ldk, c, h->Pb, h->Bl, h->ldbl, st), "lazy_b");
-          SBR_CK(mirror_lower_block(b, Ablk, lda, st), "mirror");
+          KxbArgs ka{};
+          ka.mode = 0;
+          ka.k = k;
+          ka.b = b;
+          ka.WtX = h->WtX;
+          ka.ldwx = nb;
+          ka.Y = h->Yb;
+          ka.ldy = ldn;
+          ka.X = h->Xb;
+          ka.ldx = ldn;
+          ka.c = c;
+          ka.Ph = h->Ph;
+          ka.ldph = h->ldk;
+          ka.Adiag = Ablk;
+          ka.lda = lda;
+          SBR_CK(launch_kxb(ka, st), "lazy P");
           SkinnyNN q{};
           q.A0 = h->Xh;
           q.A1 = h->Yh;
@@ -295,8 +325,12 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           q.a_rows = M;
           q.lda = h->ldk;
           q.arow0 = c;
-          q.B = h->Bl;
-          q.ldb = h->ldbl;
+          q.B0 = h->Yh;
+          q.ldb0 = h->ldk;
+          q.b0_rows = M;
+          q.brow0 = c;
+          q.B1 = h->Ph;
+          q.ldb1 = h->ldk;
           q.rows = rows;
           q.b = b;
           q.C = Ablk;
@@ -304,7 +338,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           q.D = Ablk;
           q.ldd = lda;
           SBR_CK(launch_skinny_nn(q, st), "lazy_nn");
-          h->launches += 4;
+          h->launches += 2;
         } else {
           Scope sc(h, SBR_K_LAZY, 4.0 * rows * (2.0 * k + 2 * b), 4.0 * rows * k * b);
           SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Yb + c, ldn, true, 1.f, h->Xb + c, ldn, true, h->Pb, k, st), "lazy_p");
@@ -325,12 +359,16 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.b = b;
         pa.Y = h->Yb + tb * ldn;
         pa.ldy = ldn;
-        pa.W = Wb + tb * ldwb;
+        pa.W = Wt;
         pa.ldw = ldwb;
         pa.row0 = tb;
         pa.M = M;
         pa.Yh = tc16 ? h->Yh + tb : nullptr;
         pa.ldyh = h->ldk;
+        pa.Wh = tc16 ? h->Wh : nullptr;        // W^0 (fp16, column-major): pass operand / merge B
+        pa.ldwh = h->ldwh;
+        pa.Wrh = (tc16 && t == 0) ? h->Wrh : nullptr;   // W_0 = W^0 (row-major): later merges
+        pa.ldwrh = h->ldk;
         pa.ws_v = h->pv;
         pa.ws_tau = h->ptau;
         pa.ws_r = h->pr;
@@ -348,17 +386,12 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
         h->launches += 1;
       }
-      float* Wt = Wb + tb * ldwb;  // this panel's W columns (W_t^0 from the panel, then W_t)
       if (tc16) {
-        // ---- a3 on tcgen05: G = Y^T W0, H = X^T W0 (one pass over Y, X); W^T X_t = H - (W^T X) G;
-        //      W_t = W0 - W G, written as fp32 + fp16 (column-major for the pass, row-major for later merges)
-        Scope sc(h, SBR_K_WMERGE, t >= 1 ? (2.0 * (M - tb) * 2.0 * k + 2.0 * M * k + 12.0 * M * b) : 6.0 * M * b,
-                 t >= 1 ? 2.0 * (2.0 * (M - tb) + M) * k * b : 0.0);
-        const int bn = pass_bn(b);
-        SBR_CK(to_half_cm(M, b, bn, Wt, ldwb, h->Wh, h->ldwh, st), "W0 -> fp16");
         if (t >= 1) {
-          SBR_CK(zero_matrix(k, b, h->Gb, k, st), "zero G");
-          SBR_CK(zero_matrix(k, b, h->Hb, k, st), "zero H");
+          // ---- a3 on tcgen05: G = Y^T W0, H = X^T W0 (one pass over Y, X); W^T X_t = H - (W^T X) G;
+          //      W_t = W0 - W G, written as fp32 + fp16 (column-major for the pass, row-major for later merges)
+          Scope sc(h, SBR_K_WMERGE, 2.0 * (M - tb) * 2.0 * k + 2.0 * M * k + 12.0 * M * b,
+                   2.0 * (2.0 * (M - tb) + M) * k * b);
           SkinnyTN q{};
           q.A0 = h->Yh;
           q.A1 = h->Xh;
@@ -371,16 +404,22 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           q.row0 = tb;
           q.rows = M - tb;
           q.b = b;
-          q.D0 = h->Gb;
-          q.D1 = h->Hb;
-          q.ldd = k;
+          q.D0 = Gt;
+          q.D1 = Ht;
+          q.ldd = b;
           q.num_sms = h->nsm;
           SBR_CK(launch_skinny_tn(q, st), "Y^T W0, X^T W0");
-          // W^T X_t (rows < k) = H - (W^T X) G  (symmetry of OA: W_{<t}^T OA W_t = X_{<t}^T W_t)
-          SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Gb, k, false, 1.f, h->Hb, k, false, h->WtX + tb * nb, nb, st),
-                 "WtX col");
-          SBR_CK(mirror_wtx(k, b, h->WtX, nb, st), "mirror wtx");
-          SBR_CK(to_half_cm(k, b, b, h->Gb, k, h->Gh, k, st), "G -> fp16");
+          KxbArgs ka{};
+          ka.mode = 1;
+          ka.k = k;
+          ka.b = b;
+          ka.WtX = h->WtX;
+          ka.ldwx = nb;
+          ka.G = Gt;
+          ka.H = Ht;
+          ka.Gh = h->Gh;
+          ka.ldgh = h->ldk;
+          SBR_CK(launch_kxb(ka, st), "W^T X_t, G -> fp16");
           SkinnyNN mq{};
           mq.A0 = h->Wrh;
           mq.A1 = nullptr;
@@ -389,8 +428,11 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           mq.a_rows = M;
           mq.lda = h->ldk;
           mq.arow0 = 0;
-          mq.B = h->Gh;
-          mq.ldb = k;
+          mq.B0 = h->Gh;
+          mq.ldb0 = h->ldk;
+          mq.b0_rows = b;
+          mq.brow0 = 0;
+          mq.B1 = nullptr;
           mq.rows = M;
           mq.b = b;
           mq.C = Wt;
@@ -402,12 +444,36 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           mq.Hrm = h->Wrh + tb;
           mq.ldhr = h->ldk;
           SBR_CK(launch_skinny_nn(mq, st), "W merge");
-          h->launches += 6;
-        } else {
-          SBR_CK(f32cm_to_f16rm(M, b, Wt, ldwb, h->Wrh, h->ldk, st), "W -> fp16 rm");
-          h->launches += 2;
+          h->launches += 3;
         }
-      } else if (t >= 1) {  // ---- a3 (SIMT fp32): W merge
+        {  // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA); X_t zeroed at block start
+          Scope sc(h, SBR_K_PASS, 1.0 * M * M + 6.0 * M * b, 2.0 * M * M * b);
+          PassLaunch pl{};
+          pl.shadow = h->Sh;
+          pl.n = n;
+          pl.ld_shadow = h->ldsh;
+          pl.Wh = h->Wh;
+          pl.M = M;
+          pl.ld_wh = h->ldwh;
+          pl.r0 = r0;
+          pl.b = b;
+          pl.X = h->Xb + tb * ldn;
+          pl.ldx = ldn;
+          pl.num_sms = h->nsm;
+          pl.seg_rows = 8;
+          SBR_CK(launch_pass_tc(pl, st), "pass_tc");
+          h->launches += 1;
+        }
+        {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block)
+          Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
+          SBR_CK(launch_postpass(M, b, h->Xb + tb * ldn, ldn, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb,
+                                 st),
+                 "postpass");
+          h->launches += 1;
+        }
+        continue;
+      }
+      if (t >= 1) {  // ---- a3 (SIMT fp32): W merge
         Scope sc(h, SBR_K_WMERGE, 4.0 * (M - tb) * (k + b) + 4.0 * M * (k + 2 * b), 2.0 * (2.0 * M - tb) * k * b);
         SBR_CK(zero_matrix(k, b, h->Gb, k, st), "zero G");
         SBR_CK(gemm_tn(M - tb, k, b, 1.f, h->Yb + tb, ldn, Wb + tb + tb * ldwb, ldwb, h->Gb, k, st), "Y^T W0");
@@ -416,36 +482,13 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
                "W merge");
         h->launches += 2;
       }
-      if (tc16) {  // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA)
-        Scope sc(h, SBR_K_PASS, 1.0 * M * M + 6.0 * M * b, 2.0 * M * M * b);
-        SBR_CK(zero_matrix(M, b, h->Xb + tb * ldn, ldn, st), "zero X");
-        PassLaunch pl{};
-        pl.shadow = h->Sh;
-        pl.n = n;
-        pl.ld_shadow = h->ldsh;
-        pl.Wh = h->Wh;
-        pl.M = M;
-        pl.ld_wh = h->ldwh;
-        pl.r0 = r0;
-        pl.b = b;
-        pl.X = h->Xb + tb * ldn;
-        pl.ldx = ldn;
-        pl.num_sms = h->nsm;
-        pl.seg_rows = 8;
-        SBR_CK(launch_pass_tc(pl, st), "pass_tc");
-        h->launches += 2;
-      } else {  // ---- a4 (3xTF32 mode, SIMT fp32 for now): OA frozen = A + strip copy
+      {  // ---- a4 (3xTF32 mode, SIMT fp32 for now): OA frozen = A + strip copy
         Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 8.0 * M * b, 2.0 * M * M * b);
         SBR_CK(sym_pass(M, b, OA, lda, h->Strip, ldn, sw, Wb + tb * ldwb, ldwb, h->Xb + tb * ldn, ldn, st),
                "pass");
         h->launches += 1;
       }
-      if (tc16) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b)
-        Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
-        SBR_CK(f32cm_to_f16rm(M, b, h->Xb + tb * ldn, ldn, h->Xh + tb, h->ldk, st), "X -> fp16");
-        SBR_CK(tn_small(M, b, Wt, ldwb, h->Xb + tb * ldn, ldn, h->WtX + tb + tb * nb, nb, st), "Wt^T Xt");
-        h->launches += 2;
-      } else {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
+      {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
         Scope sc(h, SBR_K_WMERGE, 4.0 * M * (k + 2 * b), 2.0 * M * (k + b) * b);
         SBR_CK(zero_matrix(k + b, b, h->WtX + tb * nb, nb, st), "zero wtx");
         SBR_CK(gemm_tn(M, k + b, b, 1.f, Wb, ldwb, h->Xb + tb * ldn, ldn, h->WtX + tb * nb, nb, st), "W^T X");
