@@ -6,9 +6,8 @@
 // The shadow stores the strict lower triangle, HALF the diagonal and zeros above it,
 // so a diagonal tile contributes T W + T^T W = L W with no special case.
 //
-// Work item = (tile-column group of C tiles, segment of tile rows).  One CTA (persistent,
-// 1 per SM) per item stream: TMA producer warp -> single-thread MMA warp -> 4 epilogue
-// warps.  Row accumulators (X_I, double-buffered) and the C column accumulators (X_J)
+// Work = a balanced contiguous range of lower tiles per CTA (PassWalk).  One CTA per SM:
+// TMA producer warp -> single-thread MMA warp -> 4 epilogue warps.  Row accumulators (X_I, double-buffered) and the C column accumulators (X_J)
 // live in TMEM; they are flushed with fp32 reductions into the L2-resident X.
 // Roofline: HBM-bound (2 bytes per stored element, 4 flops/byte at b = 32).
 #include "kernels.h"
@@ -33,24 +32,75 @@ struct PassCfg {
                                    : TMEM_USED <= 256 ? 256 : 512;
 };
 
-// item index -> (group g, tile rows [i0, i1)): group g spans tile columns [gC, gC+C) and
-// rows gC .. NT-1, cut into segments of SEG rows.
-template <int C>
-SBR_DEV int4 pass_item(int it, int NT, int SEG) {
-  for (int g = 0;; ++g) {
-    const int cnt = (NT - g * C + SEG - 1) / SEG;
-    if (it < cnt) {
-      const int i0 = g * C + it * SEG;
-      return make_int4(g, i0, min(NT, i0 + SEG), 0);
-    }
-    it -= cnt;
+// Work = the lower tiles of OA in the linear order (group g, tile row I, tile column J):
+// group g spans tile columns [gC, gC + ceff), rows I = gC .. NT-1, row I holding
+// min(ceff, I - gC + 1) tiles.  Every CTA takes an equal contiguous range of tiles
+// (balanced to one tile), so a launch ends when the slowest SM has streamed T/grid tiles.
+// The three roles walk the same range with this iterator.
+struct PassWalk {
+  int NT, C;
+  int g, J0, ceff, I, J;
+  int64_t left;
+  bool gfirst, rfirst;
+  SBR_DEV int jend() const { return min(J0 + ceff, I + 1); }
+  SBR_DEV static int64_t group_tiles(int NT, int C, int g) {
+    const int J0 = g * C, ce = min(C, NT - J0);
+    return (int64_t)ce * (ce + 1) / 2 + (int64_t)(NT - J0 - ce) * ce;
   }
-}
+  SBR_DEV void start(int NT_, int C_, int64_t t0, int64_t count) {
+    NT = NT_;
+    C = C_;
+    left = count;
+    g = 0;
+    for (;;) {
+      const int64_t gt = group_tiles(NT, C, g);
+      if (t0 < gt) break;
+      t0 -= gt;
+      ++g;
+    }
+    J0 = g * C;
+    ceff = min(C, NT - J0);
+    const int64_t tri = (int64_t)ceff * (ceff + 1) / 2;
+    if (t0 < tri) {
+      int d = 0;
+      while ((int64_t)(d + 1) * (d + 2) / 2 <= t0) ++d;
+      I = J0 + d;
+      J = J0 + (int)(t0 - (int64_t)d * (d + 1) / 2);
+    } else {
+      const int64_t o = t0 - tri;
+      I = J0 + ceff + (int)(o / ceff);
+      J = J0 + (int)(o % ceff);
+    }
+    gfirst = rfirst = true;
+  }
+  SBR_DEV bool valid() const { return left > 0; }
+  SBR_DEV bool rlast() const { return left == 1 || J + 1 == jend(); }
+  SBR_DEV bool glast() const { return left == 1 || (J + 1 == jend() && I + 1 == NT); }
+  SBR_DEV void next() {
+    --left;
+    gfirst = rfirst = false;
+    if (J + 1 < jend()) {
+      ++J;
+      return;
+    }
+    rfirst = true;
+    if (I + 1 < NT) {
+      ++I;
+      J = J0;
+      return;
+    }
+    gfirst = true;
+    ++g;
+    J0 = g * C;
+    ceff = min(C, NT - J0);
+    I = J = J0;
+  }
+};
 
 template <int BN, int C, int NS>
 __global__ void __launch_bounds__(256, 1)
     pass_tc_kernel(const __grid_constant__ CUtensorMap mapL, const __grid_constant__ CUtensorMap mapW, int r0, int M,
-                   int NT, int SEG, int nitems, int b, float* X, int64_t ldx) {
+                   int NT, int64_t T, int b, float* X, int64_t ldx) {
   using Cfg = PassCfg<BN, C, NS>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -71,6 +121,7 @@ __global__ void __launch_bounds__(256, 1)
   uint32_t* tmem_slot = (uint32_t*)(bars + Cfg::NBAR);
 
   const int warp = warp_id(), lane = lane_id();
+  const int64_t t_beg = (int64_t)blockIdx.x * T / gridDim.x, t_end = (int64_t)(blockIdx.x + 1) * T / gridDim.x;
   if (threadIdx.x == 0) {
     for (int i = 0; i < NS; ++i) { mbar_init(&l_full[i], 1); mbar_init(&l_empty[i], 1); }
     for (int i = 0; i < 2; ++i) {
@@ -89,6 +140,7 @@ __global__ void __launch_bounds__(256, 1)
   const uint32_t tmem = *tmem_slot;
   const uint32_t t_col = tmem;                 // C column accumulators: cols [jj*BN, jj*BN+BN)
   const uint32_t t_row = tmem + C * BN;        // 2 row accumulators
+  PassWalk w;
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
@@ -96,33 +148,31 @@ __global__ void __launch_bounds__(256, 1)
       int st = 0; uint32_t ph = 0;            // L ring
       int ws = 0; uint32_t wph = 0;           // W_I ring
       uint32_t jph = 0;
-      for (int it = blockIdx.x; it < nitems; it += gridDim.x) {
-        const int4 item = pass_item<C>(it, NT, SEG);
-        const int J0 = item.x * C, i0 = item.y, i1 = item.z;
-        const int ceff = min(C, NT - J0);
-        mbar_wait(wj_empty, jph ^ 1);
-        jph ^= 1;
-        mbar_expect_tx(wj_full, ceff * Cfg::WT);
-        for (int jj = 0; jj < ceff; ++jj)
-          for (int h = 0; h < 2; ++h)
-            tma_load_2d(sWj + jj * Cfg::WT + h * (Cfg::WT / 2), &mapW, wj_full, (J0 + jj) * 128 + h * 64, 0);
-        for (int I = i0; I < i1; ++I) {
+      for (w.start(NT, C, t_beg, t_end - t_beg); w.valid(); w.next()) {
+        if (w.gfirst) {
+          mbar_wait(wj_empty, jph ^ 1);
+          jph ^= 1;
+          mbar_expect_tx(wj_full, w.ceff * Cfg::WT);
+          for (int jj = 0; jj < w.ceff; ++jj)
+            for (int h = 0; h < 2; ++h)
+              tma_load_2d(sWj + jj * Cfg::WT + h * (Cfg::WT / 2), &mapW, wj_full, (w.J0 + jj) * 128 + h * 64, 0);
+        }
+        if (w.rfirst) {
           mbar_wait(&wi_empty[ws], wph ^ 1);
           mbar_expect_tx(&wi_full[ws], Cfg::WT);
           for (int h = 0; h < 2; ++h)
-            tma_load_2d(sWi + ws * Cfg::WT + h * (Cfg::WT / 2), &mapW, &wi_full[ws], I * 128 + h * 64, 0);
+            tma_load_2d(sWi + ws * Cfg::WT + h * (Cfg::WT / 2), &mapW, &wi_full[ws], w.I * 128 + h * 64, 0);
+        }
+        mbar_wait(&l_empty[st], ph ^ 1);
+        mbar_expect_tx(&l_full[st], Cfg::LT);
+        uint8_t* dst = sL + st * Cfg::LT;
+        for (int rb = 0; rb < 2; ++rb)
+          for (int cb = 0; cb < 2; ++cb)
+            tma_load_2d(dst + (rb * 2 + cb) * 8192, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64,
+                        r0 + w.J * 128 + cb * 64);
+        if (++st == NS) { st = 0; ph ^= 1; }
+        if (w.rlast()) {
           if (++ws == 2) { ws = 0; wph ^= 1; }
-          const int jend = min(J0 + ceff, I + 1);
-          for (int J = J0; J < jend; ++J) {
-            mbar_wait(&l_empty[st], ph ^ 1);
-            mbar_expect_tx(&l_full[st], Cfg::LT);
-            uint8_t* dst = sL + st * Cfg::LT;
-            for (int rb = 0; rb < 2; ++rb)
-              for (int cb = 0; cb < 2; ++cb)
-                tma_load_2d(dst + (rb * 2 + cb) * 8192, &mapL, &l_full[st], r0 + I * 128 + rb * 64,
-                            r0 + J * 128 + cb * 64);
-            if (++st == NS) { st = 0; ph ^= 1; }
-          }
         }
       }
     }
@@ -136,52 +186,56 @@ __global__ void __launch_bounds__(256, 1)
       int rb = 0; uint32_t rph = 0;
       uint32_t jph = 0, cph = 0;
       const uint32_t aL = smem_u32(sL), aWj = smem_u32(sWj), aWi = smem_u32(sWi);
-      for (int it = blockIdx.x; it < nitems; it += gridDim.x) {
-        const int4 item = pass_item<C>(it, NT, SEG);
-        const int J0 = item.x * C, i0 = item.y, i1 = item.z;
-        const int ceff = min(C, NT - J0);
-        mbar_wait(wj_full, jph);
-        jph ^= 1;
-        mbar_wait(cacc_empty, cph ^ 1);
-        cph ^= 1;
-        tc_fence_after();
-        uint32_t cinit = 0;
-        for (int I = i0; I < i1; ++I) {
+      uint32_t cinit = 0;
+      bool rowfirst = true;
+      for (w.start(NT, C, t_beg, t_end - t_beg); w.valid(); w.next()) {
+        if (w.gfirst) {
+          mbar_wait(wj_full, jph);
+          jph ^= 1;
+          mbar_wait(cacc_empty, cph ^ 1);
+          cph ^= 1;
+          tc_fence_after();
+          cinit = 0;
+        }
+        if (w.rfirst) {
           mbar_wait(&wi_full[ws], wph);
           mbar_wait(&racc_empty[rb], rph ^ 1);
           tc_fence_after();
-          const uint32_t d_row = t_row + rb * BN;
-          const int jend = min(J0 + ceff, I + 1);
-          for (int J = J0; J < jend; ++J) {
-            const int jj = J - J0;
-            mbar_wait(&l_full[st], ph);
-            tc_fence_after();
-            const uint32_t lt = aL + st * Cfg::LT;
+          rowfirst = true;
+        }
+        const uint32_t d_row = t_row + rb * BN;
+        const int jj = w.J - w.J0;
+        mbar_wait(&l_full[st], ph);
+        tc_fence_after();
+        const uint32_t lt = aL + st * Cfg::LT;
 #pragma unroll
-            for (int s = 0; s < 8; ++s) {  // X_I += L W_J : A MN-major (LBO = 16 KB between 64-row atoms)
-              const uint64_t a = sdesc_sw128(lt + (s >> 2) * 8192 + (s & 3) * 2048, 16384, 1024);
-              const uint64_t bd = sdesc_sw128(aWj + jj * Cfg::WT + (s >> 2) * (Cfg::WT / 2) + (s & 3) * 32, 16, 1024);
-              mma_f16(d_row, a, bd, idesc_dir, (J > J0 || s > 0) ? 1u : 0u);
-            }
-            const uint32_t d_col = t_col + jj * BN;
-            const uint32_t acc0 = (cinit >> jj) & 1u;
+        for (int s = 0; s < 8; ++s) {  // X_I += L W_J : A MN-major (LBO = 16 KB between 64-row atoms)
+          const uint64_t a = sdesc_sw128(lt + (s >> 2) * 8192 + (s & 3) * 2048, 16384, 1024);
+          const uint64_t bd = sdesc_sw128(aWj + jj * Cfg::WT + (s >> 2) * (Cfg::WT / 2) + (s & 3) * 32, 16, 1024);
+          mma_f16(d_row, a, bd, idesc_dir, (!rowfirst || s > 0) ? 1u : 0u);
+        }
+        const uint32_t d_col = t_col + jj * BN;
+        const uint32_t acc0 = (cinit >> jj) & 1u;
 #pragma unroll
-            for (int s = 0; s < 8; ++s) {  // X_J += L^T W_I : A K-major (same bytes)
-              const uint64_t a = sdesc_sw128(lt + (s >> 2) * 16384 + (s & 3) * 32, 16, 1024);
-              const uint64_t bd = sdesc_sw128(aWi + ws * Cfg::WT + (s >> 2) * (Cfg::WT / 2) + (s & 3) * 32, 16, 1024);
-              mma_f16(d_col, a, bd, idesc_tr, (acc0 || s > 0) ? 1u : 0u);
-            }
-            cinit |= 1u << jj;
-            mma_commit(&l_empty[st]);
-            if (++st == NS) { st = 0; ph ^= 1; }
-          }
+        for (int s = 0; s < 8; ++s) {  // X_J += L^T W_I : A K-major (same bytes)
+          const uint64_t a = sdesc_sw128(lt + (s >> 2) * 16384 + (s & 3) * 32, 16, 1024);
+          const uint64_t bd = sdesc_sw128(aWi + ws * Cfg::WT + (s >> 2) * (Cfg::WT / 2) + (s & 3) * 32, 16, 1024);
+          mma_f16(d_col, a, bd, idesc_tr, (acc0 || s > 0) ? 1u : 0u);
+        }
+        cinit |= 1u << jj;
+        rowfirst = false;
+        mma_commit(&l_empty[st]);
+        if (++st == NS) { st = 0; ph ^= 1; }
+        if (w.rlast()) {
           mma_commit(&racc_full[rb]);
           mma_commit(&wi_empty[ws]);
           if (++ws == 2) { ws = 0; wph ^= 1; }
           if (++rb == 2) { rb = 0; rph ^= 1; }
         }
-        mma_commit(cacc_full);
-        mma_commit(wj_empty);
+        if (w.glast()) {
+          mma_commit(cacc_full);
+          mma_commit(wj_empty);
+        }
       }
     }
   } else if (warp >= 4) {
@@ -191,14 +245,14 @@ __global__ void __launch_bounds__(256, 1)
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     int rb = 0; uint32_t rph = 0;
     uint32_t cph = 0;
-    for (int it = blockIdx.x; it < nitems; it += gridDim.x) {
-      const int4 item = pass_item<C>(it, NT, SEG);
-      const int J0 = item.x * C, i0 = item.y, i1 = item.z;
-      const int ceff = min(C, NT - J0);
-      for (int I = i0; I < i1; ++I) {
+    uint32_t touched = 0;
+    for (w.start(NT, C, t_beg, t_end - t_beg); w.valid(); w.next()) {
+      if (w.gfirst) touched = 0;
+      touched |= 1u << (w.J - w.J0);
+      if (w.rlast()) {
         mbar_wait(&racc_full[rb], rph);
         tc_fence_after();
-        const int64_t row = (int64_t)I * 128 + row_in_tile;
+        const int64_t row = (int64_t)w.I * 128 + row_in_tile;
 #pragma unroll
         for (int c0 = 0; c0 < BN; c0 += 32) {
           float v[32];
@@ -213,25 +267,27 @@ __global__ void __launch_bounds__(256, 1)
         mbar_arrive(&racc_empty[rb]);
         if (++rb == 2) { rb = 0; rph ^= 1; }
       }
-      mbar_wait(cacc_full, cph);
-      cph ^= 1;
-      tc_fence_after();
-      for (int jj = 0; jj < ceff; ++jj) {
-        if (i1 - 1 < J0 + jj) continue;           // no tile of this column in the segment
-        const int64_t row = (int64_t)(J0 + jj) * 128 + row_in_tile;
+      if (w.glast()) {
+        mbar_wait(cacc_full, cph);
+        cph ^= 1;
+        tc_fence_after();
+        for (int jj = 0; jj < w.ceff; ++jj) {
+          if (!((touched >> jj) & 1u)) continue;
+          const int64_t row = (int64_t)(w.J0 + jj) * 128 + row_in_tile;
 #pragma unroll
-        for (int c0 = 0; c0 < BN; c0 += 32) {
-          float v[32];
-          tmem_ld32(t_col + jj * BN + c0 + lane_off, v);
-          if (row < M) {
+          for (int c0 = 0; c0 < BN; c0 += 32) {
+            float v[32];
+            tmem_ld32(t_col + jj * BN + c0 + lane_off, v);
+            if (row < M) {
 #pragma unroll
-            for (int c = 0; c < 32; ++c)
-              if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
+              for (int c = 0; c < 32; ++c)
+                if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
+            }
           }
         }
+        tc_fence_before();
+        mbar_arrive(cacc_empty);
       }
-      tc_fence_before();
-      mbar_arrive(cacc_empty);
     }
   }
   tc_fence_before();
@@ -260,11 +316,13 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   if (e != cudaSuccess) return e;
   const int NT = (int)((p.M + 127) / 128);
   const int G = (NT + C - 1) / C;
-  const int SEG = p.seg_rows > 0 ? p.seg_rows : 8;
-  int nitems = 0;
-  for (int g = 0; g < G; ++g) nitems += (NT - g * C + SEG - 1) / SEG;
-  const int grid = std::min(nitems, p.num_sms);
-  kern<<<grid, 256, Cfg::SMEM, st>>>(mapL, mapW, (int)p.r0, (int)p.M, NT, SEG, nitems, p.b, p.X, p.ldx);
+  int64_t T = 0;
+  for (int g = 0; g < G; ++g) {
+    const int J0 = g * C, ce = std::min(C, NT - J0);
+    T += (int64_t)ce * (ce + 1) / 2 + (int64_t)(NT - J0 - ce) * ce;
+  }
+  const int grid = (int)std::min<int64_t>(T, p.num_sms);
+  kern<<<grid, 256, Cfg::SMEM, st>>>(mapL, mapW, (int)p.r0, (int)p.M, NT, T, p.b, p.X, p.ldx);
   return cudaGetLastError();
 }
 

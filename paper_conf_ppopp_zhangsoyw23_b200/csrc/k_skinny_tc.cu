@@ -247,7 +247,7 @@ __global__ void __launch_bounds__(256, 1)
           if (j < K1) {
 #pragma unroll
             for (int c = 0; c < 32; ++c)
-              if (c0 + c < b) atomicAdd(&D[(int64_t)j * ldd + (c0 + c)], v[c]);
+              if (c0 + c < b) atomicAdd(&D[j + (int64_t)(c0 + c) * ldd], v[c]);
           }
         }
       }

@@ -152,7 +152,7 @@ struct SkinnyTN {                 // D0 += A0[rows]^T B[rows], D1 += A1[rows]^T 
   int64_t b_rows, ldb;
   int64_t row0, rows;             // reduction rows [row0, row0+rows)
   int b;
-  float *D0, *D1; int64_t ldd;    // K1 x b, ROW-major (D[j*ldd + c]), pre-zeroed
+  float *D0, *D1; int64_t ldd;    // K1 x b, column-major, pre-zeroed
   int num_sms;
 };
 cudaError_t launch_skinny_tn(const SkinnyTN& p, cudaStream_t st);
@@ -161,7 +161,7 @@ cudaError_t launch_skinny_tn(const SkinnyTN& p, cudaStream_t st);
 // kxb: D[q, p] = C(q, p) - sum_r WtX[q + r*ldwx] B(r, p),  q < k, p < b, r < k.
 //   LAZY  (a5): B(r,p) = Y[(c+p) + r*ldy], C(q,p) = X[(c+p) + q*ldx]  -> Ph[p*ldph + q] = fp16(D)  (P^T)
 //               also mirrors the b x b diagonal block of the master at Adiag.
-//   MERGE (a3): B(r,p) = G[r*b + p],       C(q,p) = H[q*b + p]      -> WtX[q + (k+p)*ldwx] = D and its
+//   MERGE (a3): B(r,p) = G[r + p*ldg],     C(q,p) = H[q + p*ldg]    -> WtX[q + (k+p)*ldwx] = D and its
 //               mirror WtX[(k+p) + q*ldwx]; also Gh[r + p*ldgh] = fp16(G(r, p)).
 struct KxbArgs {
   int mode;                       // 0 = LAZY, 1 = MERGE
@@ -170,7 +170,7 @@ struct KxbArgs {
   const float* Y; int64_t ldy; const float* X; int64_t ldx; int64_t c;   // LAZY
   __half* Ph; int64_t ldph;
   float* Adiag; int64_t lda;
-  const float* G; const float* H;                                        // MERGE
+  const float* G; const float* H; int64_t ldg;                           // MERGE
   __half* Gh; int64_t ldgh;
 };
 cudaError_t launch_kxb(const KxbArgs& a, cudaStream_t st);

@@ -62,7 +62,7 @@ struct sbr_ctx {
   __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr, *Xh = nullptr, *Wrh = nullptr,
          *Bl = nullptr, *Gh = nullptr;
   float* Hb = nullptr;
-  float* GH = nullptr;     // per-block G_t / H_t (row-major k x b each, panel t at offset t*nb*b), zeroed per block
+  float* GH = nullptr;     // per-block G_t / H_t (k x b, ld nb, panel t at offset t*nb*b), zeroed per block
   __half* Ph = nullptr;    // fp16 P^T (b x k, row-major) of the lazy update
   void* chol_ws = nullptr;  // CholeskyQR panel workspace (Gram sets, barrier, LU), zeroed at allocation
   int* pfail = nullptr;
@@ -157,9 +157,13 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oPr = take(pw.r), oPq = take(pw.q), oPm = take(pw.misc), oF = take(64);
   // fp16 operands of the tensor-core path (sizes in floats = halves / 2)
   const int64_t ldwh = (M + 7) / 8 * 8;       // TMA strides must be multiples of 16 bytes
-  const int64_t ldsh = (n + 7) / 8 * 8;
+  // fp16 shadow: ld a multiple of 128 and a row offset `shoff` chosen so that every block's OA
+  // origin (row/col c0 + b, c0 = J*nb) starts on a 256-byte boundary -- the pass streams
+  // 128x128 tiles of it and unaligned tiles drag in neighbouring lines (L2 256 B promotion).
+  const int64_t shoff = (nb % 128 == 0 && (128 - b % 128) % 8 == 0) ? (128 - b % 128) % 128 : 0;
+  const int64_t ldsh = (n + shoff + 127) / 128 * 128;
   const int64_t ldk = (nb + 7) / 8 * 8;
-  const size_t oSh = take((size_t)ldsh * n / 2 + 8), oYh = take((size_t)n * ldk / 2 + 8),
+  const size_t oSh = take(((size_t)ldsh * n + shoff) / 2 + 128), oYh = take((size_t)n * ldk / 2 + 8),
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
@@ -197,7 +201,7 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->pq = (float*)(base + oPq);
   h->pmisc = (float*)(base + oPm);
   h->flag = (unsigned*)(base + oF);
-  h->Sh = (__half*)(base + oSh);
+  h->Sh = (__half*)(base + oSh) + shoff;
   h->Yh = (__half*)(base + oYh);
   h->Zh = (__half*)(base + oZh);
   h->Wh = (__half*)(base + oWh);
@@ -406,7 +410,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           q.b = b;
           q.D0 = Gt;
           q.D1 = Ht;
-          q.ldd = b;
+          q.ldd = nb;
           q.num_sms = h->nsm;
           SBR_CK(launch_skinny_tn(q, st), "Y^T W0, X^T W0");
           KxbArgs ka{};
@@ -417,6 +421,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           ka.ldwx = nb;
           ka.G = Gt;
           ka.H = Ht;
+          ka.ldg = nb;
           ka.Gh = h->Gh;
           ka.ldgh = h->ldk;
           SBR_CK(launch_kxb(ka, st), "W^T X_t, G -> fp16");
