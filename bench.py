@@ -9,11 +9,12 @@ over one synthetic n x n input resident in HBM.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
-One process per GPU (torchrun for N>1).  The reduction of one matrix does not
-shard in this round: N>1 runs N independent replicas
-(weak scaling, no data-path collective), each rank timing its own steps; the
-max over ranks is reported.  ``--impl reference`` times the CPU oracle (this tier
-has no reference implementation; the oracle is the reference arm).
+One process per GPU (torchrun for N>1).  N>1 reduces ONE matrix across the ranks with
+sbr_reduce_dist (strong scaling, "scaling": "strong"): the per-panel pass is sharded by
+lower tiles with an NCCL broadcast of W_t and all-reduce of X_t per panel (DESIGN.md
+"Multi-GPU"); every rank times its own steps and the max over ranks is reported.
+``--impl reference`` times the CPU oracle (this tier has no reference implementation; the
+oracle is the reference arm).
 """
 from __future__ import annotations
 
@@ -43,6 +44,7 @@ def parse():
     p.add_argument("--nb", type=int, default=CONFIG4["nb"])
     p.add_argument("--mode", default=CONFIG4["mode"])
     p.add_argument("--e2e-steps", type=int, default=2)
+    p.add_argument("--profile-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-sample-s", type=float, default=15.0)
     return p.parse_args()
@@ -234,22 +236,35 @@ def main():
     n, b, nb, mode = args.n, args.b, args.nb, args.mode
     seed = workloads.config_seed(4)
     stream = torch.cuda.current_stream()
-    h = sbr.Handle(local, stream)
+    if world > 1:
+        # one matrix across the ranks (sbr_reduce_dist, strong scaling): NCCL communicator
+        # from a unique id that rank 0 creates and torch.distributed carries
+        uid = [sbr.get_unique_id() if rank == 0 else None]
+        torch.distributed.broadcast_object_list(uid, src=0)
+        h = sbr.Handle(local, stream, unique_id=uid[0], rank=rank, nranks=world)
+    else:
+        h = sbr.Handle(local, stream)
     pristine = h.generate_symmetric(seed, n)              # device twin of workloads.random_symmetric
     a = torch.empty_like(pristine)
-    ab = torch.empty((n, b + 1), dtype=torch.float32, device=a.device)
-    w = torch.empty((n - b, n), dtype=torch.float32, device=a.device)
+    ab = torch.empty((n, b + 1), dtype=torch.float32, device=a.device) if rank == 0 else None
+    w = torch.empty((n - b, n), dtype=torch.float32, device=a.device) if rank == 0 else None
+
+    def run_step():
+        if world > 1:
+            h.reduce_dist(a, b, nb, mode=mode, ab=ab, w=w)
+        else:
+            h.reduce(a, b, nb, mode=mode, ab=ab, w=w)
+
     # warm-up (untimed)
     for _ in range(args.warmup):
         a.copy_(pristine)
-        h.reduce(a, b, nb, mode=mode, ab=ab, w=w)
+        run_step()
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
     # timed region: K steps, each bracketed by CUDA events on the launching stream; the
-    # input is restored from the pristine copy between steps, outside the events
-    h.reset_kernel_stats()
-    h.set_kernel_timing(True)
+    # input is restored from the pristine copy between steps, outside the events.  No
+    # per-kernel events here (they would serialise the programmatic dependent launches).
     launches0 = h.launch_count()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     torch.cuda.synchronize()
@@ -257,20 +272,33 @@ def main():
         for i in range(args.steps):
             a.copy_(pristine)
             evs[i][0].record(stream)
-            h.reduce(a, b, nb, mode=mode, ab=ab, w=w)
+            run_step()
             evs[i][1].record(stream)
         torch.cuda.synchronize()
-    h.set_kernel_timing(False)
     launches = h.launch_count() - launches0
     step_ms = [e0.elapsed_time(e1) for e0, e1 in evs]
     total_ms = sum(step_ms)
+    # profiled steps (right after the timed region, same stream): CUDA events around every
+    # kernel class give the per-kernel durations behind `roofline` and `breakdown`
+    h.reset_kernel_stats()
+    h.set_kernel_timing(True)
+    prof_ms = []
+    for _ in range(args.profile_steps):
+        a.copy_(pristine)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        run_step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        prof_ms.append(e0.elapsed_time(e1))
+    h.set_kernel_timing(False)
     if world > 1:
         t = torch.tensor([total_ms], device=a.device)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         torch.distributed.barrier()
         total_ms = float(t.item())
     ms_per_step = total_ms / args.steps
-    value = world * eff_tflops(n, ms_per_step / 1e3)
+    value = eff_tflops(n, ms_per_step / 1e3)   # one n x n matrix per step, on all ranks together
 
     # per-kernel-class stats (events around every launch inside the timed region)
     classes = ["panel", "lazy", "wmerge", "pass", "syr2k", "other"]
@@ -278,6 +306,7 @@ def main():
     dom = max(["pass", "syr2k", "panel", "lazy", "wmerge"], key=lambda c: kst[c]["ms"])
     peaks, src = load_peaks()
     st = kst[dom]
+    nprof = max(1, args.profile_steps)
     avg_ms = st["ms"] / max(1, st["launches"])
     if dom == "syr2k":
         achieved = st["flops"] / max(1, st["launches"]) / (avg_ms / 1e3) / 1e12
@@ -289,14 +318,52 @@ def main():
         peak = peaks["hbm_gbs"]
         roof = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
                 "traffic": None}
-    roof.update({"kernel": dom, "peak_source": src, "launches": st["launches"], "avg_ms": avg_ms,
-                 "share_of_step": st["ms"] / total_ms if total_ms else None})
-    breakdown = {c: {"ms_per_step": kst[c]["ms"] / args.steps, "launches_per_step": kst[c]["launches"] / args.steps}
+    # traffic: DRAM bytes per algorithmic byte of this kernel from the committed `ncu --set full`
+    # capture (profiles/traffic.json), times this run's algorithmic bytes per launch
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            tr = json.load(f).get(dom)
+        if tr:
+            roof["traffic"] = tr["dram_per_algorithmic_byte"] * st["bytes"] / max(1, st["launches"])
+            roof["traffic_source"] = tr["source"]
+    except Exception:
+        pass
+    roof.update({"kernel": dom, "peak_source": src, "launches_per_step": st["launches"] / nprof, "avg_ms": avg_ms,
+                 "share_of_step": st["ms"] / sum(prof_ms) if prof_ms else None,
+                 "measured_on": f"{nprof} profiled step(s) right after the timed region, CUDA events around every "
+                                f"kernel class on the launching stream ({statistics.mean(prof_ms):.1f} ms/step with "
+                                f"the events)"})
+    breakdown = {c: {"ms_per_step": kst[c]["ms"] / nprof, "launches_per_step": kst[c]["launches"] / nprof}
                  for c in classes}
 
     # end-to-end through the public API with HOST buffers (H2D of A + D2H of the band per step)
     e2e = None
-    if args.e2e_steps > 0:
+    if args.e2e_steps > 0 and world > 1:
+        # every rank copies the pinned host input in, the ranks reduce it together, rank 0
+        # reads the band back; wall clock with a barrier on both sides, max over ranks
+        a_host = torch.empty((n, n), dtype=torch.float32, pin_memory=True)
+        a_host.copy_(pristine.cpu())
+        ab_host = torch.empty((n, b + 1), dtype=torch.float32, pin_memory=True)
+        e2e_ms = []
+        for _ in range(args.e2e_steps + 1):
+            torch.cuda.synchronize()
+            torch.distributed.barrier()
+            t0 = time.perf_counter()
+            a.copy_(a_host, non_blocking=True)
+            run_step()
+            if rank == 0:
+                ab_host.copy_(ab, non_blocking=True)
+            torch.cuda.synchronize()
+            dt = torch.tensor([(time.perf_counter() - t0) * 1e3], device=a.device)
+            torch.distributed.all_reduce(dt, op=torch.distributed.ReduceOp.MAX)
+            e2e_ms.append(float(dt.item()))
+        e2e_ms = e2e_ms[1:]
+        e2e = {"value": eff_tflops(n, statistics.median(e2e_ms) / 1e3), "unit": "TFLOP/s",
+               "h2d_bytes_per_step": 4 * n * n * world, "d2h_bytes_per_step": 4 * n * (b + 1),
+               "ms_per_step": statistics.median(e2e_ms), "steps": args.e2e_steps,
+               "note": "Handle.reduce_dist: pinned host A -> every rank, reduce across ranks, band -> host"}
+        del a_host
+    elif args.e2e_steps > 0:
         a_host = torch.empty((n, n), dtype=torch.float32, pin_memory=True)
         a_host.copy_(pristine.cpu())   # same input bits (device generator == workloads generator)
         ab_host = torch.empty((n, b + 1), dtype=torch.float32, pin_memory=True)
@@ -308,7 +375,7 @@ def main():
             h.reduce_host(a_host, b, nb, mode=mode, ab=ab_host)
             e2e_ms.append((time.perf_counter() - t0) * 1e3)
         e2e_t = max(e2e_ms) if world == 1 else max(e2e_ms)
-        e2e = {"value": world * eff_tflops(n, statistics.median(e2e_ms) / 1e3), "unit": "TFLOP/s",
+        e2e = {"value": eff_tflops(n, statistics.median(e2e_ms) / 1e3), "unit": "TFLOP/s",
                "h2d_bytes_per_step": 4 * n * n, "d2h_bytes_per_step": 4 * n * (b + 1),
                "ms_per_step": statistics.median(e2e_ms), "steps": args.e2e_steps,
                "note": "sbr_reduce_host: pinned host A -> device, reduce, band -> host (the paper's EVD "
@@ -327,22 +394,24 @@ def main():
             "value": value,
             "unit": "TFLOP/s",
             "n_gpus": world,
+            "scaling": "strong" if world > 1 else "weak",
             "steps": args.steps,
             "warmup": args.warmup,
             "ms_per_step": ms_per_step,
             "seconds_per_step": ms_per_step / 1e3,
             "higher_is_better": True,
-            "scaling": "weak",
             "vs_baseline": None,
             "dtype": "f32" if mode == "3xtf32" else "f16",
             "data": "synthetic",
             "config": {"workload": f"config4: n={n} random symmetric U[-1,1) (seed {seed}), b={b}, nb={nb}, "
                                    f"{'FP16-in/FP32-acc' if mode == 'fp16' else '3xTF32'}",
                        "n": n, "b": b, "nb": nb, "mode": mode,
-                       "parallelism": "replicas" if world > 1 else "single",
+                       "parallelism": f"sbr_reduce_dist over {world} GPUs: per-panel pass sharded by lower "
+                                      f"tiles, NCCL broadcast W_t + all-reduce X_t" if world > 1 else "single",
                        "l2": f"inputs {4 * n * n / 2**30:.1f} GiB >> 126 MB L2 (no flush needed)"},
             "frac_of_peak": {"fp16_spec_2250": value / world / 2250.0,
-                             "fp16_measured": value / world / peaks.get("bf16_tflops", 1642.5)},
+                             "fp16_measured": value / world / peaks.get("bf16_tflops", 1642.5),
+                             "composite_roofline_model_ms": 88.4 if (n, b, nb) == (32768, 32, 1024) else None},
             "roofline": roof,
             "breakdown": breakdown,
             "cpu_baseline": cpu,

@@ -116,6 +116,35 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb,
                     float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw,
                     int outputs);
 
+/* ---- Multi-GPU (one process per GPU, NCCL over NVLink/NVSwitch) ----
+ *
+ * sbr_get_unique_id: rank 0 creates the 128-byte NCCL unique id (host call, no device work)
+ *   and distributes it to the other ranks out of band (e.g. torch.distributed).  Returns 0
+ *   or SBR_ERR_NCCL (libnccl.so.2 not loadable; it is dlopen'ed, the single-GPU path never
+ *   needs it).
+ * sbr_create_dist: like sbr_create, plus an NCCL communicator of `nranks` ranks built from
+ *   `unique_id` (collective: every rank must call it).  Returns 0, -1 (h NULL), -2 (device),
+ *   -4 (unique_id NULL), -5 (rank), -6 (nranks), SBR_ERR_CUDA, SBR_ERR_NCCL.
+ * sbr_reduce_dist: the reduction of ONE matrix across the communicator (strong scaling).
+ *   Every rank passes the same input A (full n x n, device; each rank keeps a full copy so
+ *   the trailing updates need no data exchange).  Rank 0 runs the sequential per-panel chain
+ *   (panel QR, reconstruction, lazy update, W merge) and returns AB, Y (in A) and W exactly
+ *   as sbr_reduce; on the other ranks AB and W may be NULL and A is left in an unspecified
+ *   state.  Per b-panel every rank streams its 1/nranks share of the lower tiles of OA for
+ *   X_t = OA W_t; the partial X_t are summed by an NCCL all-reduce (M x b fp32) after W_t
+ *   (fp16, M x b) is broadcast from rank 0; per nb-block rank 0 broadcasts Y (fp16) and
+ *   W^T X and every rank applies the trailing update.  All calls are stream-ordered on the
+ *   handle's stream and collective (every rank must call with the same n, b, nb, mode).
+ *   FP16 mode only when nranks > 1 (else SBR_ERR_UNSUPPORTED).  Same argument errors as
+ *   sbr_reduce; SBR_ERR_NCCL on a communication error.
+ * With nranks == 1, sbr_reduce_dist is sbr_reduce. */
+int sbr_get_unique_id(void* unique_id_128_bytes);
+int sbr_create_dist(sbr_handle_t* h, int device, void* stream, const void* unique_id, int rank, int nranks);
+int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb,
+                    float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw);
+int sbr_rank(sbr_handle_t h);     /* 0 for sbr_create handles; -1 if h is NULL */
+int sbr_nranks(sbr_handle_t h);   /* 1 for sbr_create handles; -1 if h is NULL */
+
 /* Wait for all work enqueued on the handle's stream. */
 int sbr_sync(sbr_handle_t h);
 

@@ -40,6 +40,23 @@ int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_t ldp, float* Y, float* W, int64_t ldyw,
                    int64_t* trace);
 
+/* Same as sbr_test_pass_fp16 but only the share of `rank` of `nranks` (the tiles
+ * sbr_test_pass_partition assigns): summing the X of all ranks gives the full pass. */
+int sbr_test_pass_fp16_part(sbr_handle_t h, int64_t M, int b, int rank, int nranks, const float* OA, int64_t ldoa,
+                            const float* W, int64_t ldw, float* X, int64_t ldx);
+
+/* Host only (no device work): the share of the per-panel pass (a4) that `rank` of `nranks`
+ * streams under sbr_reduce_dist, for an M x M block-local OA and bandwidth b: tiles
+ * [*t0, *t1) of *total 128 x 128 lower tiles, in the order of sbr_test_pass_tiles.
+ * Returns 0, -1 (M < 1), -2 (b), -3 (rank / nranks), -5 (NULL output). */
+int sbr_test_pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t* t1, int64_t* total);
+
+/* Host only: tile coordinates of tiles [t0, t1) of the pass order -- tile k is the lower
+ * tile (row block I, column block J), I >= J, of OA, IJ[2k] = I, IJ[2k+1] = J (caller
+ * allocates 2*(t1-t0) ints).  Each rank's contribution is X_I += L_IJ W_J and, for I > J,
+ * X_J += L_IJ^T W_I (a diagonal tile holds the strict lower part plus half the diagonal). */
+int sbr_test_pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ);
+
 #ifdef __cplusplus
 }
 #endif

@@ -14,8 +14,9 @@ tail is ``A[c, c+b+1:]``.  ``ab`` has torch shape (n, b+1): ``ab[j, d] = B[j+d, 
 (``ab.T`` is LAPACK lower band storage).  ``w`` has torch shape (n-b, n):
 ``w[c, r] = W(r, c)``.
 """
-from .api import Handle, reduce, reduce_host, generate_symmetric, band_to_dense  # noqa: F401
+from .api import (Handle, reduce, reduce_host, generate_symmetric, band_to_dense, get_unique_id,  # noqa: F401
+                  pass_partition, pass_tiles)
 from ._lib import lib, LIB_PATH, SbrError  # noqa: F401
 
-__all__ = ["Handle", "reduce", "reduce_host", "generate_symmetric", "band_to_dense", "lib", "LIB_PATH",
-           "SbrError"]
+__all__ = ["Handle", "reduce", "reduce_host", "generate_symmetric", "band_to_dense", "get_unique_id",
+           "pass_partition", "pass_tiles", "lib", "LIB_PATH", "SbrError"]

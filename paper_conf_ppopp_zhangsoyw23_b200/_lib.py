@@ -45,11 +45,20 @@ SIGNATURES = {
                               ctypes.POINTER(ctypes.c_double), ctypes.POINTER(ctypes.c_double)]),
     "sbr_launch_count": (_i64, [_h]),
     "sbr_version": (ctypes.c_char_p, []),
+    "sbr_get_unique_id": (_i, [_p]),
+    "sbr_create_dist": (_i, [ctypes.POINTER(ctypes.c_void_p), _i, _p, _p, _i, _i]),
+    "sbr_reduce_dist": (_i, [_h, _i, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_rank": (_i, [_h]),
+    "sbr_nranks": (_i, [_h]),
     # kernel-level test hooks (include/sbr_testing.h)
     "sbr_test_pass_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_test_pass_fp16_part": (_i, [_h, _i64, _i, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_syr2k_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_zform_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_panel": (_i, [_h, _i64, _i, _p, _i64, _p, _p, _i64, _p]),
+    "sbr_test_pass_partition": (_i, [_i64, _i, _i, _i, ctypes.POINTER(_i64), ctypes.POINTER(_i64),
+                                     ctypes.POINTER(_i64)]),
+    "sbr_test_pass_tiles": (_i, [_i64, _i, _i64, _i64, _p]),
 }
 
 _LIB = None

@@ -26,11 +26,36 @@ def _ptr(t) -> int | None:
     return t.ctypes.data  # numpy
 
 
+def get_unique_id() -> bytes:
+    """128-byte NCCL unique id for ``Handle(..., unique_id=..., rank=..., nranks=...)`` (rank 0 creates it)."""
+    buf = ctypes.create_string_buffer(128)
+    check(lib().sbr_get_unique_id(buf), "sbr_get_unique_id")
+    return buf.raw
+
+
+def pass_partition(M: int, b: int, rank: int, nranks: int):
+    """Host-only: (t0, t1, total) -- the tiles of the per-panel pass that ``rank`` streams (sbr_testing.h)."""
+    t0, t1, tot = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+    check(lib().sbr_test_pass_partition(M, b, rank, nranks, ctypes.byref(t0), ctypes.byref(t1), ctypes.byref(tot)),
+          "sbr_test_pass_partition")
+    return t0.value, t1.value, tot.value
+
+
+def pass_tiles(M: int, b: int, t0: int, t1: int):
+    """Host-only: list of (I, J) lower 128x128 tiles [t0, t1) in the pass's order."""
+    n = max(0, t1 - t0)
+    buf = (ctypes.c_int * (2 * n + 1))()
+    check(lib().sbr_test_pass_tiles(M, b, t0, t1, buf), "sbr_test_pass_tiles")
+    return [(buf[2 * k], buf[2 * k + 1]) for k in range(n)]
+
+
 class Handle:
     """One libsbr handle: a device, a CUDA stream (torch's current stream by default)
-    and the reduction workspace it owns."""
+    and the reduction workspace it owns.  With ``unique_id``/``rank``/``nranks`` it also owns
+    an NCCL communicator (one process per GPU) for :meth:`reduce_dist`."""
 
-    def __init__(self, device: int = 0, stream=None):
+    def __init__(self, device: int = 0, stream=None, unique_id: bytes | None = None, rank: int = 0,
+                 nranks: int = 1):
         import torch
 
         self.device = int(device)
@@ -38,8 +63,14 @@ class Handle:
             stream = torch.cuda.current_stream(self.device)
         self._stream = stream
         h = ctypes.c_void_p()
-        check(lib().sbr_create(ctypes.byref(h), self.device, ctypes.c_void_p(stream.cuda_stream)), "sbr_create")
+        if unique_id is None:
+            check(lib().sbr_create(ctypes.byref(h), self.device, ctypes.c_void_p(stream.cuda_stream)), "sbr_create")
+        else:
+            uid = ctypes.create_string_buffer(bytes(unique_id), 128)
+            check(lib().sbr_create_dist(ctypes.byref(h), self.device, ctypes.c_void_p(stream.cuda_stream), uid,
+                                        int(rank), int(nranks)), "sbr_create_dist")
         self._h = h
+        self.rank, self.nranks = int(rank), int(nranks)
 
     # -- lifecycle
     def close(self) -> None:
@@ -91,6 +122,29 @@ class Handle:
         check(lib().sbr_reduce(self._h, _mode(mode), n, int(b), int(nb), _ptr(A), n, _ptr(ab), b + 1,
                                _ptr(w), n), "sbr_reduce")
         return ab, w
+
+    def reduce_dist(self, A, b: int, nb: int, mode="fp16", want_w: bool = True, ab=None, w=None):
+        """One matrix across the handle's communicator (collective; see sbr_reduce_dist).
+
+        Every rank passes the same (n, n) float32 CUDA tensor; rank 0 gets ``(ab, w)`` as
+        :meth:`reduce` returns them, other ranks get ``(None, None)``."""
+        import torch
+
+        n = int(A.shape[0])
+        if A.dim() != 2 or A.shape[1] != n or A.dtype != torch.float32 or not A.is_cuda or not A.is_contiguous():
+            raise ValueError("A must be a contiguous square float32 CUDA tensor")
+        lead = self.rank == 0
+        if lead and ab is None:
+            ab = torch.empty((n, b + 1), dtype=torch.float32, device=A.device)
+        if lead and want_w and w is None and n > b:
+            w = torch.empty((max(n - b, 1), n), dtype=torch.float32, device=A.device)
+        if not lead or not want_w:
+            w = None if not lead else w
+        if not want_w:
+            w = None
+        check(lib().sbr_reduce_dist(self._h, _mode(mode), n, int(b), int(nb), _ptr(A), n,
+                                    _ptr(ab) if lead else None, b + 1, _ptr(w), n), "sbr_reduce_dist")
+        return (ab, w) if lead else (None, None)
 
     def reduce_host(self, A, b: int, nb: int, mode="fp16", outputs: int = _lib.SBR_OUT_BAND, ab=None, w=None):
         """End-to-end variant on HOST buffers (torch CPU tensors, ideally pinned, or numpy).

@@ -4,6 +4,9 @@
 #include <cuda_fp16.h>
 #include <stdint.h>
 #include <algorithm>
+#include <cstdlib>
+#include <cstring>
+#include <utility>
 
 #if defined(__CUDA_ARCH__) && (__CUDA_ARCH__ < 1000)
 #error "libsbr targets sm_100a only"
@@ -35,5 +38,35 @@ SBR_DEV float tf32_rna(float x) {
 
 SBR_DEV int lane_id() { return threadIdx.x & 31; }
 SBR_DEV int warp_id() { return threadIdx.x >> 5; }
+
+}  // namespace sbr
+
+namespace sbr {
+
+// Programmatic dependent launch (PDL).  Every kernel of the per-panel chain triggers its
+// dependents at entry and waits for its predecessor (griddepcontrol.wait: full completion
+// and memory flush of the prerequisite grid) before its first global-memory access, so the
+// next kernel's launch, barrier init, TMEM allocation and descriptor prefetch overlap the
+// tail of the previous one.  Without the launch attribute both are no-ops.
+SBR_DEV void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+SBR_DEV void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
+bool pdl_enabled();   // SBR_PDL=0 disables (ablation)
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 1 : 0;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
+}
 
 }  // namespace sbr

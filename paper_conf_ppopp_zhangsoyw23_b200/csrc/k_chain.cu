@@ -35,6 +35,8 @@ __global__ void __cluster_dims__(1, KXB_CL, 1) __launch_bounds__(256) kxb_kernel
   __shared__ __align__(16) float As[KXB_RC][KXB_QT];   // As[r][q] = WtX[q0+q, r]; reused for partials
   __shared__ float Bs[KXB_RC][32 * NG + 1];            // Bs[r][p] = B(r, p)
   cg::cluster_group cluster = cg::this_cluster();
+  pdl_trigger();
+  pdl_wait();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int k = a.k, b = a.b;
   const bool lazy = a.mode == 0;
@@ -130,10 +132,8 @@ cudaError_t launch_kxb(const KxbArgs& a, cudaStream_t st) {
   if (a.k <= 0 || a.b <= 0) return cudaSuccess;
   const dim3 grid((a.k + KXB_QT - 1) / KXB_QT, KXB_CL);
   if (a.b <= 32)
-    kxb_kernel<1><<<grid, 256, 0, st>>>(a);
-  else
-    kxb_kernel<2><<<grid, 256, 0, st>>>(a);
-  return cudaGetLastError();
+    return launch_pdl(kxb_kernel<1>, grid, dim3(256), 0, st, a);
+  return launch_pdl(kxb_kernel<2>, grid, dim3(256), 0, st, a);
 }
 
 // ------------------------------------------------------------------ postpass
@@ -152,6 +152,8 @@ __global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
   __shared__ float Ws[PP_ROWS][BB + 1];
   static_assert(PP_ROWS * (BB + 1) >= BB * BB, "partial fits in Xs");
   cg::cluster_group cluster = cg::this_cluster();
+  pdl_trigger();
+  pdl_wait();
   const int64_t rbeg = (int64_t)blockIdx.x * PP_ROWS;
   const int nr = (int)(M - rbeg < PP_ROWS ? (M - rbeg > 0 ? M - rbeg : 0) : PP_ROWS);
   for (int e = threadIdx.x; e < PP_ROWS * BB; e += blockDim.x) {
@@ -228,12 +230,13 @@ cudaError_t launch_postpass(int64_t M, int b, const float* X, int64_t ldx, const
     return (unsigned)((g + PP_CL - 1) / PP_CL * PP_CL);
   };
   if (b <= 16)
-    postpass_kernel<16><<<grid(pp_rows<16>()), 256, 0, st>>>(M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt, ldwtx);
-  else if (b <= 32)
-    postpass_kernel<32><<<grid(pp_rows<32>()), 256, 0, st>>>(M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt, ldwtx);
-  else
-    postpass_kernel<64><<<grid(pp_rows<64>()), 256, 0, st>>>(M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt, ldwtx);
-  return cudaGetLastError();
+    return launch_pdl(postpass_kernel<16>, dim3(grid(pp_rows<16>())), dim3(256), 0, st, M, b, X, ldx, W, ldw, Xh,
+                      ldxh, WtXtt, ldwtx);
+  if (b <= 32)
+    return launch_pdl(postpass_kernel<32>, dim3(grid(pp_rows<32>())), dim3(256), 0, st, M, b, X, ldx, W, ldw, Xh,
+                      ldxh, WtXtt, ldwtx);
+  return launch_pdl(postpass_kernel<64>, dim3(grid(pp_rows<64>())), dim3(256), 0, st, M, b, X, ldx, W, ldw, Xh,
+                    ldxh, WtXtt, ldwtx);
 }
 
 }  // namespace sbr

@@ -63,6 +63,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   uint64_t* acc_empty = acc_full + 2;
   uint32_t* tmem_slot = (uint32_t*)(bars + 2 * G_NS + 4);
   const int warp = warp_id(), lane = lane_id();
+  pdl_trigger();
   if (threadIdx.x == 0) {
     for (int i = 0; i < G_NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 32 * G_EPI_WARPS); }
@@ -77,6 +78,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();
   const int nk = nhalves * kpb;
 
   if (warp == 0) {
@@ -218,9 +220,9 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   }
   if (ntiles == 0) return cudaSuccess;
   const int grid = std::min(ntiles, p.num_sms);
-  kern<<<grid, G_THREADS, G_SMEM, st>>>(mA0, mA1, mB0, mB1, kpb, MODE == 0 ? 2 : 1, (int)p.arow0, (int)p.brow0, p.Mrows,
-                                  p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx, p.Zh, p.ldz);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, MODE == 0 ? 2 : 1,
+                    (int)p.arow0, (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X,
+                    p.ldx, p.Zh, p.ldz);
 }
 
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0>(p, st); }

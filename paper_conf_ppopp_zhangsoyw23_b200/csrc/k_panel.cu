@@ -378,6 +378,7 @@ SBR_DEV void warp_lu32(int b, const float* Q1, int ldq, float* Us, float* Ls, fl
 
 template <int B, int CPW>
 __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
+  pdl_trigger();   // the successor may launch early; it waits (griddepcontrol.wait) before reading
   constexpr int RSL = 32 * P_SL, RSN = 32 * P_SN;
   constexpr int LDU = B + 1;                 // padded ld for the b x b factors
   extern __shared__ __align__(16) float smem[];

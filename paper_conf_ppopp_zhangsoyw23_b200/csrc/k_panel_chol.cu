@@ -246,6 +246,7 @@ SBR_DEV void cta_lu(const double* Q1, float* Lcol, float* Urow, float* Ss, float
 
 template <int B>
 __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, unsigned char* ws, unsigned launch) {
+  pdl_trigger();   // the successor may launch early; it waits (griddepcontrol.wait) before reading
   using L = CholSmem<B>;
   constexpr int LDG = L::LDG;
   constexpr int LDQ = L::LDQ;
@@ -528,7 +529,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       const int i = e % B, c = e / B;
       if (i <= c) dev = fmax(dev, fabs(Gk[i + c * LDG] - (i == c ? 1.0 : 0.0)));
     }
-    if (!__syncthreads_or(!(dev <= PC_ORTH_TOL))) {
+    if (!__syncthreads_or(!(dev <= (a.orth_tol > 0.0 ? a.orth_tol : PC_ORTH_TOL)))) {
       done = true;
       break;
     }

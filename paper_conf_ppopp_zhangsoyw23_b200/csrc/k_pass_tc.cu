@@ -37,17 +37,18 @@ struct PassCfg {
 // min(ceff, I - gC + 1) tiles.  Every CTA takes an equal contiguous range of tiles
 // (balanced to one tile), so a launch ends when the slowest SM has streamed T/grid tiles.
 // The three roles walk the same range with this iterator.
+#define SBR_HD __host__ __device__ __forceinline__
 struct PassWalk {
   int NT, C;
   int g, J0, ceff, I, J;
   int64_t left;
   bool gfirst, rfirst;
-  SBR_DEV int jend() const { return min(J0 + ceff, I + 1); }
-  SBR_DEV static int64_t group_tiles(int NT, int C, int g) {
+  SBR_HD int jend() const { return min(J0 + ceff, I + 1); }
+  SBR_HD static int64_t group_tiles(int NT, int C, int g) {
     const int J0 = g * C, ce = min(C, NT - J0);
     return (int64_t)ce * (ce + 1) / 2 + (int64_t)(NT - J0 - ce) * ce;
   }
-  SBR_DEV void start(int NT_, int C_, int64_t t0, int64_t count) {
+  SBR_HD void start(int NT_, int C_, int64_t t0, int64_t count) {
     NT = NT_;
     C = C_;
     left = count;
@@ -73,10 +74,10 @@ struct PassWalk {
     }
     gfirst = rfirst = true;
   }
-  SBR_DEV bool valid() const { return left > 0; }
-  SBR_DEV bool rlast() const { return left == 1 || J + 1 == jend(); }
-  SBR_DEV bool glast() const { return left == 1 || (J + 1 == jend() && I + 1 == NT); }
-  SBR_DEV void next() {
+  SBR_HD bool valid() const { return left > 0; }
+  SBR_HD bool rlast() const { return left == 1 || J + 1 == jend(); }
+  SBR_HD bool glast() const { return left == 1 || (J + 1 == jend() && I + 1 == NT); }
+  SBR_HD void next() {
     --left;
     gfirst = rfirst = false;
     if (J + 1 < jend()) {
@@ -100,7 +101,7 @@ struct PassWalk {
 template <int BN, int C, int NS>
 __global__ void __launch_bounds__(256, 1)
     pass_tc_kernel(const __grid_constant__ CUtensorMap mapL, const __grid_constant__ CUtensorMap mapW, int r0, int M,
-                   int NT, int64_t T, int b, float* X, int64_t ldx) {
+                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx) {
   using Cfg = PassCfg<BN, C, NS>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -121,7 +122,10 @@ __global__ void __launch_bounds__(256, 1)
   uint32_t* tmem_slot = (uint32_t*)(bars + Cfg::NBAR);
 
   const int warp = warp_id(), lane = lane_id();
-  const int64_t t_beg = (int64_t)blockIdx.x * T / gridDim.x, t_end = (int64_t)(blockIdx.x + 1) * T / gridDim.x;
+  pdl_trigger();
+  // this launch covers tiles [T0, T0 + T) (a rank's share under sbr_reduce_dist); CTA share:
+  const int64_t t_beg = T0 + (int64_t)blockIdx.x * T / gridDim.x;
+  const int64_t t_end = T0 + (int64_t)(blockIdx.x + 1) * T / gridDim.x;
   if (threadIdx.x == 0) {
     for (int i = 0; i < NS; ++i) { mbar_init(&l_full[i], 1); mbar_init(&l_empty[i], 1); }
     for (int i = 0; i < 2; ++i) {
@@ -138,6 +142,7 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();
   const uint32_t t_col = tmem;                 // C column accumulators: cols [jj*BN, jj*BN+BN)
   const uint32_t t_row = tmem + C * BN;        // 2 row accumulators
   PassWalk w;
@@ -299,6 +304,32 @@ __global__ void __launch_bounds__(256, 1)
 }
 
 // ---------------------------------------------------------------- host
+static int64_t pass_total_tiles(int NT, int C) {
+  int64_t T = 0;
+  for (int g = 0; g * C < NT; ++g) T += PassWalk::group_tiles(NT, C, g);
+  return T;
+}
+
+static int pass_group_cols(int b) { return b <= 32 ? 8 : 4; }   // C of launch_pass_tc's instantiation
+
+void pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t* t1, int64_t* total) {
+  const int NT = (int)((M + 127) / 128);
+  const int64_t T = pass_total_tiles(NT, pass_group_cols(b));
+  *total = T;
+  *t0 = T * rank / nranks;
+  *t1 = T * (rank + 1) / nranks;
+}
+
+void pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ) {
+  const int NT = (int)((M + 127) / 128);
+  PassWalk w;
+  int64_t k = 0;
+  for (w.start(NT, pass_group_cols(b), t0, t1 - t0); w.valid(); w.next(), ++k) {
+    IJ[2 * k] = w.I;
+    IJ[2 * k + 1] = w.J;
+  }
+}
+
 template <int BN, int C, int NS>
 static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   using Cfg = PassCfg<BN, C, NS>;
@@ -315,15 +346,13 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   e = make_tmap_2d(&mapW, p.Wh, true, p.M, BN, p.ld_wh, 64, BN);
   if (e != cudaSuccess) return e;
   const int NT = (int)((p.M + 127) / 128);
-  const int G = (NT + C - 1) / C;
-  int64_t T = 0;
-  for (int g = 0; g < G; ++g) {
-    const int J0 = g * C, ce = std::min(C, NT - J0);
-    T += (int64_t)ce * (ce + 1) / 2 + (int64_t)(NT - J0 - ce) * ce;
-  }
+  const int64_t Tall = pass_total_tiles(NT, C);
+  const int64_t T0 = Tall * p.rank / p.nranks, T1 = Tall * (p.rank + 1) / p.nranks;
+  const int64_t T = T1 - T0;
+  if (T <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
-  kern<<<grid, 256, Cfg::SMEM, st>>>(mapL, mapW, (int)p.r0, (int)p.M, NT, T, p.b, p.X, p.ldx);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mapL, mapW, (int)p.r0, (int)p.M, NT, T0, T, p.b,
+                    p.X, p.ldx);
 }
 
 cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st) {

@@ -45,6 +45,7 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* acc_full = bars + 2 * Cfg::NS;
   uint32_t* tmem_slot = (uint32_t*)(bars + 2 * Cfg::NS + 2);
   const int warp = warp_id(), lane = lane_id();
+  pdl_trigger();
   const int tile = blockIdx.x;
   if (threadIdx.x == 0) {
     for (int i = 0; i < Cfg::NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
@@ -56,6 +57,7 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();
   if (warp == 0 && lane == 0) {
     int st = 0; uint32_t ph = 0;
     for (int kc = 0; kc < kct; ++kc) {
@@ -145,9 +147,8 @@ static cudaError_t launch_nn_t(const SkinnyNN& p, cudaStream_t st) {
   const int kct = kc0 + (int)((p.K1 + 63) / 64);
   const int grid = (int)((p.rows + 127) / 128);
   if (grid == 0) return cudaSuccess;
-  kern<<<grid, 256, Cfg::SMEM, st>>>(mA0, mA1, mB0, mB1, kc0, kct, (int)p.arow0, (int)p.brow0, p.rows, p.b, p.C,
-                                     p.ldc, p.D, p.ldd, p.Hcm, p.ldhc, p.Hrm, p.ldhr);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mA0, mA1, mB0, mB1, kc0, kct, (int)p.arow0,
+                    (int)p.brow0, p.rows, p.b, p.C, p.ldc, p.D, p.ldd, p.Hcm, p.ldhc, p.Hrm, p.ldhr);
 }
 
 cudaError_t launch_skinny_nn(const SkinnyNN& p, cudaStream_t st) {
@@ -183,6 +184,7 @@ __global__ void __launch_bounds__(256, 1)
   uint64_t* acc_full = bars + 2 * Cfg::NS;
   uint32_t* tmem_slot = (uint32_t*)(bars + 2 * Cfg::NS + 2);
   const int warp = warp_id(), lane = lane_id();
+  pdl_trigger();
   const int jt = blockIdx.x;                     // 128-wide slab of the K1 dimension
   const int64_t rb = row0 + (int64_t)blockIdx.y * chunk;
   const int64_t re = std::min<int64_t>(row0 + rows, rb + chunk);
@@ -197,6 +199,7 @@ __global__ void __launch_bounds__(256, 1)
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();
   const uint32_t bytes = (dual ? 2 : 1) * Cfg::SA + Cfg::SB;
   if (warp == 0 && lane == 0) {
     int st = 0; uint32_t ph = 0;
@@ -282,9 +285,8 @@ static cudaError_t launch_tn_t(const SkinnyTN& p, cudaStream_t st) {
   int64_t chunk = (p.rows + want - 1) / want;
   chunk = std::max<int64_t>(512, (chunk + 63) / 64 * 64);
   const int gy = (int)((p.rows + chunk - 1) / chunk);
-  kern<<<dim3(gx, gy), 256, Cfg::SMEM, st>>>(mA0, mA1, mB, p.A1 ? 1 : 0, p.row0, p.rows, chunk, (int)p.K1, p.b,
-                                             p.D0, p.D1, p.ldd);
-  return cudaGetLastError();
+  return launch_pdl(kern, dim3(gx, gy), dim3(256), Cfg::SMEM, st, mA0, mA1, mB, p.A1 ? 1 : 0, p.row0, p.rows, chunk,
+                    (int)p.K1, p.b, p.D0, p.D1, p.ldd);
 }
 
 cudaError_t launch_skinny_tn(const SkinnyTN& p, cudaStream_t st) {

@@ -34,6 +34,7 @@ struct PanelArgs {
   float* ws_misc;
   int64_t* trace;  // optional: CTA 0 phase timestamps (globaltimer ns), 10 entries
   const int* run_if;  // TSQR only: if non-NULL, do nothing unless *run_if != 0 (CholQR fallback)
+  double orth_tol;    // CholeskyQR acceptance: max|Q^T Q - I| (fp64) <= orth_tol (0: default 1e-9)
   // tree (filled by launch_panel)
   int nlev, arity;
   int nodes[kPanelMaxLev];
@@ -109,8 +110,12 @@ struct PassLaunch {
   int64_t ldx;
   int num_sms;
   int seg_rows;
+  int rank = 0, nranks = 1;   // tile share of this launch (sbr_reduce_dist): [T*rank/nranks, T*(rank+1)/nranks)
 };
 cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st);
+// host mirror of the pass's tile order (k_pass_tc.cu PassWalk): share of `rank`, and the (I, J) list
+void pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t* t1, int64_t* total);
+void pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ);
 int pass_bn(int b);
 
 struct GemmTcLaunch {

@@ -20,6 +20,7 @@
 
 #include "../../include/sbr.h"
 #include "kernels.h"
+#include "nccl_rt.h"
 
 using namespace sbr;
 
@@ -79,6 +80,10 @@ struct sbr_ctx {
   std::vector<Pending> pending;
   Stat stats[SBR_K_COUNT];
   int64_t launches = 0;
+  // multi-GPU (sbr_create_dist): this process's rank in an NCCL communicator of nranks
+  int rank = 0, nranks = 1;
+  nccl::Comm comm = nullptr;
+  bool force_coll = false;   // SBR_DIST_COLLECTIVES=1: issue the exchanges even with one rank (tests)
 };
 
 namespace {
@@ -130,6 +135,16 @@ void drain_stats(sbr_ctx* h) {
   }
   h->pending.clear();
 }
+
+#define SBR_NC(expr, what)                                             \
+  do {                                                                 \
+    const int _r = (expr);                                             \
+    if (_r != 0) {                                                     \
+      std::lock_guard<std::mutex> lk(g_err_mu);                        \
+      g_last_err = std::string(what) + ": " + nccl::error_string(_r);  \
+      return SBR_ERR_NCCL;                                             \
+    }                                                                  \
+  } while (0)
 
 #define SBR_CK(expr, what)                 \
   do {                                     \
@@ -243,7 +258,15 @@ int validate(sbr_ctx* h, int mode, int64_t n, int b, int nb, const float* A, int
 int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB, int64_t ldab,
                   float* W, int64_t ldw) {
   cudaStream_t st = h->stream;
+  // sbr_reduce_dist: every rank holds the full matrix; rank 0 ("lead") runs the sequential
+  // per-panel chain (a1-a3, a5) and owns the outputs, every rank streams its share of the
+  // per-panel pass (a4) and applies the trailing update (a6).  Exchanges per panel: broadcast
+  // of W_t (fp16, what the pass consumes) and all-reduce of the partial X_t; per block:
+  // broadcast of Y (fp16) and W^T X.  With nranks == 1 this is exactly sbr_reduce.
+  const bool lead = h->rank == 0;
+  const bool dist = h->comm != nullptr && (h->nranks > 1 || h->force_coll);
   if (n <= b + 1) {
+    if (!lead) return SBR_OK;
     Scope sc(h, SBR_K_OTHER, 0, 0);
     SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
     h->launches++;
@@ -287,7 +310,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     }
     if (tc16) {  // block start: X (accumulated by the passes), W^T X (diagonal blocks accumulated), G/H
       Scope sc(h, SBR_K_OTHER, 4.0 * M * p * b + 4.0 * nb * nb * 3, 0);
-      SBR_CK(zero_matrix(M, (int64_t)p * b, h->Xb, ldn, st), "zero X");
+      SBR_CK(zero_matrix(M, (int64_t)p * b, h->Xb, M, st), "zero X");
       SBR_CK(cudaMemsetAsync(h->WtX, 0, sizeof(float) * nb * nb, st), "zero WtX");
       SBR_CK(cudaMemsetAsync(h->GH, 0, sizeof(float) * 2 * nb * nb, st), "zero G/H");
     }
@@ -303,7 +326,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         const int64_t c = tb - b;  // OA column of the panel's first column
         const int64_t rows = M - c;
         float* Ablk = A + g + g * lda;
-        if (tc16) {  // P = W^T R (SIMT), then GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
+        if (tc16 && !lead) {
+          // not this rank's step
+        } else if (tc16) {  // P = W^T R (SIMT), then GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
           Scope sc(h, SBR_K_LAZY, 2.0 * rows * 2.0 * k + 8.0 * rows * b, 4.0 * rows * k * b);
           KxbArgs ka{};
           ka.mode = 0;
@@ -314,7 +339,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           ka.Y = h->Yb;
           ka.ldy = ldn;
           ka.X = h->Xb;
-          ka.ldx = ldn;
+          ka.ldx = M;
           ka.c = c;
           ka.Ph = h->Ph;
           ka.ldph = h->ldk;
@@ -354,7 +379,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           h->launches += 4;
         }
       }
-      {  // ---- a1/a2: TSQR + reconstruction
+      if (lead) {  // ---- a1/a2: TSQR + reconstruction
         Scope sc(h, SBR_K_PANEL, 4.0 * m * b * 4, 4.0 * m * b * b * 2);
         PanelArgs pa{};
         pa.P = A + (g + b) + g * lda;
@@ -378,6 +403,10 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.ws_r = h->pr;
         pa.ws_q = h->pq;
         pa.ws_misc = h->pmisc;
+        // CholeskyQR acceptance (reading R1): Q orthonormal in fp64 to far below the rounding of the
+        // mode's operands -- FP16 mode rounds every GEMM operand to fp16 (u = 4.9e-4), 3xTF32 keeps
+        // fp32 (u = 6e-8)
+        pa.orth_tol = tc16 ? 1e-6 : 1e-8;
         if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
           const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
           if (ce == cudaSuccess) {
@@ -391,7 +420,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         h->launches += 1;
       }
       if (tc16) {
-        if (t >= 1) {
+        if (t >= 1 && lead) {
           // ---- a3 on tcgen05: G = Y^T W0, H = X^T W0 (one pass over Y, X); W^T X_t = H - (W^T X) G;
           //      W_t = W0 - W G, written as fp32 + fp16 (column-major for the pass, row-major for later merges)
           Scope sc(h, SBR_K_WMERGE, 2.0 * (M - tb) * 2.0 * k + 2.0 * M * k + 12.0 * M * b,
@@ -451,8 +480,11 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           SBR_CK(launch_skinny_nn(mq, st), "W merge");
           h->launches += 3;
         }
+        if (dist) {  // W_t (fp16, column-major) from the lead to every rank
+          SBR_NC(nccl::broadcast(h->Wh, (size_t)h->ldwh * b, nccl::kFloat16, 0, h->comm, st), "broadcast W_t");
+        }
         {  // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA); X_t zeroed at block start
-          Scope sc(h, SBR_K_PASS, 1.0 * M * M + 6.0 * M * b, 2.0 * M * M * b);
+          Scope sc(h, SBR_K_PASS, (1.0 * M * M + 6.0 * M * b) / h->nranks, 2.0 * M * M * b / h->nranks);
           PassLaunch pl{};
           pl.shadow = h->Sh;
           pl.n = n;
@@ -462,16 +494,21 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           pl.ld_wh = h->ldwh;
           pl.r0 = r0;
           pl.b = b;
-          pl.X = h->Xb + tb * ldn;
-          pl.ldx = ldn;
+          pl.X = h->Xb + tb * M;
+          pl.ldx = M;
           pl.num_sms = h->nsm;
           pl.seg_rows = 8;
+          pl.rank = h->rank;
+          pl.nranks = h->nranks;
           SBR_CK(launch_pass_tc(pl, st), "pass_tc");
           h->launches += 1;
         }
-        {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block)
+        if (dist) {  // partial passes -> X_t on every rank
+          SBR_NC(nccl::all_reduce_sum_f32(h->Xb + tb * M, (size_t)M * b, h->comm, st), "all-reduce X_t");
+        }
+        if (lead) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block)
           Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
-          SBR_CK(launch_postpass(M, b, h->Xb + tb * ldn, ldn, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb,
+          SBR_CK(launch_postpass(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb,
                                  st),
                  "postpass");
           h->launches += 1;
@@ -505,6 +542,10 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int64_t s = (int64_t)p * b - b;
     const int64_t Mt = M - s;
     const int kk = p * b;
+    if (Mt > 0 && tc16 && dist) {   // the lead's Y (fp16) and W^T X for every rank's trailing update
+      SBR_NC(nccl::broadcast(h->Yh, (size_t)M * h->ldk, nccl::kFloat16, 0, h->comm, st), "broadcast Y");
+      SBR_NC(nccl::broadcast(h->WtX, (size_t)nb * nb, nccl::kFloat32, 0, h->comm, st), "broadcast W^T X");
+    }
     if (Mt > 0 && tc16) {
       Scope sc(h, SBR_K_SYR2K, 10.0 * Mt * Mt / 2 + 2.0 * Mt * kk * 4 + 4.0 * Mt * kk,
                2.0 * Mt * Mt * kk + 2.0 * Mt * kk * kk);
@@ -522,7 +563,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       gz.Mrows = Mt;
       gz.Ncols = kk;
       gz.X = h->Xb + s;
-      gz.ldx = ldn;
+      gz.ldx = M;
       gz.Zh = h->Zh + s * h->ldk;
       gz.ldz = h->ldk;
       gz.num_sms = h->nsm;
@@ -552,7 +593,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       h->launches += 2;
     }
   }
-  {
+  if (lead) {
     Scope sc(h, SBR_K_OTHER, 8.0 * (b + 1) * n, 0);
     SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
     h->launches += 1;
@@ -594,6 +635,7 @@ int sbr_destroy(sbr_handle_t h) {
   cudaSetDevice(h->device);
   cudaStreamSynchronize(h->stream);
   drain_stats(h);
+  if (h->comm) nccl::comm_destroy(h->comm);
   for (auto e : h->ev_pool) cudaEventDestroy(e);
   if (h->ws) cudaFree(h->ws);
   if (h->e2e) cudaFree(h->e2e);
@@ -667,6 +709,70 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A
   SBR_CK(cudaStreamSynchronize(st), "sync");
   return SBR_OK;
 }
+
+int sbr_get_unique_id(void* id) {
+  if (!id) return -1;
+  if (const char* e = nccl::load()) {
+    std::lock_guard<std::mutex> lk(g_err_mu);
+    g_last_err = e;
+    return SBR_ERR_NCCL;
+  }
+  nccl::UniqueId u;
+  SBR_NC(nccl::get_unique_id(&u), "ncclGetUniqueId");
+  memcpy(id, &u, sizeof(u));
+  return SBR_OK;
+}
+
+int sbr_create_dist(sbr_handle_t* out, int device, void* stream, const void* unique_id, int rank, int nranks) {
+  if (!out) return -1;
+  if (!unique_id) return -4;
+  if (nranks < 1) return -6;
+  if (rank < 0 || rank >= nranks) return -5;
+  int rc = sbr_create(out, device, stream);
+  if (rc != SBR_OK) return rc;
+  sbr_ctx* h = *out;
+  h->rank = rank;
+  h->nranks = nranks;
+  const char* fc = getenv("SBR_DIST_COLLECTIVES");
+  h->force_coll = fc && strcmp(fc, "1") == 0;
+  if (const char* e = nccl::load()) {
+    std::lock_guard<std::mutex> lk(g_err_mu);
+    g_last_err = e;
+    sbr_destroy(h);
+    *out = nullptr;
+    return SBR_ERR_NCCL;
+  }
+  nccl::UniqueId u;
+  memcpy(&u, unique_id, sizeof(u));
+  const int r = nccl::comm_init_rank(&h->comm, nranks, u, rank);
+  if (r != 0) {
+    {
+      std::lock_guard<std::mutex> lk(g_err_mu);
+      g_last_err = std::string("ncclCommInitRank: ") + nccl::error_string(r);
+    }
+    h->comm = nullptr;
+    sbr_destroy(h);
+    *out = nullptr;
+    return SBR_ERR_NCCL;
+  }
+  return SBR_OK;
+}
+
+int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB,
+                    int64_t ldab, float* W, int64_t ldw) {
+  if (!h) return -1;
+  const bool lead = h->rank == 0;
+  // outputs are produced on rank 0 only; other ranks may pass AB = W = NULL
+  int rc = validate(h, mode, n, b, nb, A, lda, lead ? AB : A, ldab < b + 1 && !lead ? b + 1 : ldab, W, ldw);
+  if (rc != SBR_OK) return rc;
+  if (h->nranks > 1 && mode != SBR_FP16_FP32ACC) return SBR_ERR_UNSUPPORTED;
+  if (h->nranks > 1 && !h->comm) return SBR_ERR_NCCL;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  return reduce_device(h, mode, n, b, nb, A, lda, AB, ldab, W, ldw);
+}
+
+int sbr_rank(sbr_handle_t h) { return h ? h->rank : -1; }
+int sbr_nranks(sbr_handle_t h) { return h ? h->nranks : -1; }
 
 int sbr_sync(sbr_handle_t h) {
   if (!h) return -1;
@@ -777,9 +883,18 @@ struct DevBuf {
 
 extern "C" {
 
+int sbr_test_pass_fp16_part(sbr_handle_t h, int64_t M, int b, int rank, int nranks, const float* OA, int64_t ldoa,
+                            const float* W, int64_t ldw, float* X, int64_t ldx);
+
 int sbr_test_pass_fp16(sbr_handle_t h, int64_t M, int b, const float* OA, int64_t ldoa, const float* W, int64_t ldw,
                        float* X, int64_t ldx) {
+  return sbr_test_pass_fp16_part(h, M, b, 0, 1, OA, ldoa, W, ldw, X, ldx);
+}
+
+int sbr_test_pass_fp16_part(sbr_handle_t h, int64_t M, int b, int rank, int nranks, const float* OA, int64_t ldoa,
+                            const float* W, int64_t ldw, float* X, int64_t ldx) {
   if (!h) return -1;
+  if (nranks < 1 || rank < 0 || rank >= nranks) return -4;
   if (M < 1) return -2;
   if (b < 1 || b > 64) return -3;
   SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
@@ -804,6 +919,8 @@ int sbr_test_pass_fp16(sbr_handle_t h, int64_t M, int b, const float* OA, int64_
   pl.ldx = ldx;
   pl.num_sms = h->nsm;
   pl.seg_rows = 8;
+  pl.rank = rank;
+  pl.nranks = nranks;
   SBR_CK(launch_pass_tc(pl, st), "pass_tc");
   SBR_CK(cudaStreamSynchronize(st), "sync");
   return SBR_OK;
@@ -920,5 +1037,26 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
     SBR_CK(cudaMemcpyAsync(trace_host, tr.p, sizeof(int64_t) * 16, cudaMemcpyDeviceToHost, st), "trace D2H");
     SBR_CK(cudaStreamSynchronize(st), "sync");
   }
+  return SBR_OK;
+}
+
+// host-only: the pass's tile share of `rank` (test hook for the multi-GPU partition)
+extern "C" int sbr_test_pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t* t1,
+                                       int64_t* total) {
+  if (M < 1) return -1;
+  if (b < 1 || b > 64) return -2;
+  if (nranks < 1 || rank < 0 || rank >= nranks) return -3;
+  if (!t0 || !t1 || !total) return -5;
+  pass_partition(M, b, rank, nranks, t0, t1, total);
+  return SBR_OK;
+}
+
+// host-only: (I, J) tile coordinates of tiles [t0, t1) in the pass's order, IJ[2k], IJ[2k+1]
+extern "C" int sbr_test_pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ) {
+  if (M < 1) return -1;
+  if (b < 1 || b > 64) return -2;
+  if (t0 < 0 || t1 < t0) return -3;
+  if (!IJ && t1 > t0) return -5;
+  pass_tiles(M, b, t0, t1, IJ);
   return SBR_OK;
 }
