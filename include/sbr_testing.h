@@ -57,6 +57,21 @@ int sbr_test_pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0,
  * X_J += L_IJ^T W_I (a diagonal tile holds the strict lower part plus half the diagonal). */
 int sbr_test_pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ);
 
+/* 3xTF32 mode (reading C11 / R4): X (M x b) = OA W on tcgen05 kind::tf32 from the fp32 OA
+ * (ldoa % 4 == 0; lower referenced; the upper triangle is ignored).  If S != NULL, the
+ * 128-column tiles covering OA columns [0, sw) are read from S (M x >= min(128 ceil(sw/128), M),
+ * ld lds) instead -- the frozen-strip path of sbr_reduce.  W is split rna hi/lo. */
+int sbr_test_pass_tf32(sbr_handle_t h, int64_t M, int b, const float* OA, int64_t ldoa, const float* S,
+                       int64_t lds, int64_t sw, const float* W, int64_t ldw, float* X, int64_t ldx);
+
+/* 3xTF32: C_low (M x M) -= Y Z^T + Z Y^T (hi/lo split Y, Z; 6 tf32 products per pair). */
+int sbr_test_syr2k_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* Z,
+                        int64_t ldz, float* C, int64_t ldc);
+
+/* 3xTF32: Z (M x K) = X - 1/2 Y G (G K x K symmetric); Z returned as hi + lo in fp32. */
+int sbr_test_zform_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
+                        const float* X, int64_t ldx, float* Z, int64_t ldz);
+
 #ifdef __cplusplus
 }
 #endif

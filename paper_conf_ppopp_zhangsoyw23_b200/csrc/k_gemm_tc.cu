@@ -11,6 +11,14 @@
 // SYR2K epilogue: C_new = C_old - acc on the fp32 master (lower elements only) and the
 // fp16 shadow of the next block's OA (strict lower, half diagonal; see k_pass_tc.cu).
 // ZFORM epilogue: Zh = fp16(X - acc/2), row-major.
+//
+// 3xTF32 mode (reading C11): operands are fp32 row-major arrays holding
+// [hi | lo] (hi = rna_tf32(a), lo = rna_tf32(a - hi), lo at column offset `lo_off`), and
+// the K loop runs over a SEGMENT TABLE: SYR2K = Yhi Zhi' + Yhi Zlo' + Ylo Zhi' + (Y <-> Z),
+// ZFORM = Yhi Ghi + Yhi Glo + Ylo Ghi, all accumulated in one fp32 TMEM accumulator by
+// tcgen05.mma kind::tf32 (BK = 32 fp32 = 128 B rows, the same smem bytes per stage).
+// The ZFORM epilogue then writes Z split the same way; the SYR2K epilogue writes no shadow
+// (the 3xTF32 pass reads the fp32 master).
 #include "kernels.h"
 #include "tc.cuh"
 
@@ -19,24 +27,34 @@ namespace sbr {
 using namespace tc;
 
 namespace {
-constexpr int G_BM = 128, G_BN = 256, G_BK = 64, G_NS = 4;
-constexpr int G_SA = G_BM * G_BK * 2;  // 16 KB
-constexpr int G_SB = G_BN * G_BK * 2;  // 32 KB
-constexpr int G_STAGE = G_SA + G_SB;
-constexpr int G_OFF_BAR = G_NS * G_STAGE;
-constexpr int G_SMEM = G_OFF_BAR + (2 * G_NS + 4) * 8 + 16 + 1024;
+constexpr int G_BM = 128;
+constexpr int G_ROWB = 128;            // bytes of one operand row chunk (64 fp16 or 32 fp32)
+constexpr int G_SA = G_BM * G_ROWB;    // 16 KB
+template <bool TF> struct GCfg {
+  // fp16: 128 x 256 tiles, one TMEM accumulation per tile.  3xTF32: 128 x 128 tiles and the
+  // accumulator is drained every FLUSH k-chunks (128 K elements) into fp32 registers (RN adds):
+  // the tensor core's own fp32 accumulation truncates, which over K = 6 nb terms would cost
+  // ~K^1.5 ulps (reading R4).
+  static constexpr int BN = TF ? 128 : 256;
+  static constexpr int NS = TF ? 6 : 4;
+  static constexpr int SB = BN * G_ROWB;
+  static constexpr int STAGE = G_SA + SB;
+  static constexpr int OFF_BAR = NS * STAGE;
+  static constexpr int SMEM = OFF_BAR + (2 * NS + 4) * 8 + 16 + 1024;
+  static constexpr int FLUSH = 4;
+};
 }  // namespace
 
-// tile index -> (I, Jc)
-template <int MODE>
+// tile index -> (I, Jc); SYR2K: the lower tiles, row I holding floor(I*BM/BN)+1 tiles of BN columns
+template <int MODE, int BN>
 SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
   if (MODE == 1) {  // ZFORM: full grid, row-major
     I = t / ntn;
     Jc = t % ntn;
-  } else {          // SYR2K: row I has floor(I/2)+1 tiles of 256 columns
+  } else {
     int i = 0;
     while (true) {
-      const int cnt = i / 2 + 1;
+      const int cnt = i * G_BM / BN + 1;
       if (t < cnt) { I = i; Jc = t; return; }
       t -= cnt;
       ++i;
@@ -47,16 +65,26 @@ SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
 constexpr int G_EPI_WARPS = 8;  // two warps per TMEM lane quarter, each half of the 256 columns
 constexpr int G_THREADS = 128 + 32 * G_EPI_WARPS;
 
-template <int MODE>
+// K segments: segment s multiplies columns [acol[s], acol[s] + K) of A map amap[s] with
+// columns [bcol[s], ...) of B map bmap[s]; all segments accumulate into the same tile.
+struct GemmSegs {
+  int n;
+  int amap[6], acol[6], bmap[6], bcol[6];
+};
+
+template <int MODE, bool TF>
 __global__ void __launch_bounds__(G_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap mapA0, const __grid_constant__ CUtensorMap mapA1,
                    const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
-                   int nhalves, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles, float* C,
-                   int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, const float* __restrict__ X, int64_t ldx,
-                   __half* __restrict__ Zh, int64_t ldz) {
+                   const GemmSegs segs, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles,
+                   float* C, int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, const float* __restrict__ X,
+                   int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off) {
+  using Cfg = GCfg<TF>;
+  constexpr int BK = TF ? 32 : 64;   // K elements per 128-byte row chunk
+  constexpr int G_BN = Cfg::BN, G_NS = Cfg::NS, G_STAGE = Cfg::STAGE;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint64_t* bars = (uint64_t*)(smem + G_OFF_BAR);
+  uint64_t* bars = (uint64_t*)(smem + Cfg::OFF_BAR);
   uint64_t* full = bars;
   uint64_t* empty = bars + G_NS;
   uint64_t* acc_full = bars + 2 * G_NS;
@@ -70,8 +98,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     mbar_fence_init();
   }
   if (warp == 0 && lane == 0) {
-    tma_prefetch(&mapA0); tma_prefetch(&mapB0);
-    if (nhalves > 1) { tma_prefetch(&mapA1); tma_prefetch(&mapB1); }
+    tma_prefetch(&mapA0); tma_prefetch(&mapB0); tma_prefetch(&mapA1); tma_prefetch(&mapB1);
   }
   if (warp == 2) tmem_alloc(tmem_slot, 512);
   tc_fence_before();
@@ -79,48 +106,112 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   pdl_wait();
-  const int nk = nhalves * kpb;
+  const int nk = segs.n * kpb;
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
       int st = 0; uint32_t ph = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
         int I, Jc;
-        gemm_tile<MODE>(t, ntn, I, Jc);
+        gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
         for (int kc = 0; kc < nk; ++kc) {
-          const int half = kc / kpb, kin = (kc % kpb) * G_BK;
+          const int sg = kc / kpb, kin = (kc % kpb) * BK;
           mbar_wait(&empty[st], ph ^ 1);
           mbar_expect_tx(&full[st], G_STAGE);
           uint8_t* sa = smem + st * G_STAGE;
-          tma_load_2d(sa, half ? &mapA1 : &mapA0, &full[st], kin, arow0 + I * G_BM);
-          tma_load_2d(sa + G_SA, half ? &mapB1 : &mapB0, &full[st], kin, brow0 + Jc * G_BN);
+          tma_load_2d(sa, segs.amap[sg] ? &mapA1 : &mapA0, &full[st], segs.acol[sg] + kin, arow0 + I * G_BM);
+          tma_load_2d(sa + G_SA, segs.bmap[sg] ? &mapB1 : &mapB0, &full[st], segs.bcol[sg] + kin,
+                      brow0 + Jc * G_BN);
           if (++st == G_NS) { st = 0; ph ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {  // ---------------- MMA issuer
-      constexpr uint32_t idesc = idesc_make(G_BM, G_BN, 0, 0, 0);
+      constexpr uint32_t idesc = idesc_make(G_BM, G_BN, TF ? 2 : 0, 0, 0);
       int st = 0; uint32_t ph = 0;
       int ab = 0; uint32_t aph = 0;
       const uint32_t s0 = smem_u32(smem);
+      // accumulation groups: fp16 one per tile; 3xTF32 every FLUSH k-chunks (drained by the epilogue)
+      const int ch = TF ? Cfg::FLUSH : nk;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
-        mbar_wait(&acc_empty[ab], aph ^ 1);
-        tc_fence_after();
-        const uint32_t d = tmem + ab * G_BN;
         for (int kc = 0; kc < nk; ++kc) {
+          if (kc % ch == 0) {
+            mbar_wait(&acc_empty[ab], aph ^ 1);
+            tc_fence_after();
+          }
+          const uint32_t d = tmem + ab * G_BN;
           mbar_wait(&full[st], ph);
           tc_fence_after();
           const uint32_t sa = s0 + st * G_STAGE, sb = sa + G_SA;
 #pragma unroll
-          for (int s = 0; s < G_BK / 16; ++s)
-            mma_f16(d, sdesc_sw128(sa + s * 32, 16, 1024), sdesc_sw128(sb + s * 32, 16, 1024), idesc,
-                    (kc > 0 || s > 0) ? 1u : 0u);
+          for (int s = 0; s < 4; ++s) {  // 4 MMAs of 32 bytes of K (16 fp16 / 8 tf32)
+            if (TF)
+              mma_tf32(d, sdesc_sw128(sa + s * 32, 16, 1024), sdesc_sw128(sb + s * 32, 16, 1024), idesc,
+                       (kc % ch > 0 || s > 0) ? 1u : 0u);
+            else
+              mma_f16(d, sdesc_sw128(sa + s * 32, 16, 1024), sdesc_sw128(sb + s * 32, 16, 1024), idesc,
+                      (kc % ch > 0 || s > 0) ? 1u : 0u);
+          }
           mma_commit(&empty[st]);
           if (++st == G_NS) { st = 0; ph ^= 1; }
+          if (kc % ch == ch - 1 || kc == nk - 1) {
+            mma_commit(&acc_full[ab]);
+            if (++ab == 2) { ab = 0; aph ^= 1; }
+          }
         }
-        mma_commit(&acc_full[ab]);
+      }
+    }
+  } else if (warp >= 4 && TF) {  // ---------------- 3xTF32 epilogue (8 warps: 32 lanes x 64 columns each)
+    const int e = warp - 4;
+    const int q = e & 3;
+    const int chalf = e >> 2;
+    const int rit = q * 32 + lane;
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    const int ngroups = (nk + Cfg::FLUSH - 1) / Cfg::FLUSH;
+    int ab = 0; uint32_t aph = 0;
+    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      int I, Jc;
+      gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+      float acc[64];
+#pragma unroll
+      for (int c = 0; c < 64; ++c) acc[c] = 0.f;
+      for (int gi = 0; gi < ngroups; ++gi) {   // fp32 round-to-nearest sum of the partial accumulations
+        mbar_wait(&acc_full[ab], aph);
+        tc_fence_after();
+        float v[32], u[32];
+        tmem_ld32(tmem + ab * G_BN + chalf * 64 + lane_off, v);
+        tmem_ld32(tmem + ab * G_BN + chalf * 64 + 32 + lane_off, u);
+        tc_fence_before();
+        mbar_arrive(&acc_empty[ab]);
         if (++ab == 2) { ab = 0; aph ^= 1; }
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+          acc[c] += v[c];
+          acc[32 + c] += u[c];
+        }
+      }
+      const int64_t row = (int64_t)I * G_BM + rit;
+      if (row >= Mrows) continue;
+      const int64_t col0 = (int64_t)Jc * G_BN + chalf * 64;
+      if (MODE == 0) {
+        float* cp = C + row + col0 * ldc;
+#pragma unroll
+        for (int c = 0; c < 64; ++c)
+          if (col0 + c <= row) __stcs(cp + c * ldc, __ldcs(cp + c * ldc) - acc[c]);
+      } else {   // Z split: hi = rna_tf32(z), lo = rna_tf32(z - hi), row-major
+        float* zp = (float*)Zout + row * ldz + col0;
+#pragma unroll
+        for (int c = 0; c < 64; ++c) {
+          if (col0 + c < Ncols) {
+            const float z = fmaf(-0.5f, acc[c], __ldcs(X + row + (col0 + c) * ldx));
+            const float hi = tf32_rna(z);
+            zp[c] = hi;
+            zp[c + zlo_off] = tf32_rna(z - hi);
+          } else if (col0 + c < zlo_off) {
+            zp[c] = 0.f;   // K padding of the hi half must read as zero in the SYR2K
+          }
+        }
       }
     }
   } else if (warp >= 4) {  // ---------------- epilogue (8 warps)
@@ -132,7 +223,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
-      gemm_tile<MODE>(t, ntn, I, Jc);
+      gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();
       const int64_t row = (int64_t)I * G_BM + rit;
@@ -163,6 +254,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
           float xv[32];
 #pragma unroll
           for (int c = 0; c < 32; ++c) xv[c] = (col0 + c < Ncols) ? __ldcs(X + row + (col0 + c) * ldx) : 0.f;
+          __half* Zh = (__half*)Zout;
           __align__(16) __half z[32];
 #pragma unroll
           for (int c = 0; c < 32; ++c) z[c] = __float2half_rn(fmaf(-0.5f, v[c], xv[c]));
@@ -188,9 +280,11 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   }
 }
 
-template <int MODE>
+template <int MODE, bool TF>
 static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
-  auto kern = gemm_tc_kernel<MODE>;
+  auto kern = gemm_tc_kernel<MODE, TF>;
+  constexpr int BK = TF ? 32 : 64;
+  constexpr int G_BN = GCfg<TF>::BN, G_SMEM = GCfg<TF>::SMEM;
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, G_SMEM);
@@ -199,33 +293,53 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   }
   CUtensorMap mA0, mA1, mB0, mB1;
   cudaError_t e;
-  if ((e = make_tmap_2d(&mA0, p.A0, true, p.K, p.a_rows, p.ld_a, G_BK, G_BM)) != cudaSuccess) return e;
-  if ((e = make_tmap_2d(&mB0, p.B0, true, p.K, p.b_rows, p.ld_b, G_BK, G_BN)) != cudaSuccess) return e;
+  // map width: the K columns (fp16) or the [hi | lo] columns (3xTF32: lo at lo_off)
+  const uint64_t wid = TF ? (uint64_t)(p.lo_off + p.K) : (uint64_t)p.K;
+  if ((e = make_tmap_2d(&mA0, p.A0, !TF, wid, p.a_rows, p.ld_a, BK, G_BM)) != cudaSuccess) return e;
+  if ((e = make_tmap_2d(&mB0, p.B0, !TF, wid, p.b_rows, p.ld_b, BK, G_BN)) != cudaSuccess) return e;
   if (MODE == 0) {
-    if ((e = make_tmap_2d(&mA1, p.A1, true, p.K, p.a_rows, p.ld_a, G_BK, G_BM)) != cudaSuccess) return e;
-    if ((e = make_tmap_2d(&mB1, p.B1, true, p.K, p.b_rows, p.ld_b, G_BK, G_BN)) != cudaSuccess) return e;
+    if ((e = make_tmap_2d(&mA1, p.A1, !TF, wid, p.a_rows, p.ld_a, BK, G_BM)) != cudaSuccess) return e;
+    if ((e = make_tmap_2d(&mB1, p.B1, !TF, wid, p.b_rows, p.ld_b, BK, G_BN)) != cudaSuccess) return e;
   } else {
     mA1 = mA0;
     mB1 = mB0;
   }
-  const int kpb = (int)((p.K + G_BK - 1) / G_BK);
+  const int kpb = (int)((p.K + BK - 1) / BK);
+  GemmSegs sg{};
+  const int lo = (int)p.lo_off;
+  if (!TF) {        // SYR2K: [Y | Z] [Z | Y]^T ; ZFORM: Y G
+    sg.n = MODE == 0 ? 2 : 1;
+    sg.amap[1] = 1; sg.bmap[1] = 1;
+  } else {          // hi hi' + hi lo' + lo hi' per product
+    const int half = MODE == 0 ? 2 : 1;
+    sg.n = 3 * half;
+    for (int h = 0; h < half; ++h)
+      for (int q = 0; q < 3; ++q) {
+        const int s = h * 3 + q;
+        sg.amap[s] = h; sg.bmap[s] = h;
+        sg.acol[s] = q == 2 ? lo : 0;
+        sg.bcol[s] = q == 1 ? lo : 0;
+      }
+  }
   const int ntm = (int)((p.Mrows + G_BM - 1) / G_BM);
   const int ntn = (int)((p.Ncols + G_BN - 1) / G_BN);
   int ntiles;
   if (MODE == 0) {
     ntiles = 0;
-    for (int i = 0; i < ntm; ++i) ntiles += i / 2 + 1;
+    for (int i = 0; i < ntm; ++i) ntiles += i * G_BM / G_BN + 1;
   } else {
     ntiles = ntm * ntn;
   }
   if (ntiles == 0) return cudaSuccess;
   const int grid = std::min(ntiles, p.num_sms);
-  return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, MODE == 0 ? 2 : 1,
-                    (int)p.arow0, (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X,
-                    p.ldx, p.Zh, p.ldz);
+  return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
+                    (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
+                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.lo_off);
 }
 
-cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0>(p, st); }
-cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1>(p, st); }
+cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, false>(p, st); }
+cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, false>(p, st); }
+cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, true>(p, st); }
+cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, true>(p, st); }
 
 }  // namespace sbr

@@ -118,6 +118,23 @@ void pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t
 void pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ);
 int pass_bn(int b);
 
+// 3xTF32 pass (k_pass_tf32.cu): X (M x b, b <= 32, column-major, zeroed by the caller) +=
+// OA WS with OA = A[r0:, r0:] (fp32 master, lower referenced, lda % 4 == 0) except tile
+// columns J < ceil(sw/128), read from the strip S (M x >= min(128 ceil(sw/128), M), ld lds).
+// WS: M x 64 column-major [W_hi (32 cols) | W_lo (32 cols)] from split_tf32_w (bn = 32).
+struct PassTf32Launch {
+  const float* A; int64_t n, lda, r0;
+  const float* S; int64_t lds; int64_t sw;
+  const float* WS; int64_t ldws;
+  int64_t M;
+  int b;
+  float* X; int64_t ldx;
+  int num_sms;
+  int rank = 0, nranks = 1;
+};
+cudaError_t launch_pass_tf32(const PassTf32Launch& p, cudaStream_t st);
+int64_t pass_tf32_tiles(int64_t M);
+
 struct GemmTcLaunch {
   // fp16 row-major operands (K contiguous): A rows = output rows, B rows = output cols
   const __half *A0, *A1, *B0, *B1;  // SYR2K: A=[Y|Z] (A0=Yh, A1=Zh), B=[Z|Y]; ZFORM: A0=Yh, B0=WtXh
@@ -130,9 +147,27 @@ struct GemmTcLaunch {
   const float* X; int64_t ldx;      // ZFORM: X (column-major fp32)
   __half* Zh; int64_t ldz;          // ZFORM: Z out (row-major fp16)
   int num_sms;
+  // 3xTF32 (launch_*_tf32): A0..B1 point at fp32 row-major [hi | lo] arrays (cast), lo at
+  // column lo_off >= round_up(K, 32); hi columns [K, lo_off) must be zero.  ZFORM writes Zs
+  // (fp32 row-major, ld ldz) in the same split layout.
+  int64_t lo_off = 0;
+  float* Zs = nullptr;
 };
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st);
+cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st);
+cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st);
+// fp32 column-major src (rows x cols) -> row-major split dst: dst[r*ldd + c] = rna_tf32(a),
+// dst[r*ldd + lo_off + c] = rna_tf32(a - hi), zeros in hi columns [cols, lo_off)
+cudaError_t split_tf32_rm(int64_t rows, int cols, const float* src, int64_t lds, float* dst, int64_t ldd,
+                          int64_t lo_off, cudaStream_t st);
+// fp32 column-major W (rows x b) -> column-major [W_hi | W_lo] (rows x 2*bn, hi cols [0,bn), lo [bn, 2bn);
+// pad columns b..bn-1 zero), the B operand of the 3xTF32 pass
+// inverse of split_tf32_rm (tests): dst[r + c*ldd] = src[r*lds + c] + src[r*lds + lo_off + c]
+cudaError_t splitsum_rm_to_cm(int64_t rows, int cols, const float* src, int64_t lds, int64_t lo_off, float* dst,
+                              int64_t ldd, cudaStream_t st);
+cudaError_t split_tf32_w(int64_t rows, int b, int bn, const float* W, int64_t ldw, float* dst, int64_t ldd,
+                         cudaStream_t st);
 
 // skinny tcgen05 GEMMs (k_skinny_tc.cu)
 struct SkinnyNN {                 // D[rows x b] = C - [A0 | A1] [B0 | B1]^T

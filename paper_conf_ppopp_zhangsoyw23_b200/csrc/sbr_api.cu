@@ -63,6 +63,9 @@ struct sbr_ctx {
   __half *Sh = nullptr, *Yh = nullptr, *Zh = nullptr, *Wh = nullptr, *WtXh = nullptr, *Xh = nullptr, *Wrh = nullptr,
          *Bl = nullptr, *Gh = nullptr;
   float* Hb = nullptr;
+  // 3xTF32 tensor-core path: [hi | lo] splits (row-major, lo at column tlo) of Y, Z, W^T X, and W_t
+  float *YS = nullptr, *ZS = nullptr, *GS = nullptr, *WS = nullptr;
+  int64_t tlo = 0, ldts = 0, ldws = 0;
   float* GH = nullptr;     // per-block G_t / H_t (k x b, ld nb, panel t at offset t*nb*b), zeroed per block
   __half* Ph = nullptr;    // fp16 P^T (b x k, row-major) of the lazy update
   void* chol_ws = nullptr;  // CholeskyQR panel workspace (Gram sets, barrier, LU), zeroed at allocation
@@ -84,6 +87,7 @@ struct sbr_ctx {
   int rank = 0, nranks = 1;
   nccl::Comm comm = nullptr;
   bool force_coll = false;   // SBR_DIST_COLLECTIVES=1: issue the exchanges even with one rank (tests)
+  bool tf32_tc = true;       // SBR_TF32_TC=0: 3xTF32 mode on the SIMT fp32 kernels (ablation)
 };
 
 namespace {
@@ -166,8 +170,9 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
     off += align_up(floats * sizeof(float));
     return o;
   };
+  const int64_t strip_cols = (nb + 127) / 128 * 128;   // the 3xTF32 pass reads whole 128-column tiles
   const size_t oY = take((size_t)n * nb), oX = take((size_t)n * nb), oZ = take((size_t)n * nb),
-               oW = take((size_t)n * nb), oS = take((size_t)n * nb), oWtX = take((size_t)nb * nb),
+               oW = take((size_t)n * nb), oS = take((size_t)n * strip_cols), oWtX = take((size_t)nb * nb),
                oP = take((size_t)nb * 64), oG = take((size_t)nb * 64), oPv = take(pw.v), oPt = take(pw.tau),
                oPr = take(pw.r), oPq = take(pw.q), oPm = take(pw.misc), oF = take(64);
   // fp16 operands of the tensor-core path (sizes in floats = halves / 2)
@@ -184,9 +189,18 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
                oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take(panel_chol_ws_bytes() / sizeof(float) + 64),
                oGH = take((size_t)2 * nb * nb), oPh = take((size_t)64 * ldk / 2 + 8);
+  const int64_t tlo = (nb + 31) / 32 * 32, ldts = 2 * tlo, ldws = (M + 3) / 4 * 4;
+  size_t oYS = 0, oZS = 0, oGS = 0, oWS = 0;
+  if (mode == SBR_3XTF32) {
+    oYS = take((size_t)n * ldts);
+    oZS = take((size_t)n * ldts);
+    oGS = take((size_t)nb * ldts);
+    oWS = take((size_t)ldws * 64);
+  }
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
-  if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb) return SBR_OK;
+  if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb && h->ws_mode == mode)
+    return SBR_OK;
   if (h->ws) {
     cudaFree(h->ws);
     h->ws = nullptr;
@@ -229,6 +243,13 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->chol_ws = base + oGram;
   h->GH = (float*)(base + oGH);
   h->Ph = (__half*)(base + oPh);
+  h->tlo = tlo;
+  h->ldts = ldts;
+  h->ldws = ldws;
+  h->YS = mode == SBR_3XTF32 ? (float*)(base + oYS) : nullptr;
+  h->ZS = mode == SBR_3XTF32 ? (float*)(base + oZS) : nullptr;
+  h->GS = mode == SBR_3XTF32 ? (float*)(base + oGS) : nullptr;
+  h->WS = mode == SBR_3XTF32 ? (float*)(base + oWS) : nullptr;
   h->pfail = panel_chol_fail(h->chol_ws);
   if (cudaMemset(h->chol_ws, 0, panel_chol_ws_bytes()) != cudaSuccess) return SBR_ERR_CUDA;
   h->ldbl = 2 * ldk + 128;
@@ -287,6 +308,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
   const int64_t ldn = n;        // ld of the block buffers
   const bool tc16 = (mode == SBR_FP16_FP32ACC);  // tcgen05 kind::f16 path
+  // 3xTF32 on tcgen05 kind::tf32 (pass + Z + SYR2K); the SIMT fp32 kernels remain for A that
+  // TMA cannot address (lda % 4 != 0) and for the SBR_TF32_TC=0 ablation
+  const bool tc32 = !tc16 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0;
   if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper)
     Scope sc(h, SBR_K_OTHER, 6.0 * n * n, 0);
     SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, st), "shadow_init");
@@ -303,8 +327,10 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int64_t ldwb = W ? ldw : ldn;
     float* OA = A + r0 + r0 * lda;
     const int sw = std::min<int64_t>((int64_t)(p - 1) * b, M);  // OA columns rewritten during the block
-    if (sw > 0 && !tc16) {
-      SBR_CK(cudaMemcpy2DAsync(h->Strip, ldn * sizeof(float), OA, lda * sizeof(float), M * sizeof(float), sw,
+    if (sw > 0 && !tc16) {  // tc32: whole 128-column tiles of the strip
+      const int64_t swc = tc32 ? std::min<int64_t>((sw + 127) / 128 * 128, M) : sw;
+      Scope sc(h, SBR_K_OTHER, 8.0 * M * swc, 0);
+      SBR_CK(cudaMemcpy2DAsync(h->Strip, ldn * sizeof(float), OA, lda * sizeof(float), M * sizeof(float), swc,
                                cudaMemcpyDeviceToDevice, st),
              "strip copy");
     }
@@ -524,7 +550,32 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
                "W merge");
         h->launches += 2;
       }
-      {  // ---- a4 (3xTF32 mode, SIMT fp32 for now): OA frozen = A + strip copy
+      if (tc32) {  // ---- a4 (3xTF32 on tcgen05): OA frozen = A + strip copy, 32 W columns per launch
+        Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 12.0 * M * b, 3 * 2.0 * M * M * b);
+        SBR_CK(zero_matrix(M, b, h->Xb + tb * ldn, ldn, st), "zero X_t");
+        for (int c = 0; c < b; c += 32) {
+          const int bh = std::min(32, b - c);
+          SBR_CK(split_tf32_w(M, bh, 32, Wb + (tb + c) * ldwb, ldwb, h->WS, h->ldws, st), "split W_t");
+          PassTf32Launch pl{};
+          pl.A = A;
+          pl.n = n;
+          pl.lda = lda;
+          pl.r0 = r0;
+          pl.S = h->Strip;
+          pl.lds = ldn;
+          pl.sw = sw;
+          pl.WS = h->WS;
+          pl.ldws = h->ldws;
+          pl.M = M;
+          pl.b = bh;
+          pl.X = h->Xb + (tb + c) * ldn;
+          pl.ldx = ldn;
+          pl.num_sms = h->nsm;
+          SBR_CK(launch_pass_tf32(pl, st), "pass_tf32");
+          h->launches += 2;
+        }
+        h->launches += 1;
+      } else {  // ---- a4 (3xTF32 mode, SIMT fp32): OA frozen = A + strip copy
         Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 8.0 * M * b, 2.0 * M * M * b);
         SBR_CK(sym_pass(M, b, OA, lda, h->Strip, ldn, sw, Wb + tb * ldwb, ldwb, h->Xb + tb * ldn, ldn, st),
                "pass");
@@ -585,6 +636,46 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       gs.num_sms = h->nsm;
       SBR_CK(launch_syr2k_tc(gs, st), "syr2k_tc");
       h->launches += 3;
+    } else if (Mt > 0 && tc32) {   // a6 in 3xTF32 on tcgen05: split Y, W^T X; Z (split) ; SYR2K
+      Scope sc(h, SBR_K_SYR2K, 8.0 * Mt * Mt + 4.0 * Mt * kk * 8,
+               3 * (2.0 * Mt * Mt * kk + 2.0 * Mt * kk * kk));
+      SBR_CK(split_tf32_rm(Mt, kk, h->Yb + s, ldn, h->YS + s * h->ldts, h->ldts, h->tlo, st), "split Y");
+      SBR_CK(split_tf32_rm(kk, kk, h->WtX, nb, h->GS, h->ldts, h->tlo, st), "split W^T X");
+      GemmTcLaunch gz{};
+      gz.A0 = gz.A1 = (const __half*)h->YS;
+      gz.B0 = gz.B1 = (const __half*)h->GS;
+      gz.K = kk;
+      gz.lo_off = h->tlo;
+      gz.a_rows = M;
+      gz.ld_a = h->ldts;
+      gz.b_rows = kk;
+      gz.ld_b = h->ldts;
+      gz.arow0 = s;
+      gz.brow0 = 0;
+      gz.Mrows = Mt;
+      gz.Ncols = kk;
+      gz.X = h->Xb + s;
+      gz.ldx = ldn;
+      gz.Zs = h->ZS + s * h->ldts;
+      gz.ldz = h->ldts;
+      gz.num_sms = h->nsm;
+      SBR_CK(launch_zform_tf32(gz, st), "zform_tf32");
+      GemmTcLaunch gs{};
+      gs.A0 = (const __half*)h->YS;
+      gs.A1 = (const __half*)h->ZS;
+      gs.B0 = (const __half*)h->ZS;
+      gs.B1 = (const __half*)h->YS;
+      gs.K = kk;
+      gs.lo_off = h->tlo;
+      gs.a_rows = gs.b_rows = M;
+      gs.ld_a = gs.ld_b = h->ldts;
+      gs.arow0 = gs.brow0 = s;
+      gs.Mrows = gs.Ncols = Mt;
+      gs.C = A + (r0 + s) + (r0 + s) * lda;
+      gs.ldc = lda;
+      gs.num_sms = h->nsm;
+      SBR_CK(launch_syr2k_tf32(gs, st), "syr2k_tf32");
+      h->launches += 4;
     } else if (Mt > 0) {
       Scope sc(h, SBR_K_SYR2K, 4.0 * Mt * Mt + 4.0 * Mt * kk * 3, 2.0 * Mt * Mt * kk + 2.0 * Mt * kk * kk);
       SBR_CK(gemm_nn(Mt, kk, kk, -0.5f, h->Yb + s, ldn, h->WtX, nb, false, 1.f, h->Xb + s, ldn, h->Zb + s, ldn, st),
@@ -620,6 +711,8 @@ int sbr_create(sbr_handle_t* out, int device, void* stream) {
   cudaDeviceGetAttribute(&h->nsm, cudaDevAttrMultiProcessorCount, device);
   const char* pm = getenv("SBR_PANEL");   // "tsqr": the paper's TSQR panel only (ablation)
   if (pm && strcmp(pm, "tsqr") == 0) h->panel_mode = 1;
+  const char* tt = getenv("SBR_TF32_TC");  // "0": 3xTF32 mode on the SIMT fp32 kernels (ablation)
+  if (tt && strcmp(tt, "0") == 0) h->tf32_tc = false;
   *out = h;
   return SBR_OK;
 }
@@ -990,6 +1083,107 @@ int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
   gz.num_sms = h->nsm;
   SBR_CK(launch_zform_tc(gz, st), "zform_tc");
   f16_to_f32_kernel<<<256, 256, 0, st>>>(M, K, (__half*)zh.p, kp, true, Z, ldz);
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
+
+int sbr_test_pass_tf32(sbr_handle_t h, int64_t M, int b, const float* OA, int64_t ldoa, const float* S,
+                       int64_t lds, int64_t sw, const float* W, int64_t ldw, float* X, int64_t ldx) {
+  if (!h) return -1;
+  if (M < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (ldoa < M || ldoa % 4 != 0) return -5;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t ldws = (M + 3) / 4 * 4;
+  DevBuf ws(sizeof(float) * ldws * 64);
+  if (!ws.p) return SBR_ERR_NOMEM;
+  SBR_CK(zero_matrix(M, b, X, ldx, st), "zero X");
+  for (int c = 0; c < b; c += 32) {
+    const int bh = std::min(32, b - c);
+    SBR_CK(split_tf32_w(M, bh, 32, W + c * ldw, ldw, (float*)ws.p, ldws, st), "split W");
+    PassTf32Launch pl{};
+    pl.A = OA;
+    pl.n = M;
+    pl.lda = ldoa;
+    pl.r0 = 0;
+    pl.S = S;
+    pl.lds = lds;
+    pl.sw = S ? sw : 0;
+    pl.WS = (float*)ws.p;
+    pl.ldws = ldws;
+    pl.M = M;
+    pl.b = bh;
+    pl.X = X + c * ldx;
+    pl.ldx = ldx;
+    pl.num_sms = h->nsm;
+    SBR_CK(launch_pass_tf32(pl, st), "pass_tf32");
+  }
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
+
+int sbr_test_syr2k_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* Z, int64_t ldz,
+                        float* C, int64_t ldc) {
+  if (!h) return -1;
+  if (M < 1) return -2;
+  if (K < 1) return -3;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t lo = (K + 31) / 32 * 32, ld = 2 * lo;
+  DevBuf ys(sizeof(float) * M * ld), zs(sizeof(float) * M * ld);
+  if (!ys.p || !zs.p) return SBR_ERR_NOMEM;
+  SBR_CK(split_tf32_rm(M, K, Y, ldy, (float*)ys.p, ld, lo, st), "split Y");
+  SBR_CK(split_tf32_rm(M, K, Z, ldz, (float*)zs.p, ld, lo, st), "split Z");
+  GemmTcLaunch gs{};
+  gs.A0 = (const __half*)ys.p;
+  gs.A1 = (const __half*)zs.p;
+  gs.B0 = (const __half*)zs.p;
+  gs.B1 = (const __half*)ys.p;
+  gs.K = K;
+  gs.lo_off = lo;
+  gs.a_rows = gs.b_rows = M;
+  gs.ld_a = gs.ld_b = ld;
+  gs.Mrows = gs.Ncols = M;
+  gs.C = C;
+  gs.ldc = ldc;
+  gs.num_sms = h->nsm;
+  SBR_CK(launch_syr2k_tf32(gs, st), "syr2k_tf32");
+  SBR_CK(cudaStreamSynchronize(st), "sync");
+  return SBR_OK;
+}
+
+int sbr_test_zform_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
+                        const float* X, int64_t ldx, float* Z, int64_t ldz) {
+  if (!h) return -1;
+  if (M < 1) return -2;
+  if (K < 1) return -3;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t lo = (K + 31) / 32 * 32, ld = 2 * lo;
+  DevBuf ys(sizeof(float) * M * ld), gs_(sizeof(float) * K * ld), zs(sizeof(float) * M * ld);
+  if (!ys.p || !gs_.p || !zs.p) return SBR_ERR_NOMEM;
+  SBR_CK(split_tf32_rm(M, K, Y, ldy, (float*)ys.p, ld, lo, st), "split Y");
+  SBR_CK(split_tf32_rm(K, K, G, ldg, (float*)gs_.p, ld, lo, st), "split G");
+  GemmTcLaunch gz{};
+  gz.A0 = gz.A1 = (const __half*)ys.p;
+  gz.B0 = gz.B1 = (const __half*)gs_.p;
+  gz.K = K;
+  gz.lo_off = lo;
+  gz.a_rows = M;
+  gz.ld_a = ld;
+  gz.b_rows = K;
+  gz.ld_b = ld;
+  gz.Mrows = M;
+  gz.Ncols = K;
+  gz.X = X;
+  gz.ldx = ldx;
+  gz.Zs = (float*)zs.p;
+  gz.ldz = ld;
+  gz.num_sms = h->nsm;
+  SBR_CK(launch_zform_tf32(gz, st), "zform_tf32");
+  // Z = hi + lo back to column-major fp32
+  SBR_CK(splitsum_rm_to_cm(M, K, (const float*)zs.p, ld, lo, Z, ldz, st), "Z unsplit");
   SBR_CK(cudaStreamSynchronize(st), "sync");
   return SBR_OK;
 }
