@@ -44,6 +44,8 @@ def parse():
     p.add_argument("--nb", type=int, default=CONFIG4["nb"])
     p.add_argument("--mode", default=CONFIG4["mode"])
     p.add_argument("--e2e-steps", type=int, default=2)
+    p.add_argument("--form-q-steps", type=int, default=1,
+                   help="also time sbr_form_q (Q = prod (I - W Y^T), 3xTF32) on the last step's output (0: skip)")
     p.add_argument("--profile-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-sample-s", type=float, default=15.0)
@@ -234,7 +236,9 @@ def main():
     import workloads
 
     n, b, nb, mode = args.n, args.b, args.nb, args.mode
-    seed = workloads.config_seed(4)
+    cfg_name = {(32768, 32, 1024, "fp16"): "config4", (16384, 32, 1024, "3xtf32"): "config3"}.get(
+        (n, b, nb, mode), "custom")
+    seed = workloads.config_seed(3 if cfg_name == "config3" else 4)
     stream = torch.cuda.current_stream()
     if world > 1:
         # one matrix across the ranks (sbr_reduce_dist, strong scaling): NCCL communicator
@@ -311,6 +315,8 @@ def main():
     if dom == "syr2k":
         achieved = st["flops"] / max(1, st["launches"]) / (avg_ms / 1e3) / 1e12
         peak = peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops"))
+        if mode == "3xtf32":   # tf32 dense peak = bf16 x the guide's nominal ratio 1.125 / 2.25
+            peak *= 0.5
         roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                 "frac": achieved / peak, "traffic": None}
     else:
@@ -335,6 +341,27 @@ def main():
                                 f"the events)"})
     breakdown = {c: {"ms_per_step": kst[c]["ms"] / nprof, "launches_per_step": kst[c]["launches"] / nprof}
                  for c in classes}
+
+    # sbr_form_q on the profiled step's output: not part of the step, reported beside it
+    formq = None
+    if args.form_q_steps > 0 and world == 1 and n > b:
+        q = torch.empty((n, n), dtype=torch.float32, device=a.device)
+        fq_ms = []
+        for _ in range(args.form_q_steps + 1):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            h.form_q(a, w, b, nb, q=q)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            fq_ms.append(e0.elapsed_time(e1))
+        fq = statistics.median(fq_ms[1:])
+        ncols = n - b
+        alg = sum(4.0 * (n - c0 - b) ** 2 * min(nb, ncols - c0) for c0 in range(0, ncols, nb))
+        formq = {"ms": fq, "algorithmic_tflops": alg / (fq / 1e3) / 1e12,
+                 "tensor_tflops_3xtf32": 3 * alg / (fq / 1e3) / 1e12, "steps": args.form_q_steps,
+                 "note": "Q = prod_J (I - W_J Y_J^T) by backward accumulation, 2 tcgen05 3xTF32 products per "
+                         "block, algorithmic flops sum_J 4 M_J^2 k_J; first call (allocation) untimed"}
+        del q
 
     # end-to-end through the public API with HOST buffers (H2D of A + D2H of the band per step)
     e2e = None
@@ -403,7 +430,7 @@ def main():
             "vs_baseline": None,
             "dtype": "f32" if mode == "3xtf32" else "f16",
             "data": "synthetic",
-            "config": {"workload": f"config4: n={n} random symmetric U[-1,1) (seed {seed}), b={b}, nb={nb}, "
+            "config": {"workload": f"{cfg_name}: n={n} random symmetric U[-1,1) (seed {seed}), b={b}, nb={nb}, "
                                    f"{'FP16-in/FP32-acc' if mode == 'fp16' else '3xTF32'}",
                        "n": n, "b": b, "nb": nb, "mode": mode,
                        "parallelism": f"sbr_reduce_dist over {world} GPUs: per-panel pass sharded by lower "
@@ -416,6 +443,7 @@ def main():
             "breakdown": breakdown,
             "cpu_baseline": cpu,
             "e2e": e2e,
+            "form_q": formq,
             "gpu_launches": launches,
             "clocks": clk.summary(),
             "step_ms": step_ms,

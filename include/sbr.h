@@ -116,6 +116,24 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb,
                     float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw,
                     int outputs);
 
+/* Explicit Q of a reduction ("Q = I - W Y^T", P:115 A = Q B Q^T):
+ *   Q = prod_J (I - W_J Y_J^T), block J (c0 = J nb, k_J = min(nb, n-b-c0) reflector columns)
+ *   acting on rows/cols c0+b .. n-1, with Y_J and W_J read from sbr_reduce's outputs (same
+ *   n, b, nb): Y_J column jj = unit at row c0+jj+b, tail A[c0+jj+b+1 : n, c0+jj], zero above;
+ *   W_J = W[c0+b : n, c0 : c0+k_J].
+ *   A   : device fp32, column-major, lda >= n (read only).               (args 5, 6)
+ *   W   : device fp32, column-major, ldw >= n (read only).               (args 7, 8)
+ *   Q   : device fp32, column-major n x n, ldq >= n; overwritten.        (args 9, 10)
+ * Backward accumulation, last block first: Q[r0:, r0:] -= W_J (Y_J^T Q[r0:, r0:]), both
+ * products on tcgen05 in 3xTF32 (FP32-accurate) whatever the reduction's mode: Q feeds the
+ * eigenvector back-transformation, where FP32 accuracy is what the paper targets.
+ * Temporary split operands (about 8 (n-b)^2 + 16 n nb bytes) are allocated stream-ordered
+ * and freed before return; the call is stream-ordered and returns after enqueue.
+ * Returns 0, -1 (h), -2 (n < 1), -3 (b not in 1..64), -4 (nb), -5 (A NULL), -6 (lda),
+ * -7 (W NULL), -8 (ldw), -9 (Q NULL), -10 (ldq), SBR_ERR_NOMEM, SBR_ERR_CUDA. */
+int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
+               float* Q, int64_t ldq);
+
 /* ---- Multi-GPU (one process per GPU, NCCL over NVLink/NVSwitch) ----
  *
  * sbr_get_unique_id: rank 0 creates the 128-byte NCCL unique id (host call, no device work)

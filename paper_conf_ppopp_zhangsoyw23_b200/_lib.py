@@ -48,6 +48,7 @@ SIGNATURES = {
     "sbr_get_unique_id": (_i, [_p]),
     "sbr_create_dist": (_i, [ctypes.POINTER(ctypes.c_void_p), _i, _p, _p, _i, _i]),
     "sbr_reduce_dist": (_i, [_h, _i, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_form_q": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_rank": (_i, [_h]),
     "sbr_nranks": (_i, [_h]),
     # kernel-level test hooks (include/sbr_testing.h)

@@ -123,6 +123,22 @@ class Handle:
                                _ptr(w), n), "sbr_reduce")
         return ab, w
 
+    def form_q(self, A, w, b: int, nb: int, q=None):
+        """Explicit Q = prod_J (I - W_J Y_J^T) from :meth:`reduce`'s outputs (A holding Y, and ``w``)
+        with the same b, nb (sbr_form_q; 3xTF32 on tcgen05).  Returns the (n, n) float32 tensor
+        ``q`` with ``q[c, r] = Q(r, c)`` (column-major Q, i.e. ``Q = q.T``)."""
+        import torch
+
+        n = int(A.shape[0])
+        if A.dim() != 2 or A.shape[1] != n or A.dtype != torch.float32 or not A.is_cuda or not A.is_contiguous():
+            raise ValueError("A must be a contiguous square float32 CUDA tensor")
+        if w is None or w.dtype != torch.float32 or not w.is_contiguous() or w.shape[-1] != n:
+            raise ValueError("w must be the (n-b, n) float32 tensor returned by reduce")
+        if q is None:
+            q = torch.empty((n, n), dtype=torch.float32, device=A.device)
+        check(lib().sbr_form_q(self._h, n, int(b), int(nb), _ptr(A), n, _ptr(w), n, _ptr(q), n), "sbr_form_q")
+        return q
+
     def reduce_dist(self, A, b: int, nb: int, mode="fp16", want_w: bool = True, ab=None, w=None):
         """One matrix across the handle's communicator (collective; see sbr_reduce_dist).
 

@@ -48,7 +48,7 @@ template <bool TF> struct GCfg {
 // tile index -> (I, Jc); SYR2K: the lower tiles, row I holding floor(I*BM/BN)+1 tiles of BN columns
 template <int MODE, int BN>
 SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
-  if (MODE == 1) {  // ZFORM: full grid, row-major
+  if (MODE != 0) {  // ZFORM / GEMM modes: full grid, row-major
     I = t / ntn;
     Jc = t % ntn;
   } else {
@@ -194,17 +194,18 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       const int64_t row = (int64_t)I * G_BM + rit;
       if (row >= Mrows) continue;
       const int64_t col0 = (int64_t)Jc * G_BN + chalf * 64;
-      if (MODE == 0) {
+      if (MODE == 0 || MODE == 3) {   // SYR2K: lower elements; GEMM_SUB: all of C
         float* cp = C + row + col0 * ldc;
 #pragma unroll
         for (int c = 0; c < 64; ++c)
-          if (col0 + c <= row) __stcs(cp + c * ldc, __ldcs(cp + c * ldc) - acc[c]);
+          if (MODE == 0 ? (col0 + c <= row) : (col0 + c < Ncols)) __stcs(cp + c * ldc, __ldcs(cp + c * ldc) - acc[c]);
       } else {   // Z split: hi = rna_tf32(z), lo = rna_tf32(z - hi), row-major
         float* zp = (float*)Zout + row * ldz + col0;
 #pragma unroll
         for (int c = 0; c < 64; ++c) {
           if (col0 + c < Ncols) {
-            const float z = fmaf(-0.5f, acc[c], __ldcs(X + row + (col0 + c) * ldx));
+            // ZFORM: z = X - acc/2 ; GEMM_SPLIT: z = acc
+            const float z = MODE == 1 ? fmaf(-0.5f, acc[c], __ldcs(X + row + (col0 + c) * ldx)) : acc[c];
             const float hi = tf32_rna(z);
             zp[c] = hi;
             zp[c + zlo_off] = tf32_rna(z - hi);
@@ -334,12 +335,14 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   const int grid = std::min(ntiles, p.num_sms);
   return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
                     (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
-                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.lo_off);
+                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off);
 }
 
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, false>(p, st); }
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, false>(p, st); }
 cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, true>(p, st); }
 cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, true>(p, st); }
+cudaError_t launch_gemm_split_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<2, true>(p, st); }
+cudaError_t launch_gemm_sub_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<3, true>(p, st); }
 
 }  // namespace sbr

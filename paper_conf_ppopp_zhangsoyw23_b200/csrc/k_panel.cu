@@ -391,6 +391,7 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
   const int b = a.b;
   const int lane = lane_id(), warp = warp_id();
   cg::grid_group grid = cg::this_grid();
+  pdl_wait();                                 // launched with PDL: predecessor complete
   if (a.run_if && *a.run_if == 0) return;    // CholeskyQR already factored this panel
   float x[CPW][P_SN];
   PTRACE(0);
@@ -661,8 +662,19 @@ static cudaError_t launch_panel_t(PanelArgs& a, int max_ctas, cudaStream_t st) {
     nodes = (nodes + a.arity - 1) / a.arity;
     if (a.nlev >= kPanelMaxLev) return cudaErrorInvalidValue;
   }
-  void* args[] = {&a};
-  return cudaLaunchCooperativeKernel((const void*)kern, dim3(L), dim3(P_NW * 32), args, smem, st);
+  cudaLaunchConfig_t cfg = {};   // cooperative + programmatic dependent launch (see k_panel_chol.cu)
+  cfg.gridDim = dim3(L);
+  cfg.blockDim = dim3(P_NW * 32);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, a);
 }
 
 cudaError_t launch_panel(PanelArgs& a, int max_ctas, cudaStream_t st) {

@@ -289,6 +289,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     }
   };
   stamp(0);
+  pdl_wait();   // launched with PDL: the predecessor (lazy update) must be complete before any read
   // ---- load the CTA's rows (column-major fp32 -> row-major fp64): all loads issued first
   {
     constexpr int CPW = (B + 7) / 8, RPL = pc_maxr<B>() / 32;
@@ -683,8 +684,21 @@ static cudaError_t launch_chol_t(PanelArgs& a, void* ws, unsigned launch, cudaSt
   if ((int64_t)G * pc_maxr<B>() < a.m) G = (int)((a.m + pc_maxr<B>() - 1) / pc_maxr<B>());
   if (G > cap || G < 1) return cudaErrorNotSupported;   // caller uses TSQR
   unsigned char* wsp = (unsigned char*)ws;
-  void* args[] = {&a, &wsp, &launch};
-  return cudaLaunchCooperativeKernel((const void*)kern, dim3(G), dim3(PC_THREADS), args, smem, st);
+  // cooperative (grid-wide barriers) AND programmatic dependent launch: the launch and the
+  // prologue overlap the tail of the lazy update; all CTAs are co-resident once it drains
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(G);
+  cfg.blockDim = dim3(PC_THREADS);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeCooperative;
+  at[0].val.cooperative = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, a, wsp, launch);
 }
 
 cudaError_t launch_panel_chol(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st) {

@@ -407,6 +407,42 @@ cudaError_t splitsum_rm_to_cm(int64_t rows, int cols, const float* src, int64_t 
   return cudaGetLastError();
 }
 
+__global__ void split_tf32_cm_kernel(int64_t rows, int cols, const float* __restrict__ src, int64_t lds,
+                                     bool unit_y, float* __restrict__ dst, int64_t ldd, int64_t lo_off) {
+  const int64_t rpad = (rows + 31) / 32 * 32;
+  for (int64_t c = blockIdx.y; c < cols; c += gridDim.y) {
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < rpad; r += (int64_t)gridDim.x * blockDim.x) {
+      float a = 0.f;
+      if (r < rows) a = unit_y ? (r < c ? 0.f : r == c ? 1.f : src[r + c * lds]) : src[r + c * lds];
+      const float hi = tf32_rna(a);
+      dst[c * ldd + r] = hi;
+      if (r < rows) dst[c * ldd + lo_off + r] = tf32_rna(a - hi);
+    }
+  }
+}
+
+cudaError_t split_tf32_cm(int64_t rows, int cols, const float* src, int64_t lds, bool unit_y, float* dst,
+                          int64_t ldd, int64_t lo_off, cudaStream_t st) {
+  if (rows <= 0 || cols <= 0) return cudaSuccess;
+  const int gx = (int)std::min<int64_t>((rows + 255) / 256, 64);
+  const int gy = std::min(cols, 2048);
+  split_tf32_cm_kernel<<<dim3(gx, gy), 256, 0, st>>>(rows, cols, src, lds, unit_y, dst, ldd, lo_off);
+  return cudaGetLastError();
+}
+
+__global__ void set_identity_kernel(int64_t n, float* Q, int64_t ldq) {
+  for (int64_t c = blockIdx.y; c < n; c += gridDim.y)
+    for (int64_t r = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x)
+      Q[r + c * ldq] = r == c ? 1.f : 0.f;
+}
+
+cudaError_t set_identity(int64_t n, float* Q, int64_t ldq, cudaStream_t st) {
+  if (n <= 0) return cudaSuccess;
+  set_identity_kernel<<<dim3((unsigned)std::min<int64_t>((n + 255) / 256, 64), (unsigned)std::min<int64_t>(n, 4096)),
+                        256, 0, st>>>(n, Q, ldq);
+  return cudaGetLastError();
+}
+
 __global__ void split_tf32_w_kernel(int64_t rows, int b, int bn, const float* __restrict__ W, int64_t ldw,
                                     float* __restrict__ dst, int64_t ldd) {
   const int64_t total = rows * bn;

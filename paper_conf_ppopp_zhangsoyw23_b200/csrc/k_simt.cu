@@ -123,10 +123,110 @@ __global__ void __launch_bounds__(256) gemm_nn_kernel(int64_t M, int N, int K, f
     }
 }
 
+// ---------------------------------------------------------------- skinny in-place update (3xTF32 chain)
+// D[M x N] += alpha * A[M x K] op(B), N <= 64, fp32 SIMT: the skinny steps a3/a5 of the 3xTF32
+// mode (X Y_c^T, Y P, W G).  Bound by fp32 FMA issue (8 FMA per A byte at N = 32), so the grid
+// is 128-row blocks x a K split sized to fill every SM twice; partial sums go to D with fp32
+// atomics (D = C in place, beta = 1).  Per thread 4 rows x NG*4 columns; A / B chunks of 32 K
+// staged through shared memory with a register prefetch of the next chunk.
+template <int NG>   // NG = N / 32 rounded up (1 or 2)
+__global__ void __launch_bounds__(256) skinny_upd_kernel(int64_t M, int N, int K, int kper, float alpha,
+                                                         const float* __restrict__ A, int64_t lda,
+                                                         const float* __restrict__ B, int64_t ldb, bool transB,
+                                                         float* D, int64_t ldd) {
+  constexpr int RB = 128, KC = 32, NC = 32 * NG;
+  __shared__ __align__(16) float As[KC][RB];
+  __shared__ __align__(16) float Bs[KC][NC];
+  const int64_t i0 = (int64_t)blockIdx.x * RB;
+  const int kb = blockIdx.y * kper, ke = min(K, kb + kper);
+  const int tr = threadIdx.x & 31, tc = threadIdx.x >> 5;   // rows tr*4.., cols tc*4*NG..
+  float acc[4][4 * NG];
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 4 * NG; ++v) acc[u][v] = 0.f;
+  float ra[16], rbv[4 * NG];
+  auto load = [&](int k0) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {   // A: 32 k x 128 rows, rows contiguous
+      const int e = threadIdx.x + q * 256, ii = e & (RB - 1), kk = e >> 7;
+      const int64_t i = i0 + ii;
+      const int k = k0 + kk;
+      ra[q] = (i < M && k < ke) ? __ldg(A + i + (int64_t)k * lda) : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < 4 * NG; ++q) {   // B: 32 k x NC columns
+      const int e = threadIdx.x + q * 256;
+      int kk, jj;
+      if (transB) { jj = e % NC; kk = e / NC; } else { kk = e % KC; jj = e / KC; }
+      const int k = k0 + kk;
+      rbv[q] = (k < ke && jj < N) ? __ldg(transB ? B + jj + (int64_t)k * ldb : B + k + (int64_t)jj * ldb) : 0.f;
+    }
+  };
+  auto store = [&]() {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const int e = threadIdx.x + q * 256;
+      As[e >> 7][e & (RB - 1)] = ra[q];
+    }
+#pragma unroll
+    for (int q = 0; q < 4 * NG; ++q) {
+      const int e = threadIdx.x + q * 256;
+      if (transB) Bs[e / NC][e % NC] = rbv[q];
+      else Bs[e % KC][e / KC] = rbv[q];
+    }
+  };
+  if (kb < ke) load(kb);
+  for (int k0 = kb; k0 < ke; k0 += KC) {
+    __syncthreads();
+    store();
+    __syncthreads();
+    if (k0 + KC < ke) load(k0 + KC);   // next chunk's loads in flight during this chunk's FMAs
+#pragma unroll 8
+    for (int kk = 0; kk < KC; ++kk) {
+      const float4 a4 = *reinterpret_cast<const float4*>(&As[kk][tr * 4]);
+      const float a[4] = {a4.x, a4.y, a4.z, a4.w};
+      float bb[4 * NG];
+#pragma unroll
+      for (int g = 0; g < NG; ++g) {
+        const float4 b4 = *reinterpret_cast<const float4*>(&Bs[kk][tc * 4 + 32 * g]);
+        bb[4 * g] = b4.x; bb[4 * g + 1] = b4.y; bb[4 * g + 2] = b4.z; bb[4 * g + 3] = b4.w;
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u)
+#pragma unroll
+        for (int v = 0; v < 4 * NG; ++v) acc[u][v] = fmaf(a[u], bb[v], acc[u][v]);
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u) {
+    const int64_t i = i0 + tr * 4 + u;
+    if (i >= M) continue;
+#pragma unroll
+    for (int g = 0; g < NG; ++g)
+#pragma unroll
+      for (int v = 0; v < 4; ++v) {
+        const int j = tc * 4 + 32 * g + v;
+        if (j < N) atomicAdd(D + i + (int64_t)j * ldd, alpha * acc[u][4 * g + v]);
+      }
+  }
+}
+
 cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_t lda, const float* B,
                     int64_t ldb, bool transB, float beta, const float* C, int64_t ldc, float* D, int64_t ldd,
                     cudaStream_t st) {
   if (M <= 0 || N <= 0) return cudaSuccess;
+  if (N <= 64 && beta == 1.f && C == D && ldc == ldd && K > 0) {   // in-place skinny update
+    const int gx = (int)((M + 127) / 128);
+    int ks = std::max(1, std::min((K + 63) / 64, (2 * 148 + gx - 1) / gx));
+    const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
+    ks = (K + kper - 1) / kper;
+    if (N <= 32)
+      skinny_upd_kernel<1><<<dim3(gx, ks), 256, 0, st>>>(M, N, K, kper, alpha, A, lda, B, ldb, transB, D, ldd);
+    else
+      skinny_upd_kernel<2><<<dim3(gx, ks), 256, 0, st>>>(M, N, K, kper, alpha, A, lda, B, ldb, transB, D, ldd);
+    return cudaGetLastError();
+  }
   dim3 grid((unsigned)((M + NN_T - 1) / NN_T), (N + NN_T - 1) / NN_T);
   gemm_nn_kernel<<<grid, 256, 0, st>>>(M, N, K, alpha, A, lda, B, ldb, transB, beta, C, ldc, D, ldd);
   return cudaGetLastError();

@@ -152,11 +152,22 @@ struct GemmTcLaunch {
   // (fp32 row-major, ld ldz) in the same split layout.
   int64_t lo_off = 0;
   float* Zs = nullptr;
+  int64_t zlo_off = -1;   // lo offset of the Zs output (default lo_off)
 };
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st);
+// general 3xTF32 products (sbr_form_q): Zs = split(A B^T) (row-major [hi | lo], Mrows x Ncols),
+// and C (column-major fp32, Mrows x Ncols) -= A B^T
+cudaError_t launch_gemm_split_tf32(const GemmTcLaunch& p, cudaStream_t st);
+cudaError_t launch_gemm_sub_tf32(const GemmTcLaunch& p, cudaStream_t st);
+// column-major src (rows x cols) -> dst row c = split of column c: dst[c*ldd + r] = rna_tf32(a),
+// dst[c*ldd + lo_off + r] = rna_tf32(a - hi), zeros in [rows, lo_off).  unit_y: src is the Y of
+// sbr_reduce's output (column c: zero above row c, 1 at row c, the stored tail below).
+cudaError_t split_tf32_cm(int64_t rows, int cols, const float* src, int64_t lds, bool unit_y, float* dst,
+                          int64_t ldd, int64_t lo_off, cudaStream_t st);
+cudaError_t set_identity(int64_t n, float* Q, int64_t ldq, cudaStream_t st);
 // fp32 column-major src (rows x cols) -> row-major split dst: dst[r*ldd + c] = rna_tf32(a),
 // dst[r*ldd + lo_off + c] = rna_tf32(a - hi), zeros in hi columns [cols, lo_off)
 cudaError_t split_tf32_rm(int64_t rows, int cols, const float* src, int64_t lds, float* dst, int64_t ldd,

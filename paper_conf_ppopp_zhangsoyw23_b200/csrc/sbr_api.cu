@@ -717,6 +717,92 @@ int sbr_create(sbr_handle_t* out, int device, void* stream) {
   return SBR_OK;
 }
 
+int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
+               float* Q, int64_t ldq) {
+  if (!h) return -1;
+  if (n < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (nb < b || nb % b != 0 || nb > 4096) return -4;
+  if (!A) return -5;
+  if (lda < n) return -6;
+  if (!W) return -7;
+  if (ldw < n) return -8;
+  if (!Q) return -9;
+  if (ldq < n) return -10;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  SBR_CK(set_identity(n, Q, ldq, st), "Q = I");
+  h->launches++;
+  const int64_t ncols = n - b;
+  if (ncols <= 0) return SBR_OK;
+  // backward accumulation Q = H_1 (H_2 (... I)): block J (last first) updates Q[r0:, r0:] -=
+  // W_J (Y_J^T Q[r0:, r0:]) -- two 3xTF32 tcgen05 products per block over [hi | lo] splits
+  const int64_t M0 = n - b;
+  const int64_t loM = (M0 + 31) / 32 * 32, ldM = 2 * loM;
+  const int64_t lok = (nb + 31) / 32 * 32, ldk = 2 * lok;
+  float *QS = nullptr, *YS = nullptr, *WS = nullptr, *TS = nullptr;
+  auto release = [&]() {
+    if (QS) cudaFreeAsync(QS, st);
+    if (YS) cudaFreeAsync(YS, st);
+    if (WS) cudaFreeAsync(WS, st);
+    if (TS) cudaFreeAsync(TS, st);
+  };
+  if (cudaMallocAsync((void**)&QS, sizeof(float) * M0 * ldM, st) != cudaSuccess ||
+      cudaMallocAsync((void**)&YS, sizeof(float) * nb * ldM, st) != cudaSuccess ||
+      cudaMallocAsync((void**)&WS, sizeof(float) * M0 * ldk, st) != cudaSuccess ||
+      cudaMallocAsync((void**)&TS, sizeof(float) * M0 * ldk, st) != cudaSuccess) {
+    cudaGetLastError();
+    release();
+    return SBR_ERR_NOMEM;
+  }
+  const int64_t nblk = (ncols + nb - 1) / nb;
+  cudaError_t e = cudaSuccess;
+  for (int64_t J = nblk - 1; J >= 0 && e == cudaSuccess; --J) {
+    const int64_t c0 = J * nb, r0 = c0 + b, M = n - r0;
+    const int k = (int)std::min<int64_t>(nb, ncols - c0);
+    float* Qs = Q + r0 + r0 * ldq;
+    Scope sc(h, SBR_K_OTHER, 4.0 * M * M * 4 + 8.0 * M * k * 4, 3 * 4.0 * M * M * k);
+    if ((e = split_tf32_cm(M, k, A + r0 + c0 * lda, lda, true, YS, ldM, loM, st)) != cudaSuccess) break;
+    if ((e = split_tf32_rm(M, k, W + r0 + c0 * ldw, ldw, WS, ldk, lok, st)) != cudaSuccess) break;
+    if ((e = split_tf32_cm(M, (int)M, Qs, ldq, false, QS, ldM, loM, st)) != cudaSuccess) break;
+    GemmTcLaunch g1{};   // T^T = Q_sub^T Y_J  (M x k), written split row-major
+    g1.A0 = g1.A1 = (const __half*)QS;
+    g1.B0 = g1.B1 = (const __half*)YS;
+    g1.K = M;
+    g1.lo_off = loM;
+    g1.a_rows = M;
+    g1.ld_a = ldM;
+    g1.b_rows = k;
+    g1.ld_b = ldM;
+    g1.Mrows = M;
+    g1.Ncols = k;
+    g1.Zs = TS;
+    g1.ldz = ldk;
+    g1.zlo_off = lok;
+    g1.num_sms = h->nsm;
+    if ((e = launch_gemm_split_tf32(g1, st)) != cudaSuccess) break;
+    GemmTcLaunch g2{};   // Q_sub -= W_J T
+    g2.A0 = g2.A1 = (const __half*)WS;
+    g2.B0 = g2.B1 = (const __half*)TS;
+    g2.K = k;
+    g2.lo_off = lok;
+    g2.a_rows = M;
+    g2.ld_a = ldk;
+    g2.b_rows = M;
+    g2.ld_b = ldk;
+    g2.Mrows = M;
+    g2.Ncols = M;
+    g2.C = Qs;
+    g2.ldc = ldq;
+    g2.num_sms = h->nsm;
+    if ((e = launch_gemm_sub_tf32(g2, st)) != cudaSuccess) break;
+    h->launches += 5;
+  }
+  release();
+  SBR_CK(e, "form_q");
+  return SBR_OK;
+}
+
 int sbr_set_stream(sbr_handle_t h, void* stream) {
   if (!h) return -1;
   h->stream = (cudaStream_t)stream;
