@@ -310,7 +310,12 @@ static int64_t pass_total_tiles(int NT, int C) {
   return T;
 }
 
-static int pass_group_cols(int b) { return b <= 32 ? 8 : 4; }   // C of launch_pass_tc's instantiation
+static int pass_variant();
+static int pass_group_cols(int b) {   // C of launch_pass_tc's instantiation
+  if (b <= 16) return 8;
+  if (b <= 32) return pass_variant() == 1 ? 4 : pass_variant() == 2 ? 2 : 8;
+  return 4;
+}
 
 void pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t* t1, int64_t* total) {
   const int NT = (int)((M + 127) / 128);
@@ -355,9 +360,25 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
                     p.X, p.ldx);
 }
 
+static int pass_variant() {   // SBR_PASS_CFG (tuning experiments only): 0 = C8/NS4, 1 = C4/NS5, 2 = C2/NS6
+  static int v = -1;
+  if (v < 0) {
+    const char* e = getenv("SBR_PASS_CFG");
+    v = e ? atoi(e) : 0;
+    if (v < 0 || v > 2) v = 0;
+  }
+  return v;
+}
+
 cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st) {
   if (p.b <= 16) return launch_pass_t<16, 8, 4>(p, st);
-  if (p.b <= 32) return launch_pass_t<32, 8, 4>(p, st);
+  if (p.b <= 32) {
+    switch (pass_variant()) {
+      case 1: return launch_pass_t<32, 4, 5>(p, st);
+      case 2: return launch_pass_t<32, 2, 6>(p, st);
+      default: return launch_pass_t<32, 8, 4>(p, st);
+    }
+  }
   return launch_pass_t<64, 4, 3>(p, st);
 }
 
