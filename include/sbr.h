@@ -127,8 +127,8 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb,
  * Backward accumulation, last block first: Q[r0:, r0:] -= W_J (Y_J^T Q[r0:, r0:]), both
  * products on tcgen05 in 3xTF32 (FP32-accurate) whatever the reduction's mode: Q feeds the
  * eigenvector back-transformation, where FP32 accuracy is what the paper targets.
- * Temporary split operands (about 8 (n-b)^2 + 16 n nb bytes) are allocated stream-ordered
- * and freed before return; the call is stream-ordered and returns after enqueue.
+ * The split operands (about 8 (n-b)^2 + 24 n nb bytes) live in handle-owned device memory,
+ * grown on demand and freed by sbr_destroy; the call is stream-ordered and returns after enqueue.
  * Returns 0, -1 (h), -2 (n < 1), -3 (b not in 1..64), -4 (nb), -5 (A NULL), -6 (lda),
  * -7 (W NULL), -8 (ldw), -9 (Q NULL), -10 (ldq), SBR_ERR_NOMEM, SBR_ERR_CUDA. */
 int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,

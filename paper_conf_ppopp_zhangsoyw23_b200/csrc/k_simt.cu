@@ -51,9 +51,85 @@ __global__ void __launch_bounds__(256) gemm_tn_kernel(int64_t rows, int64_t chun
     }
 }
 
+// Skinny reduction C[m1 x n2] += alpha * A^T B over `rows` (n2 <= 32): the 3xTF32 chain's
+// G = Y^T W0 and W^T X_t.  64 x 32 output tiles (no half-empty 64 x 64 tile at n2 = b = 32),
+// rows split to fill every SM twice, register prefetch of the next 64-row chunk, fp32 atomics.
+__global__ void __launch_bounds__(256) skinny_tn32_kernel(int64_t rows, int64_t chunk, int m1, int n2, float alpha,
+                                                          const float* __restrict__ A, int64_t lda,
+                                                          const float* __restrict__ B, int64_t ldb, float* C,
+                                                          int64_t ldc) {
+  constexpr int KC = 64, TI = 64, TJ = 32;
+  __shared__ float As[TI][KC + 1];
+  __shared__ float Bs[TJ][KC + 1];
+  const int i0 = blockIdx.x * TI;
+  const int64_t r_beg = (int64_t)blockIdx.z * chunk, r_end = min(rows, r_beg + chunk);
+  const int ti = threadIdx.x & 15, tj = threadIdx.x >> 4;   // outputs i = ti*4 .. +3, j = tj*2 .. +1
+  float acc[4][2] = {};
+  float ra[16], rb[8];
+  auto load = [&](int64_t r0) {
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {   // A: 64 rows (contiguous) x 64 columns
+      const int e = threadIdx.x + q * 256, rr = e & (KC - 1), ii = e >> 6;
+      const int64_t r = r0 + rr;
+      ra[q] = (r < r_end && i0 + ii < m1) ? __ldg(A + r + (int64_t)(i0 + ii) * lda) : 0.f;
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {    // B: 64 rows x 32 columns
+      const int e = threadIdx.x + q * 256, rr = e & (KC - 1), jj = e >> 6;
+      const int64_t r = r0 + rr;
+      rb[q] = (r < r_end && jj < n2) ? __ldg(B + r + (int64_t)jj * ldb) : 0.f;
+    }
+  };
+  if (r_beg < r_end) load(r_beg);
+  for (int64_t r0 = r_beg; r0 < r_end; r0 += KC) {
+    __syncthreads();
+#pragma unroll
+    for (int q = 0; q < 16; ++q) {
+      const int e = threadIdx.x + q * 256;
+      As[e >> 6][e & (KC - 1)] = ra[q];
+    }
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const int e = threadIdx.x + q * 256;
+      Bs[e >> 6][e & (KC - 1)] = rb[q];
+    }
+    __syncthreads();
+    if (r0 + KC < r_end) load(r0 + KC);
+#pragma unroll 16
+    for (int rr = 0; rr < KC; ++rr) {
+      float a[4], bb[2];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) a[u] = As[ti * 4 + u][rr];
+      bb[0] = Bs[tj * 2][rr];
+      bb[1] = Bs[tj * 2 + 1][rr];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        acc[u][0] = fmaf(a[u], bb[0], acc[u][0]);
+        acc[u][1] = fmaf(a[u], bb[1], acc[u][1]);
+      }
+    }
+  }
+#pragma unroll
+  for (int u = 0; u < 4; ++u)
+#pragma unroll
+    for (int v = 0; v < 2; ++v) {
+      const int i = i0 + ti * 4 + u, j = tj * 2 + v;
+      if (i < m1 && j < n2) atomicAdd(&C[i + (int64_t)j * ldc], alpha * acc[u][v]);
+    }
+}
+
 cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, int64_t lda, const float* B,
                     int64_t ldb, float* C, int64_t ldc, cudaStream_t st) {
   if (rows <= 0 || m1 <= 0 || n2 <= 0) return cudaSuccess;
+  if (n2 <= 32) {
+    const int gx = (m1 + 63) / 64;
+    int64_t want = std::max<int64_t>(1, (2 * 148 + gx - 1) / gx);
+    int64_t chunk = std::max<int64_t>((rows + want - 1) / want, 128);
+    chunk = (chunk + 63) / 64 * 64;
+    const int gz = (int)((rows + chunk - 1) / chunk);
+    skinny_tn32_kernel<<<dim3(gx, 1, gz), 256, 0, st>>>(rows, chunk, m1, n2, alpha, A, lda, B, ldb, C, ldc);
+    return cudaGetLastError();
+  }
   const int gx = (m1 + TN_T - 1) / TN_T, gy = (n2 + TN_T - 1) / TN_T;
   int64_t want = std::max<int64_t>(1, 296 / (gx * gy));
   int64_t chunk = (rows + want - 1) / want;

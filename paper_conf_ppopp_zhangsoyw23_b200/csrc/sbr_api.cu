@@ -77,6 +77,9 @@ struct sbr_ctx {
   // host-buffer (e2e) device copies
   void* e2e = nullptr;
   size_t e2e_bytes = 0;
+  // sbr_form_q split operands (grown on demand, kept for the next call)
+  void* fq = nullptr;
+  size_t fq_bytes = 0;
   // stats
   bool timing = false;
   std::vector<cudaEvent_t> ev_pool;
@@ -740,21 +743,26 @@ int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t
   const int64_t M0 = n - b;
   const int64_t loM = (M0 + 31) / 32 * 32, ldM = 2 * loM;
   const int64_t lok = (nb + 31) / 32 * 32, ldk = 2 * lok;
-  float *QS = nullptr, *YS = nullptr, *WS = nullptr, *TS = nullptr;
-  auto release = [&]() {
-    if (QS) cudaFreeAsync(QS, st);
-    if (YS) cudaFreeAsync(YS, st);
-    if (WS) cudaFreeAsync(WS, st);
-    if (TS) cudaFreeAsync(TS, st);
-  };
-  if (cudaMallocAsync((void**)&QS, sizeof(float) * M0 * ldM, st) != cudaSuccess ||
-      cudaMallocAsync((void**)&YS, sizeof(float) * nb * ldM, st) != cudaSuccess ||
-      cudaMallocAsync((void**)&WS, sizeof(float) * M0 * ldk, st) != cudaSuccess ||
-      cudaMallocAsync((void**)&TS, sizeof(float) * M0 * ldk, st) != cudaSuccess) {
-    cudaGetLastError();
-    release();
-    return SBR_ERR_NOMEM;
+  // split operands in handle-owned memory (a per-call cudaMallocAsync of these GB-sized buffers
+  // costs more than the products when the pool returns the pages in between)
+  const size_t nQS = align_up(sizeof(float) * M0 * ldM), nYS = align_up(sizeof(float) * nb * ldM),
+               nWS = align_up(sizeof(float) * M0 * ldk);
+  const size_t need = nQS + nYS + 2 * nWS;
+  if (h->fq_bytes < need) {
+    SBR_CK(cudaStreamSynchronize(st), "sync");   // a previous call may still use the old buffer
+    if (h->fq) cudaFree(h->fq);
+    h->fq = nullptr;
+    h->fq_bytes = 0;
+    if (cudaMalloc(&h->fq, need) != cudaSuccess) {
+      cudaGetLastError();
+      return SBR_ERR_NOMEM;
+    }
+    h->fq_bytes = need;
   }
+  float* QS = (float*)h->fq;
+  float* YS = (float*)((char*)h->fq + nQS);
+  float* WS = (float*)((char*)h->fq + nQS + nYS);
+  float* TS = (float*)((char*)h->fq + nQS + nYS + nWS);
   const int64_t nblk = (ncols + nb - 1) / nb;
   cudaError_t e = cudaSuccess;
   for (int64_t J = nblk - 1; J >= 0 && e == cudaSuccess; --J) {
@@ -798,7 +806,6 @@ int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t
     if ((e = launch_gemm_sub_tf32(g2, st)) != cudaSuccess) break;
     h->launches += 5;
   }
-  release();
   SBR_CK(e, "form_q");
   return SBR_OK;
 }
@@ -818,6 +825,7 @@ int sbr_destroy(sbr_handle_t h) {
   for (auto e : h->ev_pool) cudaEventDestroy(e);
   if (h->ws) cudaFree(h->ws);
   if (h->e2e) cudaFree(h->e2e);
+  if (h->fq) cudaFree(h->fq);
   delete h;
   return SBR_OK;
 }
