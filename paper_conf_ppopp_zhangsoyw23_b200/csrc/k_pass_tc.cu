@@ -101,7 +101,7 @@ struct PassWalk {
 template <int BN, int C, int NS>
 __global__ void __launch_bounds__(256, 1)
     pass_tc_kernel(const __grid_constant__ CUtensorMap mapL, const __grid_constant__ CUtensorMap mapW, int r0, int M,
-                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx) {
+                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx, int exper) {
   using Cfg = PassCfg<BN, C, NS>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -213,6 +213,7 @@ __global__ void __launch_bounds__(256, 1)
         mbar_wait(&l_full[st], ph);
         tc_fence_after();
         const uint32_t lt = aL + st * Cfg::LT;
+        if (!(exper & 1))   // (exper: timing experiments only, SBR_PASS_EXPER; 0 in production)
 #pragma unroll
         for (int s = 0; s < 8; ++s) {  // X_I += L W_J : A MN-major (LBO = 16 KB between 64-row atoms)
           const uint64_t a = sdesc_sw128(lt + (s >> 2) * 8192 + (s & 3) * 2048, 16384, 1024);
@@ -221,6 +222,7 @@ __global__ void __launch_bounds__(256, 1)
         }
         const uint32_t d_col = t_col + jj * BN;
         const uint32_t acc0 = (cinit >> jj) & 1u;
+        if (!(exper & 2))
 #pragma unroll
         for (int s = 0; s < 8; ++s) {  // X_J += L^T W_I : A K-major (same bytes)
           const uint64_t a = sdesc_sw128(lt + (s >> 2) * 16384 + (s & 3) * 32, 16, 1024);
@@ -356,8 +358,9 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   const int64_t T = T1 - T0;
   if (T <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
+  static const int exper = getenv("SBR_PASS_EXPER") ? atoi(getenv("SBR_PASS_EXPER")) : 0;
   return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mapL, mapW, (int)p.r0, (int)p.M, NT, T0, T, p.b,
-                    p.X, p.ldx);
+                    p.X, p.ldx, exper);
 }
 
 static int pass_variant() {   // SBR_PASS_CFG (tuning experiments only): 0 = C8/NS4, 1 = C4/NS5, 2 = C2/NS6

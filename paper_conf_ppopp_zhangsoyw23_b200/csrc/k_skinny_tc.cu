@@ -35,7 +35,9 @@ __global__ void __launch_bounds__(256, 1)
                      const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kc0,
                      int kct, int arow0, int brow0, int64_t rows, int b,
                      const float* Cin, int64_t ldc, float* Dout, int64_t ldd, __half* __restrict__ Hcm, int64_t ldhc,
-                     __half* __restrict__ Hrm, int64_t ldhr) {
+                     __half* __restrict__ Hrm, int64_t ldhr, int kper) {
+  // split-K (gridDim.y > 1, only when D = C in place and no fp16 copies): CTA (tile, s) takes
+  // k-chunks [s*kper, s*kper + kper) and subtracts its partial with fp32 reductions
   using Cfg = NnCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -58,9 +60,11 @@ __global__ void __launch_bounds__(256, 1)
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   pdl_wait();
+  const int kb = blockIdx.y * kper, ke = min(kct, kb + kper);
+  const bool split = gridDim.y > 1;
   if (warp == 0 && lane == 0) {
     int st = 0; uint32_t ph = 0;
-    for (int kc = 0; kc < kct; ++kc) {
+    for (int kc = kb; kc < ke; ++kc) {
       mbar_wait(&empty[st], ph ^ 1);
       mbar_expect_tx(&full[st], Cfg::STAGE);
       uint8_t* sa = smem + st * Cfg::STAGE;
@@ -74,14 +78,14 @@ __global__ void __launch_bounds__(256, 1)
     constexpr uint32_t idesc = idesc_make(128, BN, 0, 0, 0);
     int st = 0; uint32_t ph = 0;
     const uint32_t s0 = smem_u32(smem);
-    for (int kc = 0; kc < kct; ++kc) {
+    for (int kc = kb; kc < ke; ++kc) {
       mbar_wait(&full[st], ph);
       tc_fence_after();
       const uint32_t sa = s0 + st * Cfg::STAGE, sb = sa + Cfg::SA;
 #pragma unroll
       for (int s = 0; s < 4; ++s)
         mma_f16(tmem, sdesc_sw128(sa + s * 32, 16, 1024), sdesc_sw128(sb + s * 32, 16, 1024), idesc,
-                (kc > 0 || s > 0) ? 1u : 0u);
+                (kc > kb || s > 0) ? 1u : 0u);
       mma_commit(&empty[st]);
       if (++st == Cfg::NS) { st = 0; ph ^= 1; }
     }
@@ -94,10 +98,18 @@ __global__ void __launch_bounds__(256, 1)
 #pragma unroll
     for (int c0 = 0; c0 < BN; c0 += 32) {
       float v[32];
-      if (kct > 0) tmem_ld32(tmem + c0 + ((uint32_t)(q * 32) << 16), v);
+      if (ke > kb) tmem_ld32(tmem + c0 + ((uint32_t)(q * 32) << 16), v);
       else {
 #pragma unroll
         for (int c = 0; c < 32; ++c) v[c] = 0.f;
+      }
+      if (split) {
+        if (r < rows && ke > kb) {
+#pragma unroll
+          for (int c = 0; c < 32; ++c)
+            if (c0 + c < b) atomicAdd(Dout + r + (int64_t)(c0 + c) * ldd, -v[c]);
+        }
+        continue;
       }
       if (r < rows) {
         float o[32];
@@ -147,8 +159,15 @@ static cudaError_t launch_nn_t(const SkinnyNN& p, cudaStream_t st) {
   const int kct = kc0 + (int)((p.K1 + 63) / 64);
   const int grid = (int)((p.rows + 127) / 128);
   if (grid == 0) return cudaSuccess;
-  return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mA0, mA1, mB0, mB1, kc0, kct, (int)p.arow0,
-                    (int)p.brow0, p.rows, p.b, p.C, p.ldc, p.D, p.ldd, p.Hcm, p.ldhc, p.Hrm, p.ldhr);
+  // split-K when the update is in place without fp16 copies (the lazy update): >= 2 CTAs per SM
+  // stream shorter K ranges (2 fit per SM: 80 KB smem, 32-64 TMEM columns)
+  int ns = 1;
+  if (!p.Hcm && !p.Hrm && p.C == p.D && p.ldc == p.ldd && kct >= 4) ns = std::min(kct / 2, (2 * 148 + grid - 1) / grid);
+  const int kper = (kct + ns - 1) / ns;
+  ns = kct > 0 ? (kct + kper - 1) / kper : 1;
+  return launch_pdl(kern, dim3(grid, ns), dim3(256), Cfg::SMEM, st, mA0, mA1, mB0, mB1, kc0, kct, (int)p.arow0,
+                    (int)p.brow0, p.rows, p.b, p.C, p.ldc, p.D, p.ldd, p.Hcm, p.ldhc, p.Hrm, p.ldhr,
+                    std::max(kper, 1));
 }
 
 cudaError_t launch_skinny_nn(const SkinnyNN& p, cudaStream_t st) {
