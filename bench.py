@@ -236,9 +236,9 @@ def main():
     import workloads
 
     n, b, nb, mode = args.n, args.b, args.nb, args.mode
-    cfg_name = {(32768, 32, 1024, "fp16"): "config4", (16384, 32, 1024, "3xtf32"): "config3"}.get(
-        (n, b, nb, mode), "custom")
-    seed = workloads.config_seed(3 if cfg_name == "config3" else 4)
+    cfg_name = {(32768, 32, 1024, "fp16"): "config4", (16384, 32, 1024, "3xtf32"): "config3",
+                (65536, 64, 2048, "3xtf32"): "config5-params"}.get((n, b, nb, mode), "custom")
+    seed = workloads.config_seed({"config3": 3, "config5-params": 5}.get(cfg_name, 4))
     stream = torch.cuda.current_stream()
     if world > 1:
         # one matrix across the ranks (sbr_reduce_dist, strong scaling): NCCL communicator

@@ -97,8 +97,11 @@ int sbr_workspace_query(sbr_handle_t h, int64_t n, int b, int nb, int mode, size
  *           If NULL, W lives in handle workspace (per block) and is dropped. (arg 10)
  *   ldw   : >= n if W != NULL.                                (arg 11)
  * Trivial case n <= b+1: AB = band of A, W untouched, no reflectors.
- * Returns 0, -i, SBR_ERR_NONFINITE, SBR_ERR_CUDA, SBR_ERR_NOMEM.  Synchronises
- * the stream once at the start (4-byte read of the input's finiteness flag). */
+ * Returns 0, -i, SBR_ERR_NONFINITE, SBR_ERR_CUDA, SBR_ERR_NOMEM, or SBR_ERR_UNSUPPORTED when
+ * a panel taller than the TSQR fallback's capacity (148 x 256 rows at b <= 32, n >~ 37900)
+ * is numerically rank deficient for CholeskyQR (the results are then invalid).  Synchronises
+ * the stream once at the start (4-byte read of the input's finiteness flag), and once more at
+ * the end only when such tall panels occurred (4-byte read of the fallback flag). */
 int sbr_reduce(sbr_handle_t h, int mode, int64_t n, int b, int nb,
                float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw);
 

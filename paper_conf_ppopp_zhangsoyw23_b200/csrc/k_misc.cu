@@ -58,6 +58,18 @@ cudaError_t check_finite(int64_t n, const float* A, int64_t lda, unsigned* flag,
   return cudaGetLastError();
 }
 
+// Sticky record of a CholeskyQR panel that declined (rank deficient / not orthonormal) when the
+// TSQR fallback cannot run (more leaves than co-resident CTAs): *sticky |= *fail.
+__global__ void note_unhandled_kernel(const int* fail, unsigned* sticky) {
+  pdl_trigger();
+  pdl_wait();
+  if (threadIdx.x == 0 && *fail) atomicOr(sticky, 1u);
+}
+
+cudaError_t note_unhandled(const int* fail, unsigned* sticky, cudaStream_t st) {
+  return launch_pdl(note_unhandled_kernel, dim3(1), dim3(32), 0, st, fail, sticky);
+}
+
 __global__ void extract_band_kernel(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
   const int d = threadIdx.x;

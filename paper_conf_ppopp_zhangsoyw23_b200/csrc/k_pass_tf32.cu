@@ -20,9 +20,10 @@
 // Diagonal tiles: the master's upper triangle is stale, so the converter zeroes it and halves
 // the diagonal first (then L W + L^T W = OA_JJ W as with the fp16 shadow).
 //
-// One CTA per SM, 384 threads: warp 0 TMA producer, warp 1 MMA issuer, warp 2 TMEM allocator
-// (all 512 columns: A copy hi/lo 256, row and column accumulators 2 x 64 each), warps 4-7
-// converter, warps 8-11 epilogue (fp32 reductions into X).  2 stages of {L tile 64 KB, W_I
+// One CTA per SM, 512 threads: warp 0 TMA producer, warp 1 MMA issuer, warp 2 TMEM allocator
+// (all 512 columns: A copy hi/lo 256, row and column accumulators 2 x 64 each), warps 4-7 and
+// 12-15 converter (two groups, half of the columns each), warps 8-11 epilogue (fp32 reductions
+// into X).  2 stages of {L tile 64 KB, W_I
 // 32 KB} + W_J 32 KB = 224 KB smem.  Work: tile columns J in order, rows I = J .. NT-1 (group
 // = one tile column, W_J resident), a balanced contiguous range of tiles per CTA.
 #include "kernels.h"
@@ -43,7 +44,7 @@ constexpr int P3_NBAR = 5 * P3_NS + 2 + 4 + 4 + 2 + 1;
 // TMEM columns: row-major A copy (hi, lo) for X_I, row / column accumulators (2 x 64 each)
 constexpr uint32_t P3_AHI = 0, P3_ALO = 128, P3_RACC = 256, P3_CACC = 384;
 constexpr int P3_SMEM = P3_OFF_BAR + P3_NBAR * 8 + 16 + 1024;
-constexpr int P3_THREADS = 384;
+constexpr int P3_THREADS = 512;   // + converter warps 12-15 (two converter groups of 4 warps)
 static_assert(P3_SMEM <= 232448, "3xTF32 pass smem");
 
 struct Walk1 {   // C = 1 tile walk: column J, rows I = J .. NT-1
@@ -98,10 +99,10 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
   if (threadIdx.x == 0) {
     for (int i = 0; i < P3_NS; ++i) {
       mbar_init(&l_full[i], 1); mbar_init(&l_empty[i], 1); mbar_init(&hi_done[i], 1);
-      mbar_init(&lo_ready[i], 128); mbar_init(&diag_ready[i], 128);
+      mbar_init(&lo_ready[i], 256); mbar_init(&diag_ready[i], 256);
     }
     mbar_init(wj_full, 1); mbar_init(wj_empty, 1);
-    mbar_init(ta_full, 128); mbar_init(ta_empty, 1);
+    mbar_init(ta_full, 256); mbar_init(ta_empty, 1);
     for (int i = 0; i < 2; ++i) {
       mbar_init(&racc_full[i], 1); mbar_init(&racc_empty[i], 128);
       mbar_init(&cacc_full[i], 1); mbar_init(&cacc_empty[i], 128);
@@ -206,9 +207,12 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
         if (++rb == 2) { rb = 0; rph ^= 1; }
       }
     }
-  } else if (warp >= 4 && warp < 8) {
-    // ------------------------------------------------ converter
-    const int tid = threadIdx.x - 128;
+  } else if ((warp >= 4 && warp < 8) || warp >= 12) {
+    // ------------------------------------------------ converter: group cg (warps 4-7 / 12-15) takes
+    // half of the columns of the TMEM copy and half of the in-place lo pass
+    const int cgp = warp >= 12 ? 1 : 0;
+    const int tid = threadIdx.x - (cgp ? 384 : 128);   // 0..127 within the group
+    const int u = cgp * 128 + tid;                      // 0..255 over both groups
     const int q = warp & 3;                 // TMEM lane quarter = row box of the tile
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     int st = 0; uint32_t ph = 0;
@@ -217,15 +221,15 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
       uint8_t* lt = smem + st * P3_STAGE;
       mbar_wait(&l_full[st], ph);
       if (w.I == w.J) {   // stale upper triangle -> 0, diagonal halved
-        const int c = tid;
-        for (int r = 0; r <= c; ++r) {
+        const int c = u >> 1;                 // column; rows of parity u & 1
+        for (int r = u & 1; r <= c; r += 2) {
           const int rc = r >> 5, rr = r & 31;
           float* p = (float*)(lt + rc * 16384 + c * 128 + ((((rr >> 2) ^ (c & 7))) << 4) + (rr & 3) * 4);
           *p = (r == c) ? 0.5f * *p : 0.f;
         }
         fence_proxy_async_smem();
         __syncwarp();
-        asm volatile("bar.sync 1, 128;" ::: "memory");   // all columns fixed before any row is read
+        asm volatile("bar.sync 1, 256;" ::: "memory");   // all columns fixed before any row is read
         mbar_arrive(&diag_ready[st]);
       }
       // row-major split copy for X_I: thread = tile row 32q + lane, hi = rna_tf32(a), lo = rna_tf32(a - hi)
@@ -234,7 +238,7 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
       tc_fence_after();
       const uint8_t* rowbase = lt + q * 16384 + (lane & 3) * 4;
 #pragma unroll 1
-      for (int cc = 0; cc < 4; ++cc) {
+      for (int cc = 2 * cgp; cc < 2 * cgp + 2; ++cc) {
         float hi[32], lo[32];
 #pragma unroll
         for (int j = 0; j < 32; ++j) {
@@ -253,7 +257,7 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
       mbar_wait(&hi_done[st], ph);
       float4* v = (float4*)lt;
 #pragma unroll 8
-      for (int i = tid; i < P3_LT / 16; i += 128) {
+      for (int i = u; i < P3_LT / 16; i += 256) {
         float4 x = v[i];
         x.x -= __uint_as_float(__float_as_uint(x.x) & 0xffffe000u);
         x.y -= __uint_as_float(__float_as_uint(x.y) & 0xffffe000u);
@@ -265,7 +269,7 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
       mbar_arrive(&lo_ready[st]);
       if (++st == P3_NS) { st = 0; ph ^= 1; }
     }
-  } else if (warp >= 8) {
+  } else if (warp >= 8 && warp < 12) {
     // ------------------------------------------------ epilogue: TMEM -> fp32 reductions into X
     const int q = warp & 3;
     const int row_in_tile = q * 32 + lane;

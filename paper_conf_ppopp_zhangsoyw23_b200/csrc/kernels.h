@@ -78,6 +78,7 @@ cudaError_t tn_small(int64_t rows, int b, const float* A, int64_t lda, const flo
 // ---- misc ----
 cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaStream_t st);
 cudaError_t check_finite(int64_t n, const float* A, int64_t lda, unsigned* flag, cudaStream_t st);
+cudaError_t note_unhandled(const int* fail, unsigned* sticky, cudaStream_t st);
 cudaError_t extract_band(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab,
                          cudaStream_t st);
 cudaError_t mirror_lower_block(int b, float* A, int64_t lda, cudaStream_t st);

@@ -307,6 +307,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   SBR_CK(cudaMemcpyAsync(&flag, h->flag, sizeof(unsigned), cudaMemcpyDeviceToHost, st), "flag D2H");
   SBR_CK(cudaStreamSynchronize(st), "sync");
   if (flag) return SBR_ERR_NONFINITE;
+  SBR_CK(cudaMemsetAsync(h->flag + 1, 0, sizeof(unsigned), st), "zero sticky");
+  bool unguarded = false;   // some panel ran CholeskyQR without a TSQR fallback
 
   const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
   const int64_t ldn = n;        // ld of the block buffers
@@ -436,16 +438,33 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         // mode's operands -- FP16 mode rounds every GEMM operand to fp16 (u = 4.9e-4), 3xTF32 keeps
         // fp32 (u = 6e-8)
         pa.orth_tol = tc16 ? 1e-6 : 1e-8;
+        bool chol = false;
         if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
           const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
           if (ce == cudaSuccess) {
             pa.run_if = h->pfail;
             h->launches += 1;
+            chol = true;
           } else if (ce != cudaErrorNotSupported) {
             SBR_CK(ce, "panel_chol");
           }
         }
-        SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
+        const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
+        if (te == cudaErrorInvalidValue && chol) {
+          // panel taller than the TSQR tree can hold (one co-resident CTA per 256-row leaf): no
+          // fallback; a declined CholeskyQR is recorded and reported after the reduction
+          cudaGetLastError();
+          SBR_CK(note_unhandled(h->pfail, h->flag + 1, st), "note_unhandled");
+          unguarded = true;
+        } else if (te == cudaErrorInvalidValue) {
+          cudaGetLastError();
+          std::lock_guard<std::mutex> lk(g_err_mu);
+          g_last_err = "panel of " + std::to_string(m) + " x " + std::to_string(b) +
+                       " exceeds the panel kernels' capacity (CholeskyQR: 148 CTAs x rows in smem)";
+          return SBR_ERR_UNSUPPORTED;
+        } else {
+          SBR_CK(te, "panel");
+        }
         h->launches += 1;
       }
       if (tc16) {
@@ -691,6 +710,16 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     Scope sc(h, SBR_K_OTHER, 8.0 * (b + 1) * n, 0);
     SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
     h->launches += 1;
+  }
+  if (unguarded) {   // one 4-byte read at the end, only for panels beyond the TSQR capacity
+    unsigned sticky = 0;
+    SBR_CK(cudaMemcpyAsync(&sticky, h->flag + 1, sizeof(unsigned), cudaMemcpyDeviceToHost, st), "sticky D2H");
+    SBR_CK(cudaStreamSynchronize(st), "sync");
+    if (sticky) {
+      std::lock_guard<std::mutex> lk(g_err_mu);
+      g_last_err = "a panel taller than the TSQR capacity was rank deficient for CholeskyQR";
+      return SBR_ERR_UNSUPPORTED;
+    }
   }
   return SBR_OK;
 }
