@@ -72,7 +72,8 @@ struct CholSmem {
   static constexpr size_t OFF_S = OFF_RROW + sizeof(double) * B;                 // float B signs
   static constexpr size_t OFF_DI = OFF_S + sizeof(float) * B;                    // float B 1/U[k][k]
   static constexpr size_t OFF_LR = OFF_DI + sizeof(float) * B;
-  static constexpr size_t BYTES = OFF_LR + sizeof(float) * B + 64;
+  static constexpr size_t OFF_RDA = (OFF_LR + sizeof(float) * B + 15) / 16 * 16;   // double B: 1 / Racc_jj
+  static constexpr size_t BYTES = OFF_RDA + sizeof(double) * B + 64;
 };
 
 SBR_DEV unsigned ld_acquire_u32(const unsigned* p) {
@@ -244,7 +245,7 @@ SBR_DEV void cta_lu(const double* Q1, float* Lcol, float* Urow, float* Ss, float
   __syncthreads();
 }
 
-template <int B>
+template <int B, bool STREAM>
 __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, unsigned char* ws, unsigned launch) {
   pdl_trigger();   // the successor may launch early; it waits (griddepcontrol.wait) before reading
   using L = CholSmem<B>;
@@ -264,6 +265,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   float* Ur = reinterpret_cast<float*>(smem_raw + L::OFF_UR);
   float* Ss = reinterpret_cast<float*>(smem_raw + L::OFF_S);
   float* Di = reinterpret_cast<float*>(smem_raw + L::OFF_DI);
+  double* rda = reinterpret_cast<double*>(smem_raw + L::OFF_RDA);
 
   const unsigned par = launch & 1u;
   double* sets = reinterpret_cast<double*>(ws + PCW_SETS) + (size_t)par * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
@@ -281,6 +283,13 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   const int G = gridDim.x;
   const int64_t r_beg = (int64_t)blockIdx.x * m / G, r_end = (int64_t)(blockIdx.x + 1) * m / G;
   const int rows = (int)(r_end - r_beg);
+  // Panels taller than the shared-memory row capacity (148 CTAs x CH rows) are STREAMED: the CTA's
+  // rows are processed in chunks of CH, and every round recomputes Q = P Racc^-1 (fp64) from the
+  // fp32 panel instead of keeping Q resident.  Grid-uniform (row counts differ by at most one).
+  constexpr int CH = pc_maxr<B>();
+  constexpr bool stream = STREAM;   // the host picks it when (m + G - 1) / G > CH
+  const int nch = STREAM ? (rows + CH - 1) / CH : 1;
+  auto crows = [&](int ch) { return STREAM ? min(CH, rows - ch * CH) : rows; };
   auto stamp = [&](int k) {
     if (a.trace && blockIdx.x == 0 && threadIdx.x == 0) {
       int64_t t;
@@ -290,18 +299,19 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   };
   stamp(0);
   pdl_wait();   // launched with PDL: the predecessor (lazy update) must be complete before any read
-  // ---- load the CTA's rows (column-major fp32 -> row-major fp64): all loads issued first
-  {
+  // ---- load rows [c0, c0 + n) of the CTA's range (column-major fp32 -> row-major fp64): all
+  //      loads issued first
+  auto load_rows = [&](int c0, int n) {
     constexpr int CPW = (B + 7) / 8, RPL = pc_maxr<B>() / 32;
     float v[CPW][RPL];
 #pragma unroll
     for (int ci = 0; ci < CPW; ++ci) {
       const int c = warp + 8 * ci;
-      const float* src = a.P + r_beg + (int64_t)c * a.ldp;
+      const float* src = a.P + r_beg + c0 + (int64_t)c * a.ldp;
 #pragma unroll
       for (int k = 0; k < RPL; ++k) {
         const int r = lane + 32 * k;
-        v[ci][k] = (c < B && r < rows) ? __ldg(src + r) : 0.f;
+        v[ci][k] = (c < B && r < n) ? __ldg(src + r) : 0.f;
       }
     }
 #pragma unroll
@@ -310,10 +320,11 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
 #pragma unroll
       for (int k = 0; k < RPL; ++k) {
         const int r = lane + 32 * k;
-        if (c < B && r < rows) Qd[r * LDQ + c] = (double)v[ci][k];
+        if (c < B && r < n) Qd[r * LDQ + c] = (double)v[ci][k];
       }
     }
-  }
+  };
+  load_rows(0, crows(0));
   // ---- zero the other parity's Gram sets and barrier counter (used by the next launch)
   {
     double* other = reinterpret_cast<double*>(ws + PCW_SETS) + (size_t)(par ^ 1u) * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
@@ -334,15 +345,17 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     ++ti;
   }
   tj += ti;
-  auto gram_arrive = [&](int set) {   // partial Gram of Qd -> atomics into set -> barrier arrive
-    double acc[4][4];
+  double acc[4][4];
+  auto gram_zero = [&]() {
 #pragma unroll
     for (int u = 0; u < 4; ++u)
 #pragma unroll
       for (int v = 0; v < 4; ++v) acc[u][v] = 0.0;
+  };
+  auto gram_acc = [&](int n) {   // this thread's 4x4 Gram tile over Qd rows [0, n) of its row group
     if (grp < NGRP) {
 #pragma unroll 2
-      for (int r = grp; r < rows; r += NGRP) {
+      for (int r = grp; r < n; r += NGRP) {
         const double2 a0 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * ti);
         const double2 a1 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * ti + 2);
         const double2 b0 = *reinterpret_cast<const double2*>(Qd + r * LDQ + 4 * tj);
@@ -354,6 +367,10 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
 #pragma unroll
           for (int v = 0; v < 4; ++v) acc[u][v] = fma(aa[u], bb[v], acc[u][v]);
       }
+    }
+  };
+  auto gram_arrive = [&](int set) {   // partial Gram tiles -> smem reduction -> set -> barrier arrive
+    if (grp < NGRP) {
 #pragma unroll
       for (int u = 0; u < 4; ++u)
 #pragma unroll
@@ -411,12 +428,13 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       return cta_chol<B, LDG>(Gk, Rrm, rd, floor_rel);
     }
   };
-  auto solve = [&]() {   // Q <- Q R^-1: forward substitution, 2 rows per thread (R row-major in Rrm)
-    const int half = (rows + 1) >> 1;
+  // Q <- Q R^-1 on Qd rows [0, n): forward substitution, 2 rows per thread (R row-major, rdg = 1/R_jj)
+  auto solve = [&](const double* Rm, const double* rdg, int n) {
+    const int half = (n + 1) >> 1;
     for (int r = threadIdx.x; r < half; r += blockDim.x) {
       const int r2 = r + half;
-      const bool two = r2 < rows;
-      const double2* R2 = reinterpret_cast<const double2*>(Rrm);
+      const bool two = r2 < n;
+      const double2* R2 = reinterpret_cast<const double2*>(Rm);
       asm volatile("" : "+l"(R2));   // opaque: no hoisting of the b^2 loads out of the row loop
       double q[B], p[B];
 #pragma unroll
@@ -430,8 +448,8 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       }
 #pragma unroll
       for (int c = 0; c < B; ++c) {
-        q[c] *= rd[c];
-        p[c] *= rd[c];
+        q[c] *= rdg[c];
+        p[c] *= rdg[c];
 #pragma unroll
         for (int h = (c + 1) / 2; h < B / 2; ++h) {
           const double2 rr = R2[c * (B / 2) + h];
@@ -451,9 +469,10 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     }
     __syncthreads();
   };
-  auto racc_update = [&](bool first) {   // CTA 0: Racc <- R_k Racc (upper triangular product)
+  auto racc_update = [&](bool first) {   // Racc <- R_k Racc (upper triangular product); streaming: rda
     if (first) {
       for (int e = threadIdx.x; e < B * B; e += blockDim.x) Racc[e] = Rrm[e];
+      if (threadIdx.x < B) rda[threadIdx.x] = rd[threadIdx.x];
       __syncthreads();
       return;
     }
@@ -476,6 +495,15 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       if (e < B * B) Racc[e] = t4[k];
     }
     __syncthreads();
+    if (threadIdx.x < B) rda[threadIdx.x] = 1.0 / Racc[threadIdx.x * B + threadIdx.x];
+    __syncthreads();
+  };
+  // streaming: Q rows of chunk ch = P rows Racc^-1, into Qd
+  auto stream_q = [&](int ch) {
+    __syncthreads();   // previous users of Qd are done
+    load_rows(ch * CH, crows(ch));
+    __syncthreads();
+    solve(Racc, rda, crows(ch));
   };
   auto lu_publish = [&](unsigned gen) {   // CTA 0: LU of Q_1 - S, to smem and to global
     if constexpr (B <= 32) {
@@ -500,6 +528,14 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   };
 
   // ---- round 0: G = P^T P, R_0 = chol(G), Q = P R_0^-1
+  gram_zero();
+  gram_acc(crows(0));
+  for (int ch = 1; ch < nch; ++ch) {   // streaming only
+    __syncthreads();
+    load_rows(ch * CH, crows(ch));
+    __syncthreads();
+    gram_acc(crows(ch));
+  }
   gram_arrive(0);
   stamp(2);
   bar_wait(ctr, (unsigned)G);
@@ -510,17 +546,29 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     return;
   }
   stamp(4);
-  solve();
-  if (blockIdx.x == 0) racc_update(true);
+  if (!stream) solve(Rrm, rd, rows);
+  if (blockIdx.x == 0 || stream) racc_update(true);
   stamp(5);
   // ---- rounds k = 1..3: check G = Q^T Q ~ I, else one more CholeskyQR step
   unsigned gen = 0;
   bool done = false;
   for (int k = 1; k < PC_NSET; ++k) {
+    gram_zero();
+    if (!stream) {
+      gram_acc(rows);
+    } else {
+      for (int ch = 0; ch < nch; ++ch) {
+        stream_q(ch);
+        gram_acc(crows(ch));
+      }
+    }
     gram_arrive(k);
     gen = launch * 4u + (unsigned)k;
     if (k == 1) stamp(6);
-    if (blockIdx.x == 0) lu_publish(gen);   // speculative: valid if this round's check passes
+    if (blockIdx.x == 0) {   // speculative: valid if this round's check passes
+      if (stream) stream_q(0);   // the top b rows of Q
+      lu_publish(gen);
+    }
     if (k == 1) stamp(7);
     bar_wait(ctr, (unsigned)G * (k + 1));
     if (k == 1) stamp(8);
@@ -535,8 +583,8 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       break;
     }
     if (k == PC_NSET - 1 || !chol(0.0)) break;
-    solve();
-    if (blockIdx.x == 0) racc_update(false);
+    if (!stream) solve(Rrm, rd, rows);
+    if (blockIdx.x == 0 || stream) racc_update(false);
   }
   if (!done) {
     if (blockIdx.x == 0 && threadIdx.x == 0) *fail = 1;
@@ -565,8 +613,11 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   stamp(10);
   // ---- rows: w L_1^T = e_il - q S ;  y = L_1 row (il < B) or y U = q ;  compact panel
   const int64_t row0 = a.row0;
-  for (int r = threadIdx.x; r < rows; r += blockDim.x) {
-    const int64_t il = r_beg + r;
+  for (int ch = 0; ch < nch; ++ch) {
+  const int c0 = ch * CH, nr = crows(ch);
+  if (stream) stream_q(ch);   // Q rows of this chunk (resident otherwise)
+  for (int r = threadIdx.x; r < nr; r += blockDim.x) {
+    const int64_t il = r_beg + c0 + r;
     const int64_t gr = row0 + il;
     // opaque per-iteration copies of the smem factors: keeps the compiler from hoisting
     // all b^2 loads out of the row loop (which spills)
@@ -645,6 +696,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       }
     }
   }
+  }   // chunks
   // rows of the block above the panel: Y = W = 0
   const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const int64_t nth = (int64_t)gridDim.x * blockDim.x;
@@ -666,23 +718,28 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
 
 template <int B>
 static cudaError_t launch_chol_t(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st) {
-  auto kern = panel_chol_kernel<B>;
   constexpr size_t smem = CholSmem<B>::BYTES;
   static int per_sm = -1, nsm = 0;
   if (per_sm < 0) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = cudaFuncSetAttribute(panel_chol_kernel<B, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)smem);
     if (e != cudaSuccess) return e;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, PC_THREADS, smem);
+    e = cudaFuncSetAttribute(panel_chol_kernel<B, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, panel_chol_kernel<B, false>, PC_THREADS, smem);
     if (per_sm < 1) per_sm = 1;
     int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   }
   const int cap = per_sm * nsm;
-  // >= 64 rows per CTA (CTA 0 must hold the b top rows); enough CTAs for the smem row cap
+  // >= 64 rows per CTA (CTA 0 must hold the b top rows); panels beyond cap x pc_maxr rows are
+  // streamed in row chunks (see the kernel)
   int G = (int)std::min<int64_t>(cap, a.m / 64);
-  if ((int64_t)G * pc_maxr<B>() < a.m) G = (int)((a.m + pc_maxr<B>() - 1) / pc_maxr<B>());
-  if (G > cap || G < 1) return cudaErrorNotSupported;   // caller uses TSQR
+  if ((int64_t)G * pc_maxr<B>() < a.m) G = (int)std::min<int64_t>(cap, (a.m + pc_maxr<B>() - 1) / pc_maxr<B>());
+  if (G < 1) return cudaErrorNotSupported;   // caller uses TSQR
+  const bool stream = (a.m + G - 1) / G > pc_maxr<B>();
+  auto kern = stream ? panel_chol_kernel<B, true> : panel_chol_kernel<B, false>;
   unsigned char* wsp = (unsigned char*)ws;
   // cooperative (grid-wide barriers) AND programmatic dependent launch: the launch and the
   // prologue overlap the tail of the lazy update; all CTAs are co-resident once it drains

@@ -1344,12 +1344,26 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
   pa.ws_q = h->pq;
   pa.ws_misc = h->pmisc;
   pa.trace = trace_host ? (int64_t*)tr.p : nullptr;
+  bool chol = false;
   if (h->panel_mode == 0 && m > 512) {
     const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
-    if (ce == cudaSuccess) pa.run_if = h->pfail;
-    else if (ce != cudaErrorNotSupported) SBR_CK(ce, "panel_chol");
+    if (ce == cudaSuccess) {
+      pa.run_if = h->pfail;
+      chol = true;
+    } else if (ce != cudaErrorNotSupported) {
+      SBR_CK(ce, "panel_chol");
+    }
   }
-  SBR_CK(launch_panel(pa, h->panel_ctas, st), "panel");
+  const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
+  if (te == cudaErrorInvalidValue && chol) {   // taller than the TSQR tree: CholeskyQR only (as sbr_reduce)
+    cudaGetLastError();
+    int failed = 0;
+    SBR_CK(cudaMemcpyAsync(&failed, h->pfail, sizeof(int), cudaMemcpyDeviceToHost, st), "fail D2H");
+    SBR_CK(cudaStreamSynchronize(st), "sync");
+    if (failed) return SBR_ERR_UNSUPPORTED;
+  } else {
+    SBR_CK(te, "panel");
+  }
   if (trace_host) {
     SBR_CK(cudaMemcpyAsync(trace_host, tr.p, sizeof(int64_t) * 16, cudaMemcpyDeviceToHost, st), "trace D2H");
     SBR_CK(cudaStreamSynchronize(st), "sync");
