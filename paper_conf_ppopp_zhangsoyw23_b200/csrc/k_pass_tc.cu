@@ -171,10 +171,8 @@ __global__ void __launch_bounds__(256, 1)
         mbar_wait(&l_empty[st], ph ^ 1);
         mbar_expect_tx(&l_full[st], Cfg::LT);
         uint8_t* dst = sL + st * Cfg::LT;
-        for (int rb = 0; rb < 2; ++rb)
-          for (int cb = 0; cb < 2; ++cb)
-            tma_load_2d(dst + (rb * 2 + cb) * 8192, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64,
-                        r0 + w.J * 128 + cb * 64);
+        for (int rb = 0; rb < 2; ++rb)   // box = 64 rows x 128 columns (same smem image as 2 boxes of 64)
+          tma_load_2d(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, r0 + w.J * 128);
         if (++st == NS) { st = 0; ph ^= 1; }
         if (w.rlast()) {
           if (++ws == 2) { ws = 0; wph ^= 1; }
@@ -348,7 +346,7 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
     attr = true;
   }
   CUtensorMap mapL, mapW;
-  cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 64);
+  cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 128);
   if (e != cudaSuccess) return e;
   e = make_tmap_2d(&mapW, p.Wh, true, p.M, BN, p.ld_wh, 64, BN);
   if (e != cudaSuccess) return e;

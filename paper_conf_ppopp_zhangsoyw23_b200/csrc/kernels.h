@@ -98,7 +98,7 @@ cudaError_t syr2k_lower(int64_t M, int K, const float* Y, int64_t ldy, const flo
 
 // ---- tcgen05 / TMA path (FP16 mode) ----
 cudaError_t make_tmap_2d(CUtensorMap* map, const void* base, bool fp16, uint64_t inner, uint64_t outer, uint64_t ld,
-                         uint32_t box_inner, uint32_t box_outer);
+                         uint32_t box_inner, uint32_t box_outer, int l2_promo = 256);
 
 struct PassLaunch {
   const __half* shadow;  // n x n fp16 shadow of the trailing matrix (strict lower, half diag, zero upper)

@@ -26,7 +26,7 @@ static EncodeTiledFn get_encode() {
 // 2-D map over a column-major-like array: `inner` contiguous elements per line, `outer`
 // lines `ld` elements apart; box = box_inner x box_outer; 128-byte swizzle; OOB -> 0.
 cudaError_t make_tmap_2d(CUtensorMap* map, const void* base, bool fp16, uint64_t inner, uint64_t outer,
-                         uint64_t ld, uint32_t box_inner, uint32_t box_outer) {
+                         uint64_t ld, uint32_t box_inner, uint32_t box_outer, int l2_promo) {
   EncodeTiledFn fn = get_encode();
   if (!fn) return cudaErrorNotSupported;
   const size_t es = fp16 ? 2 : 4;
@@ -36,7 +36,8 @@ cudaError_t make_tmap_2d(CUtensorMap* map, const void* base, bool fp16, uint64_t
   cuuint32_t estr[2] = {1, 1};
   CUresult r = fn(map, fp16 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16 : CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2,
                   const_cast<void*>(base), dims, strides, box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
-                  CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                  CU_TENSOR_MAP_SWIZZLE_128B,
+                  l2_promo == 128 ? CU_TENSOR_MAP_L2_PROMOTION_L2_128B : CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
