@@ -12,8 +12,8 @@
 // All three are fp32 SIMT: k x k x b is tiny and the operands (W^T X, b rows of X and Y) sit in
 // L2, so these kernels are latency-bound.  Design for latency:
 //   * every CTA issues all of its global loads before the first use (one round trip);
-//   * the reduction dimension is split over the 8 CTAs of a thread-block cluster and the
-//     partial results are summed through distributed shared memory -- no global atomics on
+//   * the reduction dimension is split over the 16 CTAs of a thread-block cluster (kxb; 8 for
+//     the postpass) and the partial results are summed through distributed shared memory -- no global atomics on
 //     the hot addresses, no pre-zeroed outputs, no second launch.
 #include <cooperative_groups.h>
 
@@ -25,24 +25,26 @@ namespace cg = cooperative_groups;
 namespace sbr {
 
 constexpr int KXB_QT = 32;   // output rows (q) per cluster
-constexpr int KXB_CL = 8;    // CTAs per cluster (split of the reduction dimension r)
-template <int NG>            // r-chunk staged in shared memory (48 KB static)
-constexpr int kxb_rc() { return NG == 1 ? 128 : 96; }
+constexpr int KXB_RC = 64;   // r-chunk staged in shared memory per iteration
 
-template <int NG>  // NG = 32-column groups of b (1: b <= 32, 2: b <= 64)
-__global__ void __cluster_dims__(1, KXB_CL, 1) __launch_bounds__(256) kxb_kernel(KxbArgs a) {
-  constexpr int KXB_RC = kxb_rc<NG>();
+// CL = CTAs per cluster (split of the reduction dimension r): 16 (non-portable cluster size,
+// halves each warp's dependent chain and doubles the resident warps), 8 if that launch fails.
+// NG = 32-column groups of b (1: b <= 32, 2: b <= 64).
+template <int CL, int NG>
+__global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
+  constexpr int NB = 32 * NG;
+  constexpr int LA = KXB_RC * KXB_QT / 256;   // A elements staged per thread per chunk
+  constexpr int LB = KXB_RC * NB / 256;       // B elements staged per thread per chunk
   __shared__ __align__(16) float As[KXB_RC][KXB_QT];   // As[r][q] = WtX[q0+q, r]; reused for partials
-  __shared__ float Bs[KXB_RC][32 * NG + 1];            // Bs[r][p] = B(r, p)
+  __shared__ float Bs[KXB_RC][NB + 1];                  // Bs[r][p] = B(r, p)
   cg::cluster_group cluster = cg::this_cluster();
   pdl_trigger();
-  pdl_wait();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int k = a.k, b = a.b;
   const bool lazy = a.mode == 0;
   const int q0 = blockIdx.x * KXB_QT;
   const int rank = (int)cluster.block_rank();
-  const int rper = (k + KXB_CL - 1) / KXB_CL;
+  const int rper = (k + CL - 1) / CL;
   const int rb = rank * rper, re = min(k, rb + rper);
   float* __restrict__ WtX = a.WtX;
   const int64_t ldwx = a.ldwx;
@@ -51,54 +53,76 @@ __global__ void __cluster_dims__(1, KXB_CL, 1) __launch_bounds__(256) kxb_kernel
   for (int i = 0; i < 4; ++i)
 #pragma unroll
     for (int g = 0; g < NG; ++g) acc[i][g] = 0.f;
+  pdl_wait();
   for (int r0 = rb; r0 < re; r0 += KXB_RC) {
     const int nr = min(KXB_RC, re - r0);
-    // stage: all loads issued before any use
-    for (int e = threadIdx.x; e < KXB_RC * KXB_QT; e += blockDim.x) {
+    // stage: every load of the chunk issued (into registers) before the first shared store
+    float av[LA], bv[LB];
+#pragma unroll
+    for (int u = 0; u < LA; ++u) {
+      const int e = threadIdx.x + u * 256;
       const int q = e % KXB_QT, r = e / KXB_QT;
-      As[r][q] = (r < nr && q0 + q < k) ? __ldcg(WtX + (q0 + q) + (int64_t)(r0 + r) * ldwx) : 0.f;
+      av[u] = (r < nr && q0 + q < k) ? __ldcg(WtX + (q0 + q) + (int64_t)(r0 + r) * ldwx) : 0.f;
     }
     if (lazy) {
-      for (int e = threadIdx.x; e < KXB_RC * 32 * NG; e += blockDim.x) {
-        const int p = e % (32 * NG), r = e / (32 * NG);
-        Bs[r][p] = (r < nr && p < b) ? __ldcg(a.Y + (a.c + p) + (int64_t)(r0 + r) * a.ldy) : 0.f;
+#pragma unroll
+      for (int u = 0; u < LB; ++u) {
+        const int e = threadIdx.x + u * 256;
+        const int p = e % NB, r = e / NB;
+        bv[u] = (r < nr && p < b) ? __ldcg(a.Y + (a.c + p) + (int64_t)(r0 + r) * a.ldy) : 0.f;
       }
     } else {
-      for (int e = threadIdx.x; e < KXB_RC * 32 * NG; e += blockDim.x) {
+#pragma unroll
+      for (int u = 0; u < LB; ++u) {
+        const int e = threadIdx.x + u * 256;
         const int r = e % KXB_RC, p = e / KXB_RC;
-        Bs[r][p] = (r < nr && p < b) ? __ldcg(a.G + (r0 + r) + (int64_t)p * a.ldg) : 0.f;
+        bv[u] = (r < nr && p < b) ? __ldcg(a.G + (r0 + r) + (int64_t)p * a.ldg) : 0.f;
       }
+    }
+#pragma unroll
+    for (int u = 0; u < LA; ++u) {
+      const int e = threadIdx.x + u * 256;
+      As[e / KXB_QT][e % KXB_QT] = av[u];
+    }
+#pragma unroll
+    for (int u = 0; u < LB; ++u) {
+      const int e = threadIdx.x + u * 256;
+      if (lazy) Bs[e / NB][e % NB] = bv[u];
+      else Bs[e % KXB_RC][e / KXB_RC] = bv[u];
     }
     __syncthreads();
 #pragma unroll 4
     for (int r = 0; r < nr; ++r) {
-      const float4 av = *reinterpret_cast<const float4*>(&As[r][warp * 4]);
-      const float aa[4] = {av.x, av.y, av.z, av.w};
+      const float4 a4 = *reinterpret_cast<const float4*>(&As[r][warp * 4]);
+      const float aa[4] = {a4.x, a4.y, a4.z, a4.w};
 #pragma unroll
       for (int g = 0; g < NG; ++g) {
-        const float bv = Bs[r][lane + 32 * g];
+        const float bb = Bs[r][lane + 32 * g];
 #pragma unroll
-        for (int i = 0; i < 4; ++i) acc[i][g] = fmaf(aa[i], bv, acc[i][g]);
+        for (int i = 0; i < 4; ++i) acc[i][g] = fmaf(aa[i], bb, acc[i][g]);
       }
     }
     __syncthreads();
   }
-  // partials -> shared (As reused as Ps[q][p], p < 32*NG), then the cluster reduction:
-  // CTA `rank` finalises rows q in [rank*4, rank*4 + 4) of the cluster's 32.
+  // partials -> shared (As reused as Ps[q][p], p < NB), then the cluster reduction:
+  // CTA `rank` finalises rows q in [rank*QPC, rank*QPC + QPC) of the cluster's 32.
+  constexpr int QPC = KXB_QT / CL;
   static_assert(KXB_RC * KXB_QT >= KXB_QT * 64, "partials fit in As");
   float* Ps = &As[0][0];
-  constexpr int LDP = 32 * NG;
 #pragma unroll
   for (int i = 0; i < 4; ++i)
 #pragma unroll
-    for (int g = 0; g < NG; ++g) Ps[(warp * 4 + i) * LDP + lane + 32 * g] = acc[i][g];
+    for (int g = 0; g < NG; ++g) Ps[(warp * 4 + i) * NB + lane + 32 * g] = acc[i][g];
   cluster.sync();
-  for (int e = threadIdx.x; e < 4 * b; e += blockDim.x) {
-    const int qi = rank * 4 + e / b, p = e % b;
+  for (int e = threadIdx.x; e < QPC * b; e += blockDim.x) {
+    const int qi = rank * QPC + e / b, p = e % b;
     const int q = q0 + qi;
+    float part[CL];
+#pragma unroll
+    for (int j = 0; j < CL; ++j) part[j] = cluster.map_shared_rank(Ps, j)[qi * NB + p];
     float s = 0.f;
 #pragma unroll
-    for (int j = 0; j < KXB_CL; ++j) s += cluster.map_shared_rank(Ps, j)[qi * LDP + p];
+    for (int j = 0; j < CL; ++j) s += part[j];
     if (q < k) {
       if (lazy) {
         const float d = __ldcg(a.X + (a.c + p) + (int64_t)q * a.ldx) - s;
@@ -128,19 +152,59 @@ __global__ void __cluster_dims__(1, KXB_CL, 1) __launch_bounds__(256) kxb_kernel
   cluster.sync();   // keep this CTA's partials alive until every reader is done
 }
 
+template <int CL, int NG>
+static cudaError_t launch_kxb_t(const KxbArgs& a, cudaStream_t st) {
+  auto kern = kxb_kernel<CL, NG>;
+  if (CL > 8) {
+    static bool attr = false;
+    if (!attr) {
+      const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+      if (e != cudaSuccess) return e;
+      attr = true;
+    }
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((a.k + KXB_QT - 1) / KXB_QT, CL);
+  cfg.blockDim = dim3(256);
+  cfg.dynamicSmemBytes = 0;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 1;
+  at[0].val.clusterDim.y = CL;
+  at[0].val.clusterDim.z = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, a);
+}
+
+static int kxb_cluster() {   // SBR_KXB_CL=8 forces the portable cluster size (ablation)
+  static int cl = [] {
+    const char* e = std::getenv("SBR_KXB_CL");
+    return (e && std::atoi(e) == 8) ? 8 : 16;
+  }();
+  return cl;
+}
+
 cudaError_t launch_kxb(const KxbArgs& a, cudaStream_t st) {
   if (a.k <= 0 || a.b <= 0) return cudaSuccess;
-  const dim3 grid((a.k + KXB_QT - 1) / KXB_QT, KXB_CL);
-  if (a.b <= 32)
-    return launch_pdl(kxb_kernel<1>, grid, dim3(256), 0, st, a);
-  return launch_pdl(kxb_kernel<2>, grid, dim3(256), 0, st, a);
+  static bool cl16_ok = true;
+  if (cl16_ok && kxb_cluster() == 16) {
+    const cudaError_t e = a.b <= 32 ? launch_kxb_t<16, 1>(a, st) : launch_kxb_t<16, 2>(a, st);
+    if (e == cudaSuccess) return e;
+    cudaGetLastError();   // cluster of 16 not schedulable here: portable size from now on
+    cl16_ok = false;
+  }
+  return a.b <= 32 ? launch_kxb_t<8, 1>(a, st) : launch_kxb_t<8, 2>(a, st);
 }
 
 // ------------------------------------------------------------------ postpass
 constexpr int PP_CL = 8;
 
 template <int BB>  // BB >= b, multiple of 16; rows per CTA sized for 48 KB of static smem
-constexpr int pp_rows() { return BB <= 16 ? 256 : BB <= 32 ? 128 : 64; }
+constexpr int pp_rows() { return BB <= 16 ? 128 : 64; }   // 8-16 loads per thread and array, ~3 CTAs per SM
 
 template <int BB>
 __global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
@@ -156,15 +220,21 @@ __global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
   pdl_wait();
   const int64_t rbeg = (int64_t)blockIdx.x * PP_ROWS;
   const int nr = (int)(M - rbeg < PP_ROWS ? (M - rbeg > 0 ? M - rbeg : 0) : PP_ROWS);
-  for (int e = threadIdx.x; e < PP_ROWS * BB; e += blockDim.x) {
+  constexpr int LU = PP_ROWS * BB / 256;   // elements per thread and array, all loads issued before any store
+  float xv[LU], wv[LU];
+#pragma unroll
+  for (int u = 0; u < LU; ++u) {
+    const int e = threadIdx.x + u * 256;
     const int r = e % PP_ROWS, c = e / PP_ROWS;
-    float xv = 0.f, wv = 0.f;
-    if (r < nr && c < b) {
-      xv = __ldcg(X + (rbeg + r) + (int64_t)c * ldx);
-      wv = __ldcg(W + (rbeg + r) + (int64_t)c * ldw);
-    }
-    Xs[r][c] = xv;
-    Ws[r][c] = wv;
+    const bool in = r < nr && c < b;
+    xv[u] = in ? __ldcg(X + (rbeg + r) + (int64_t)c * ldx) : 0.f;
+    wv[u] = in ? __ldcg(W + (rbeg + r) + (int64_t)c * ldw) : 0.f;
+  }
+#pragma unroll
+  for (int u = 0; u < LU; ++u) {
+    const int e = threadIdx.x + u * 256;
+    Xs[e % PP_ROWS][e / PP_ROWS] = xv[u];
+    Ws[e % PP_ROWS][e / PP_ROWS] = wv[u];
   }
   __syncthreads();
   // X_t rows -> fp16 row-major
