@@ -159,10 +159,18 @@ static cudaError_t launch_nn_t(const SkinnyNN& p, cudaStream_t st) {
   const int kct = kc0 + (int)((p.K1 + 63) / 64);
   const int grid = (int)((p.rows + 127) / 128);
   if (grid == 0) return cudaSuccess;
-  // split-K when the update is in place without fp16 copies (the lazy update): >= 2 CTAs per SM
-  // stream shorter K ranges (2 fit per SM: 80 KB smem, 32-64 TMEM columns)
+  // split-K when the update is in place without fp16 copies (the lazy update): CTAs stream shorter
+  // K ranges (2 fit per SM: 80 KB smem, 32-64 TMEM columns), the split chosen to minimise the wave-quantised time ceil(grid*ns/slots)/ns with
+  // at least 4 K-chunks per CTA
   int ns = 1;
-  if (!p.Hcm && !p.Hrm && p.C == p.D && p.ldc == p.ldd && kct >= 4) ns = std::min(kct / 2, (2 * 148 + grid - 1) / grid);
+  if (!p.Hcm && !p.Hrm && p.C == p.D && p.ldc == p.ldd && kct >= 8) {
+    const int slots = 2 * 148;
+    double best = 1e30;
+    for (int s = 1; s <= std::min(8, kct / 4); ++s) {
+      const double cost = (double)((grid * s + slots - 1) / slots) / s + 0.02 * s;   // + atomics / prologue per split
+      if (cost < best) { best = cost; ns = s; }
+    }
+  }
   const int kper = (kct + ns - 1) / ns;
   ns = kct > 0 ? (kct + kper - 1) / kper : 1;
   return launch_pdl(kern, dim3(grid, ns), dim3(256), Cfg::SMEM, st, mA0, mA1, mB0, mB1, kc0, kct, (int)p.arow0,
@@ -180,7 +188,7 @@ cudaError_t launch_skinny_nn(const SkinnyNN& p, cudaStream_t st) {
 // ------------------------------------------------------------------ skinny_tn (dual)
 template <int BN>
 struct TnCfg {
-  static constexpr int NS = 4;
+  static constexpr int NS = 3;   // 3 x 36 KB: two CTAs per SM (one wave of 2 x 148, 216 KB in flight per SM)
   static constexpr int SA = 128 * 64 * 2;   // one A operand: 128 (K1 dim) x 64 rows, 2 boxes of 64x64
   static constexpr int SB = BN * 64 * 2;
   static constexpr int STAGE = 2 * SA + SB;
@@ -300,7 +308,7 @@ static cudaError_t launch_tn_t(const SkinnyTN& p, cudaStream_t st) {
   if ((e = make_tmap_2d(&mA1, p.A1 ? p.A1 : p.A0, true, p.K1, p.a_rows, p.lda, 64, 64)) != cudaSuccess) return e;
   if ((e = make_tmap_2d(&mB, p.B, true, p.b_rows, p.b, p.ldb, 64, BN)) != cudaSuccess) return e;
   const int gx = (int)((p.K1 + 127) / 128);
-  int64_t want = std::max<int64_t>(1, (2 * p.num_sms) / gx);
+  int64_t want = std::max<int64_t>(1, (2 * p.num_sms) / gx);   // one wave at two CTAs per SM
   int64_t chunk = (p.rows + want - 1) / want;
   chunk = std::max<int64_t>(512, (chunk + 63) / 64 * 64);
   const int gy = (int)((p.rows + chunk - 1) / chunk);

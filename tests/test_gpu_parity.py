@@ -34,6 +34,7 @@ def _oracle(a, b):
     (1000, 32, 128),  # multi-leaf TSQR (first panel m = 968 > 512) + reconstruction
     (1024, 64, 128),  # b = 64 (config-5 bandwidth): 4 leaves, arity 4
     (96, 32, 32),     # nb = b (non-lazy degenerate case)
+    (1500, 16, 256),  # tile-contiguous FP16 shadow over several blocks, ragged last tile (n - b = 1484)
 ])
 def test_parity_vs_oracle(n, b, nb, mode):
     a = workloads.random_symmetric(n, workloads.config_seed(1) + n + b)
