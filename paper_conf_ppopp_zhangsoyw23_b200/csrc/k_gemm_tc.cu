@@ -77,8 +77,8 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap mapA0, const __grid_constant__ CUtensorMap mapA1,
                    const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
                    const GemmSegs segs, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles,
-                   float* C, int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, int sh_nt, int64_t sh_g0,
-                   const float* __restrict__ X, int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off) {
+                   float* C, int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, const float* __restrict__ X,
+                   int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off) {
   using Cfg = GCfg<TF>;
   constexpr int BK = TF ? 32 : 64;   // K elements per 128-byte row chunk
   constexpr int G_BN = Cfg::BN, G_NS = Cfg::NS, G_STAGE = Cfg::STAGE;
@@ -248,13 +248,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
             if (col <= row) {
               const float nv = old[c] - v[c];
               __stcs(cp + c * ldc, nv);
-              const __half hv = __float2half_rn(col == row ? 0.5f * nv : nv);
-              if (sh_nt > 0) {   // tile-contiguous shadow (k_misc.cu shadow_init_tiles)
-                const int64_t gr = sh_g0 + row, gc = sh_g0 + col;
-                shadow[(((gr >> 7) + (gc >> 7) * sh_nt) << 14) + ((gc & 127) << 7) + (gr & 127)] = hv;
-              } else {
-                shadow[row + col * ldsh] = hv;
-              }
+              shadow[row + col * ldsh] = __float2half_rn(col == row ? 0.5f * nv : nv);
             }
           }
         } else {
@@ -340,7 +334,7 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   if (ntiles == 0) return cudaSuccess;
   const int grid = std::min(ntiles, p.num_sms);
   return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
-                    (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.sh_nt, p.sh_g0, p.X, p.ldx,
+                    (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
                     TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off);
 }
 

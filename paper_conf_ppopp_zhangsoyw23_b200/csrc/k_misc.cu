@@ -154,31 +154,6 @@ cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int6
   return cudaGetLastError();
 }
 
-// Tile-contiguous shadow: grid tile (gi, gj), gi >= gj, holds A[b + gi*128 + ri, b + gj*128 + cj]
-// at Sh[(gi + gj*nt)*16384 + cj*128 + ri] (strict lower as is, HALF the diagonal, zero above and
-// beyond n -- the pass streams whole tiles, so the padding must read as zero).  One CTA per tile.
-__global__ void shadow_init_tiles_kernel(int64_t n, int b, int nt, const float* A, int64_t lda, __half* Sh) {
-  const int gj = blockIdx.x, gi = blockIdx.y;
-  if (gi < gj) return;
-  __half* tile = Sh + ((int64_t)gi + (int64_t)gj * nt) * 16384;
-  for (int e = threadIdx.x; e < 16384; e += blockDim.x) {
-    const int ri = e & 127, cj = e >> 7;
-    const int64_t i = b + (int64_t)gi * 128 + ri, j = b + (int64_t)gj * 128 + cj;
-    float v = 0.f;
-    if (i < n && j < n) {
-      if (i > j) v = A[i + j * lda];
-      else if (i == j) v = 0.5f * A[i + j * lda];
-    }
-    tile[e] = __float2half_rn(v);
-  }
-}
-
-cudaError_t shadow_init_tiles(int64_t n, int b, int nt, const float* A, int64_t lda, __half* Sh, cudaStream_t st) {
-  if (nt <= 0) return cudaSuccess;
-  shadow_init_tiles_kernel<<<dim3(nt, nt), 256, 0, st>>>(n, b, nt, A, lda, Sh);
-  return cudaGetLastError();
-}
-
 __global__ void to_half_cm_kernel(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd) {
   const int c = blockIdx.y;
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += (int64_t)gridDim.x * blockDim.x)

@@ -101,8 +101,7 @@ struct PassWalk {
 template <int BN, int C, int NS>
 __global__ void __launch_bounds__(256, 1)
     pass_tc_kernel(const __grid_constant__ CUtensorMap mapL, const __grid_constant__ CUtensorMap mapW, int r0, int M,
-                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx, int exper, int sh_nt,
-                   int sh_ofs) {
+                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx, int exper) {
   using Cfg = PassCfg<BN, C, NS>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -172,13 +171,8 @@ __global__ void __launch_bounds__(256, 1)
         mbar_wait(&l_empty[st], ph ^ 1);
         mbar_expect_tx(&l_full[st], Cfg::LT);
         uint8_t* dst = sL + st * Cfg::LT;
-        if (sh_nt > 0) {   // tile-contiguous shadow: one 32 KB run of HBM per tile
-          const int tix = (sh_ofs + w.I) + (sh_ofs + w.J) * sh_nt;
-          for (int rb = 0; rb < 2; ++rb) tma_load_3d(dst + rb * 16384, &mapL, &l_full[st], rb * 64, 0, tix);
-        } else {
-          for (int rb = 0; rb < 2; ++rb)   // box = 64 rows x 128 columns (same smem image as 2 boxes of 64)
-            tma_load_2d(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, r0 + w.J * 128);
-        }
+        for (int rb = 0; rb < 2; ++rb)   // box = 64 rows x 128 columns (same smem image as 2 boxes of 64)
+          tma_load_2d(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, r0 + w.J * 128);
         if (++st == NS) { st = 0; ph ^= 1; }
         if (w.rlast()) {
           if (++ws == 2) { ws = 0; wph ^= 1; }
@@ -352,8 +346,7 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
     attr = true;
   }
   CUtensorMap mapL, mapW;
-  cudaError_t e = p.sh_nt > 0 ? make_tmap_tiles(&mapL, p.shadow, (uint64_t)p.sh_nt * p.sh_nt)
-                              : make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 128);
+  cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 128);
   if (e != cudaSuccess) return e;
   e = make_tmap_2d(&mapW, p.Wh, true, p.M, BN, p.ld_wh, 64, BN);
   if (e != cudaSuccess) return e;
@@ -365,7 +358,7 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
   static const int exper = getenv("SBR_PASS_EXPER") ? atoi(getenv("SBR_PASS_EXPER")) : 0;
   return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mapL, mapW, (int)p.r0, (int)p.M, NT, T0, T, p.b,
-                    p.X, p.ldx, exper, p.sh_nt, p.sh_ofs);
+                    p.X, p.ldx, exper);
 }
 
 static int pass_variant() {   // SBR_PASS_CFG (tuning experiments only): 0 = C8/NS4, 1 = C4/NS5, 2 = C2/NS6

@@ -93,6 +93,14 @@ __global__ void __launch_bounds__(256, 1)
   } else if (warp >= 4) {
     const int q = warp - 4;
     const int64_t r = (int64_t)tile * 128 + q * 32 + lane;
+    // C is independent of the accumulator: its loads are issued before the wait, so their latency
+    // hides under the mainloop
+    constexpr int BO = BN < 32 ? 32 : BN;
+    float o[BO];
+#pragma unroll
+    for (int c = 0; c < BO; ++c) o[c] = (!split && r < rows && c < b) ? Cin[r + (int64_t)c * ldc] : 0.f;
+    // row-major fp16 copy in 16-byte stores (8 halves) when aligned
+    const bool hvec = Hrm && (b % 8 == 0) && (ldhr % 8 == 0) && ((reinterpret_cast<uintptr_t>(Hrm) & 15) == 0);
     mbar_wait(acc_full, 0);
     tc_fence_after();
 #pragma unroll
@@ -112,18 +120,23 @@ __global__ void __launch_bounds__(256, 1)
         continue;
       }
       if (r < rows) {
-        float o[32];
-#pragma unroll
-        for (int c = 0; c < 32; ++c) o[c] = (c0 + c < b) ? Cin[r + (int64_t)(c0 + c) * ldc] : 0.f;
+        __align__(16) __half hv[32];
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
           const int n = c0 + c;
+          const float d = o[n] - v[c];
+          hv[c] = __float2half_rn(d);
           if (n < b) {
-            const float d = o[c] - v[c];
             Dout[r + (int64_t)n * ldd] = d;
-            if (Hcm) Hcm[r + (int64_t)n * ldhc] = __float2half_rn(d);
-            if (Hrm) Hrm[r * ldhr + n] = __float2half_rn(d);
+            if (Hcm) Hcm[r + (int64_t)n * ldhc] = hv[c];
+            if (Hrm && !hvec) Hrm[r * ldhr + n] = hv[c];
           }
+        }
+        if (hvec) {
+#pragma unroll
+          for (int g = 0; g < 4; ++g)
+            if (c0 + g * 8 < b)
+              *reinterpret_cast<uint4*>(Hrm + r * ldhr + c0 + g * 8) = *reinterpret_cast<const uint4*>(hv + g * 8);
         }
       }
     }

@@ -99,7 +99,6 @@ cudaError_t syr2k_lower(int64_t M, int K, const float* Y, int64_t ldy, const flo
 // ---- tcgen05 / TMA path (FP16 mode) ----
 cudaError_t make_tmap_2d(CUtensorMap* map, const void* base, bool fp16, uint64_t inner, uint64_t outer, uint64_t ld,
                          uint32_t box_inner, uint32_t box_outer, int l2_promo = 256);
-cudaError_t make_tmap_tiles(CUtensorMap* map, const void* base, uint64_t ntiles);
 
 struct PassLaunch {
   const __half* shadow;  // n x n fp16 shadow of the trailing matrix (strict lower, half diag, zero upper)
@@ -113,9 +112,6 @@ struct PassLaunch {
   int num_sms;
   int seg_rows;
   int rank = 0, nranks = 1;   // tile share of this launch (sbr_reduce_dist): [T*rank/nranks, T*(rank+1)/nranks)
-  // tile-contiguous shadow (shadow_init_tiles): sh_nt > 0 tiles per side of the global grid whose
-  // origin is row/col b; OA tile (I, J) is grid tile (sh_ofs + I, sh_ofs + J).  0: column-major.
-  int sh_nt = 0, sh_ofs = 0;
 };
 cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st);
 // host mirror of the pass's tile order (k_pass_tc.cu PassWalk): share of `rank`, and the (I, J) list
@@ -149,7 +145,6 @@ struct GemmTcLaunch {
   int64_t Mrows, Ncols;             // output size
   float* C; int64_t ldc;            // SYR2K: fp32 master (lower), column-major
   __half* shadow; int64_t ld_shadow;
-  int sh_nt = 0; int64_t sh_g0 = 0; // tile-contiguous shadow: C(0,0) is grid element (sh_g0, sh_g0)
   const float* X; int64_t ldx;      // ZFORM: X (column-major fp32)
   __half* Zh; int64_t ldz;          // ZFORM: Z out (row-major fp16)
   int num_sms;
@@ -241,8 +236,6 @@ cudaError_t f32cm_to_f16rm(int64_t rows, int cols, const float* src, int64_t lds
 cudaError_t build_lazy_b(int k, int b, const __half* Yh, int64_t ldyh, int64_t c, const float* P, __half* Bl,
                          int64_t ldbl, cudaStream_t st);
 cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int64_t ldsh, cudaStream_t st);
-// tile-contiguous shadow of A[b:, b:] (nt x nt grid of 128 x 128 tiles, lower tiles written)
-cudaError_t shadow_init_tiles(int64_t n, int b, int nt, const float* A, int64_t lda, __half* Sh, cudaStream_t st);
 cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
                        int64_t ldd, cudaStream_t st);
 

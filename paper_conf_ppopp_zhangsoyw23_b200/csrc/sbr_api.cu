@@ -73,7 +73,6 @@ struct sbr_ctx {
   unsigned chol_launches = 0;
   int panel_mode = 0;      // 0: CholeskyQR3 + TSQR fallback, 1: TSQR only (SBR_PANEL=tsqr)
   int64_t ldwh = 0, ldsh = 0, ldk = 0, ldbl = 0;
-  int sh_nt = 0;           // > 0: tile-contiguous fp16 shadow (sh_nt x sh_nt grid of 128 x 128 tiles from row/col b)
   int panel_ctas = 0;
   // host-buffer (e2e) device copies
   void* e2e = nullptr;
@@ -186,18 +185,8 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   // 128x128 tiles of it and unaligned tiles drag in neighbouring lines (L2 256 B promotion).
   const int64_t shoff = (nb % 128 == 0 && (128 - b % 128) % 8 == 0) ? (128 - b % 128) % 128 : 0;
   const int64_t ldsh = (n + shoff + 127) / 128 * 128;
-  // Experiment (opt-in, SBR_SHADOW_TILED=1; FP16 mode with nb % 128 == 0): every block's OA origin
-  // c0 + b sits on one fixed grid of 128 x 128 tiles (origin row/col b), so the shadow can be stored
-  // tile-contiguous -- each tile the pass streams is one 32 KB run of HBM instead of 128 column
-  // segments of 256 B.  A pure TMA stream of the pass's walk is 10% faster that way
-  // (tools/ubench/ubench_stream.cu, profiles/r08), but the pass itself did not move (94.7 vs 94.8 ms
-  // per step) and the SYR2K's scattered shadow stores cost 2 ms, so the column-major layout stays
-  // the default.
-  static const bool tiled_ok = getenv("SBR_SHADOW_TILED") && atoi(getenv("SBR_SHADOW_TILED")) == 1;
-  const int sh_nt = (tiled_ok && mode == SBR_FP16_FP32ACC && nb % 128 == 0) ? (int)((M + 127) / 128) : 0;
-  const size_t sh_halves = sh_nt > 0 ? (size_t)sh_nt * sh_nt * 16384 : (size_t)ldsh * n + shoff;
   const int64_t ldk = (nb + 7) / 8 * 8;
-  const size_t oSh = take(sh_halves / 2 + 128), oYh = take((size_t)n * ldk / 2 + 8),
+  const size_t oSh = take(((size_t)ldsh * n + shoff) / 2 + 128), oYh = take((size_t)n * ldk / 2 + 8),
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
@@ -244,8 +233,7 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->pq = (float*)(base + oPq);
   h->pmisc = (float*)(base + oPm);
   h->flag = (unsigned*)(base + oF);
-  h->Sh = (__half*)(base + oSh) + (sh_nt > 0 ? 0 : shoff);
-  h->sh_nt = sh_nt;
+  h->Sh = (__half*)(base + oSh) + shoff;
   h->Yh = (__half*)(base + oYh);
   h->Zh = (__half*)(base + oZh);
   h->Wh = (__half*)(base + oWh);
@@ -330,10 +318,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   const bool tc32 = !tc16 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0;
   if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper)
     Scope sc(h, SBR_K_OTHER, 6.0 * n * n, 0);
-    if (h->sh_nt > 0)
-      SBR_CK(shadow_init_tiles(n, b, h->sh_nt, A, lda, h->Sh, st), "shadow_init_tiles");
-    else
-      SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, st), "shadow_init");
+    SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, st), "shadow_init");
     h->launches += (n + 65534) / 65535;
   }
   if (tc16) {  // fp16 W copies: pad columns (b < BN) must read as zero in the pass
@@ -563,8 +548,6 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           pl.seg_rows = 8;
           pl.rank = h->rank;
           pl.nranks = h->nranks;
-          pl.sh_nt = h->sh_nt;
-          pl.sh_ofs = (int)(c0 / 128);
           SBR_CK(launch_pass_tc(pl, st), "pass_tc");
           h->launches += 1;
         }
@@ -670,10 +653,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       gs.Mrows = gs.Ncols = Mt;
       gs.C = A + (r0 + s) + (r0 + s) * lda;
       gs.ldc = lda;
-      gs.shadow = h->sh_nt > 0 ? h->Sh : h->Sh + (r0 + s) + (r0 + s) * h->ldsh;
+      gs.shadow = h->Sh + (r0 + s) + (r0 + s) * h->ldsh;
       gs.ld_shadow = h->ldsh;
-      gs.sh_nt = h->sh_nt;
-      gs.sh_g0 = r0 + s - b;   // grid coordinates of C(0,0)
       gs.num_sms = h->nsm;
       SBR_CK(launch_syr2k_tc(gs, st), "syr2k_tc");
       h->launches += 3;

@@ -41,19 +41,4 @@ cudaError_t make_tmap_2d(CUtensorMap* map, const void* base, bool fp16, uint64_t
   return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
 }
 
-// 3-D map over the tile-contiguous fp16 shadow: `ntiles` tiles of 128 x 128 halves, column-major
-// inside a tile (32 KB each); box = 64 rows x 128 columns of one tile; 128-byte swizzle.
-cudaError_t make_tmap_tiles(CUtensorMap* map, const void* base, uint64_t ntiles) {
-  EncodeTiledFn fn = get_encode();
-  if (!fn) return cudaErrorNotSupported;
-  cuuint64_t dims[3] = {128, 128, ntiles};
-  cuuint64_t strides[2] = {256, 32768};
-  cuuint32_t box[3] = {64, 128, 1};
-  cuuint32_t estr[3] = {1, 1, 1};
-  CUresult r = fn(map, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 3, const_cast<void*>(base), dims, strides, box, estr,
-                  CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-                  CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
-}
-
 }  // namespace sbr
