@@ -40,6 +40,13 @@ int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_t ldp, float* Y, float* W, int64_t ldyw,
                    int64_t* trace);
 
+/* Diagnostic: per-panel CholeskyQR phase stamps inside sbr_reduce.  cap > 0 arms recording
+ * for the next cap panels (device buffer owned by the handle, 16 int64 globaltimer stamps in
+ * ns per panel, CTA 0's view, stamp 0 taken before the PDL wait); host != NULL copies the
+ * stamps recorded so far (count * 16 int64) after synchronising the handle's stream and
+ * stores the panel count in *count (NULL count with non-NULL host: -4). */
+int sbr_test_panel_trace(sbr_handle_t h, int cap, int64_t* host, int* count);
+
 /* Same as sbr_test_pass_fp16 but only the share of `rank` of `nranks` (the tiles
  * sbr_test_pass_partition assigns): summing the X of all ranks gives the full pass. */
 int sbr_test_pass_fp16_part(sbr_handle_t h, int64_t M, int b, int rank, int nranks, const float* OA, int64_t ldoa,

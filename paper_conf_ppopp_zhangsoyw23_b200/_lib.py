@@ -57,6 +57,7 @@ SIGNATURES = {
     "sbr_test_syr2k_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_zform_fp16": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_panel": (_i, [_h, _i64, _i, _p, _i64, _p, _p, _i64, _p]),
+    "sbr_test_panel_trace": (_i, [_h, _i, _p, _p]),
     "sbr_test_pass_tf32": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _i64, _p, _i64, _p, _i64]),
     "sbr_test_syr2k_tf32": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_test_zform_tf32": (_i, [_h, _i64, _i, _p, _i64, _p, _i64, _p, _i64, _p, _i64]),

@@ -91,6 +91,9 @@ struct sbr_ctx {
   nccl::Comm comm = nullptr;
   bool force_coll = false;   // SBR_DIST_COLLECTIVES=1: issue the exchanges even with one rank (tests)
   bool tf32_tc = true;       // SBR_TF32_TC=0: 3xTF32 mode on the SIMT fp32 kernels (ablation)
+  // sbr_test_panel_trace: per-panel CholeskyQR phase stamps of the next sbr_reduce (16 int64 per panel)
+  int64_t* ptrace = nullptr;
+  int ptrace_cap = 0, ptrace_used = 0;
 };
 
 namespace {
@@ -438,6 +441,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         // mode's operands -- FP16 mode rounds every GEMM operand to fp16 (u = 4.9e-4), 3xTF32 keeps
         // fp32 (u = 6e-8)
         pa.orth_tol = tc16 ? 1e-6 : 1e-8;
+        if (h->ptrace && h->ptrace_used < h->ptrace_cap) pa.trace = h->ptrace + 16 * (int64_t)h->ptrace_used++;
         bool chol = false;
         if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
           const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
@@ -449,6 +453,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
             SBR_CK(ce, "panel_chol");
           }
         }
+        pa.trace = nullptr;   // the phase trace is CholeskyQR's (the TSQR fallback has its own stamps)
         const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
         if (te == cudaErrorInvalidValue && chol) {
           // panel taller than the TSQR tree can hold (one co-resident CTA per 256-row leaf): no
@@ -855,6 +860,7 @@ int sbr_destroy(sbr_handle_t h) {
   if (h->ws) cudaFree(h->ws);
   if (h->e2e) cudaFree(h->e2e);
   if (h->fq) cudaFree(h->fq);
+  if (h->ptrace) cudaFree(h->ptrace);
   delete h;
   return SBR_OK;
 }
@@ -1367,6 +1373,31 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
   if (trace_host) {
     SBR_CK(cudaMemcpyAsync(trace_host, tr.p, sizeof(int64_t) * 16, cudaMemcpyDeviceToHost, st), "trace D2H");
     SBR_CK(cudaStreamSynchronize(st), "sync");
+  }
+  return SBR_OK;
+}
+
+// Per-panel phase trace of the reduction: arm (cap > 0: the next cap CholeskyQR panels of
+// sbr_reduce record their 16 globaltimer stamps), then read (host != NULL: copies the stamps
+// of the recorded panels, returns their count in *count).  Diagnostic only.
+extern "C" int sbr_test_panel_trace(sbr_handle_t h, int cap, int64_t* host, int* count) {
+  if (!h) return -1;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  if (cap > 0) {
+    if (h->ptrace) cudaFree(h->ptrace);
+    h->ptrace = nullptr;
+    SBR_CK(cudaMalloc(&h->ptrace, sizeof(int64_t) * 16 * (size_t)cap), "trace alloc");
+    SBR_CK(cudaMemsetAsync(h->ptrace, 0, sizeof(int64_t) * 16 * (size_t)cap, h->stream), "trace memset");
+    h->ptrace_cap = cap;
+    h->ptrace_used = 0;
+  }
+  if (host) {
+    if (!count) return -4;
+    SBR_CK(cudaStreamSynchronize(h->stream), "sync");
+    *count = h->ptrace_used;
+    if (h->ptrace_used > 0)
+      SBR_CK(cudaMemcpy(host, h->ptrace, sizeof(int64_t) * 16 * (size_t)h->ptrace_used, cudaMemcpyDeviceToHost),
+             "trace D2H");
   }
   return SBR_OK;
 }
