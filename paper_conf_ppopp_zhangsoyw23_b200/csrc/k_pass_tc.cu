@@ -150,6 +150,8 @@ __global__ void __launch_bounds__(256, 1)
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
     if (lane == 0) {
+      // OA tiles are read once per pass: evict_first (SBR_PASS_EXPER bit 2 = normal, ablation)
+      const uint64_t lpol = (exper & 4) ? l2_policy_evict_normal() : l2_policy_evict_first();
       int st = 0; uint32_t ph = 0;            // L ring
       int ws = 0; uint32_t wph = 0;           // W_I ring
       uint32_t jph = 0;
@@ -172,7 +174,7 @@ __global__ void __launch_bounds__(256, 1)
         mbar_expect_tx(&l_full[st], Cfg::LT);
         uint8_t* dst = sL + st * Cfg::LT;
         for (int rb = 0; rb < 2; ++rb)   // box = 64 rows x 128 columns (same smem image as 2 boxes of 64)
-          tma_load_2d(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, r0 + w.J * 128);
+          tma_load_2d_hint(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, r0 + w.J * 128, lpol);
         if (++st == NS) { st = 0; ph ^= 1; }
         if (w.rlast()) {
           if (++ws == 2) { ws = 0; wph ^= 1; }

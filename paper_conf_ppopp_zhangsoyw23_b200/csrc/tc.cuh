@@ -49,6 +49,28 @@ SBR_DEV void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int c
       : "memory");
 }
 
+// L2 eviction policies for streamed operands: a tile read exactly once is loaded evict_first so
+// the stream does not push the per-panel working set (X, Y, W, the chain kernels' code) out of L2.
+SBR_DEV uint64_t l2_policy_evict_first() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+SBR_DEV uint64_t l2_policy_evict_normal() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+// 2-D tile load with an L2 cache policy (from l2_policy_*).
+SBR_DEV void tma_load_2d_hint(void* dst, const CUtensorMap* map, uint64_t* bar, int c_inner, int c_outer,
+                              uint64_t policy) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c_inner), "r"(c_outer), "l"(policy)
+      : "memory");
+}
+
 // ------------------------------------------------------------------ tcgen05
 SBR_DEV void tmem_alloc(uint32_t* dst_smem, uint32_t ncols) {  // whole warp
   asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
