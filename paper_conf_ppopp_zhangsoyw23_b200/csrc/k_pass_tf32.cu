@@ -26,6 +26,9 @@
 // into X).  2 stages of {L tile 64 KB, W_I
 // 32 KB} + W_J 32 KB = 224 KB smem.  Work: tile columns J in order, rows I = J .. NT-1 (group
 // = one tile column, W_J resident), a balanced contiguous range of tiles per CTA.
+#include <cstdlib>
+#include <cstring>
+
 #include "kernels.h"
 #include "tc.cuh"
 
@@ -74,7 +77,7 @@ SBR_DEV void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::
 __global__ void __launch_bounds__(P3_THREADS, 1)
     pass_tf32_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapS,
                      const __grid_constant__ CUtensorMap mapW, int r0, int M, int NT, int jstrip, int64_t T0,
-                     int64_t T, int b, float* X, int64_t ldx) {
+                     int64_t T, int b, float* X, int64_t ldx, int l2normal) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint64_t* bars = (uint64_t*)(smem + P3_OFF_BAR);
@@ -121,6 +124,8 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
     if (lane == 0) {
+      // OA / strip tiles are read once per pass: evict_first (SBR_TF32_L2=normal: ablation)
+      const uint64_t lpol = l2normal ? l2_policy_evict_normal() : l2_policy_evict_first();
       int st = 0; uint32_t ph = 0;
       uint32_t jph = 0;
       for (w.start(NT, t_beg, t_end - t_beg); w.valid(); w.next()) {
@@ -137,9 +142,9 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
         const bool strip = w.J < jstrip;
         for (int rc = 0; rc < 4; ++rc) {
           if (strip)
-            tma_load_2d(dst + rc * 16384, &mapS, &l_full[st], w.I * 128 + rc * 32, w.J * 128);
+            tma_load_2d_hint(dst + rc * 16384, &mapS, &l_full[st], w.I * 128 + rc * 32, w.J * 128, lpol);
           else
-            tma_load_2d(dst + rc * 16384, &mapA, &l_full[st], r0 + w.I * 128 + rc * 32, r0 + w.J * 128);
+            tma_load_2d_hint(dst + rc * 16384, &mapA, &l_full[st], r0 + w.I * 128 + rc * 32, r0 + w.J * 128, lpol);
         }
         for (int rc = 0; rc < 4; ++rc)
           tma_load_2d(dst + P3_LT + rc * 8192, &mapW, &l_full[st], w.I * 128 + rc * 32, 0);
@@ -362,8 +367,9 @@ cudaError_t launch_pass_tf32(const PassTf32Launch& p, cudaStream_t st) {
   const int64_t T = T1 - T0;
   if (T <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
+  static const int l2normal = (getenv("SBR_TF32_L2") && !strcmp(getenv("SBR_TF32_L2"), "normal")) ? 1 : 0;
   return launch_pdl(kern, dim3(grid), dim3(P3_THREADS), P3_SMEM, st, mapA, mapS, mapW, (int)p.r0, (int)p.M, NT,
-                    jstrip, T0, T, p.b, p.X, p.ldx);
+                    jstrip, T0, T, p.b, p.X, p.ldx, l2normal);
 }
 
 // ---------------------------------------------------------------- operand splits (3xTF32)
