@@ -43,12 +43,17 @@ def parse():
     p.add_argument("--b", type=int, default=CONFIG4["b"])
     p.add_argument("--nb", type=int, default=CONFIG4["nb"])
     p.add_argument("--mode", default=CONFIG4["mode"])
+    p.add_argument("--input", default="uniform", choices=["uniform", "geo"],
+                   help="uniform: random symmetric U[-1,1) (configs 1, 3, 4); geo: prescribed spectrum "
+                        "SVD_Geo kappa=1e5 (configs 2, 5)")
     p.add_argument("--e2e-steps", type=int, default=2)
     p.add_argument("--form-q-steps", type=int, default=1,
                    help="also time sbr_form_q (Q = prod (I - W Y^T), 3xTF32) on the last step's output (0: skip)")
     p.add_argument("--profile-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-sample-s", type=float, default=15.0)
+    p.add_argument("--lapack-n", type=int, default=4096,
+                   help="n of the LAPACK ssytrd_sy2sb/dsytrd_sy2sb host baseline (0: skip)")
     return p.parse_args()
 
 
@@ -162,6 +167,63 @@ def cpu_oracle_sample(n: int, b: int, a_host, budget_s: float):
     }
 
 
+def lapack_sy2sb_baseline(n_lapack: int, b: int, n_target: int, seed: int):
+    """LAPACK ssytrd_sy2sb / dsytrd_sy2sb (UPLO='L', kd=b) from scipy's bundled OpenBLAS on all
+    host cores (north_star / BASELINE.md §4): the same reduction (entry-wise equal up to
+    rounding) in fp32 and fp64, at n_lapack (bounded: finishes in seconds), reported
+    as effective TFLOP/s ((4/3) n^3) and extrapolated by n^3 to n_target."""
+    import ctypes
+    import glob
+
+    import numpy as np
+    import scipy
+
+    import workloads
+
+    d = os.path.join(os.path.dirname(scipy.__file__), "..", "scipy.libs")
+    cands = sorted(glob.glob(os.path.join(d, "libscipy_openblas*.so")))
+    if not cands:
+        return None
+    lib = ctypes.CDLL(cands[0])
+    a0 = workloads.random_symmetric(n_lapack, seed)
+    out = {}
+    for name, dtype, fn in (("ssytrd_sy2sb", np.float32, "scipy_ssytrd_sy2sb_"),
+                            ("dsytrd_sy2sb", np.float64, "scipy_dsytrd_sy2sb_")):
+        if not hasattr(lib, fn):
+            continue
+        f = getattr(lib, fn)
+        n = n_lapack
+        af = np.asfortranarray(a0.astype(dtype))
+        ab = np.zeros((b + 1, n), dtype=dtype, order="F")
+        tau = np.zeros(max(1, n - b), dtype=dtype)
+        info = ctypes.c_int(0)
+        uplo = ctypes.c_char(b"L")
+        i32 = ctypes.c_int
+        ptr = lambda x: x.ctypes.data_as(ctypes.c_void_p)  # noqa: E731
+        wq = np.zeros(1, dtype=dtype)
+        args = [ctypes.byref(uplo), ctypes.byref(i32(n)), ctypes.byref(i32(b)), ptr(af), ctypes.byref(i32(n)),
+                ptr(ab), ctypes.byref(i32(b + 1)), ptr(tau)]
+        f(*args, ptr(wq), ctypes.byref(i32(-1)), ctypes.byref(info), ctypes.c_size_t(1))
+        work = np.zeros(max(1, int(wq[0])), dtype=dtype)
+        t0 = time.perf_counter()
+        f(*args, ptr(work), ctypes.byref(i32(work.size)), ctypes.byref(info), ctypes.c_size_t(1))
+        dt = time.perf_counter() - t0
+        out[name] = {"seconds": dt, "n": n, "tflops": eff_tflops(n, dt),
+                     "extrapolated_seconds_at_n_target": dt * (n_target / n) ** 3, "info": info.value}
+    try:
+        from threadpoolctl import threadpool_info
+
+        thr = max((i.get("num_threads", 1) for i in threadpool_info() if "openblas" in i.get("internal_api", "")),
+                  default=len(os.sched_getaffinity(0)))
+    except Exception:
+        thr = len(os.sched_getaffinity(0))
+    out["cores"] = int(thr)
+    out["host_cpus"] = len(os.sched_getaffinity(0))
+    out["note"] = (f"LAPACK (scipy OpenBLAS) dense->band, UPLO=L, kd={b}, on the same seeded generator at "
+                   f"n={n_lapack} (bounded; n^3-extrapolated to n={n_target})")
+    return out
+
+
 def dist_setup():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -190,13 +252,17 @@ def run_reference(args, rank, world):
     a_host = workloads.random_symmetric(n, workloads.config_seed(4))
     ncol_total = max(0, n - b - 1)
     w = (n - np.arange(ncol_total, dtype=np.float64) - b)
+    # the oracle's setup (fp64 copy + symmetrisation of the n x n input) is timed once; every
+    # step then times ONE column of the plain unblocked reduction on that input, and the full
+    # reduction time is extrapolated by the per-column cost (n - c - b)
+    st = {}
+    t0 = time.perf_counter()
+    osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=1, stats=st)
+    setup = time.perf_counter() - t0 - st["loop_seconds"]
     vals, last = [], None
     for i in range(args.warmup + args.steps):
         st = {}
-        t0 = time.perf_counter()
         osbr.sbr_unblocked(a_host, b, want_q=False, max_cols=1, stats=st)
-        total = time.perf_counter() - t0
-        setup = total - st["loop_seconds"]
         t_full = setup + st["loop_seconds"] * float(w.sum() / w[0])
         if i >= args.warmup:
             vals.append(eff_tflops(n, t_full))
@@ -204,8 +270,8 @@ def run_reference(args, rank, world):
     v = statistics.median(vals)
     cores = len(os.sched_getaffinity(0))
     sample = (f"per step: oracle.sbr.sbr_unblocked (fp64 numpy, as it stands) on the n={n} b={b} input for 1 "
-              f"of {ncol_total} columns (setup {last[0]:.1f} s + column {last[1]:.2f} s), extrapolated by "
-              f"per-column cost (n-c-b) to ~{last[2]:.3g} s for the full reduction")
+              f"of {ncol_total} columns ({last[1]:.2f} s; the oracle's setup, {last[0]:.1f} s, timed once), "
+              f"extrapolated by per-column cost (n-c-b) to ~{last[2]:.3g} s for the full reduction")
     line = {
         "impl": "reference",
         "metric": METRIC, "value": v, "unit": "TFLOP/s", "n_gpus": args.gpus, "steps": args.steps,
@@ -237,8 +303,9 @@ def main():
 
     n, b, nb, mode = args.n, args.b, args.nb, args.mode
     cfg_name = {(32768, 32, 1024, "fp16"): "config4", (16384, 32, 1024, "3xtf32"): "config3",
+                (4096, 32, 256, "fp16"): "config2", (65536, 64, 2048, "3xtf32"): "config5",
                 (65536, 64, 2048, "3xtf32"): "config5-params"}.get((n, b, nb, mode), "custom")
-    seed = workloads.config_seed({"config3": 3, "config5-params": 5}.get(cfg_name, 4))
+    seed = workloads.config_seed({"config2": 2, "config3": 3, "config5": 5, "config5-params": 5}.get(cfg_name, 4))
     stream = torch.cuda.current_stream()
     if world > 1:
         # one matrix across the ranks (sbr_reduce_dist, strong scaling): NCCL communicator
@@ -248,7 +315,12 @@ def main():
         h = sbr.Handle(local, stream, unique_id=uid[0], rank=rank, nranks=world)
     else:
         h = sbr.Handle(local, stream)
-    pristine = h.generate_symmetric(seed, n)              # device twin of workloads.random_symmetric
+    if args.input == "uniform":
+        pristine = h.generate_symmetric(seed, n)          # device twin of workloads.random_symmetric
+        input_desc = f"random symmetric U[-1,1) (seed {seed})"
+    else:   # prescribed spectrum, SVD_Geo kappa = 1e5: Haar Q (host) or randomised Hadamard Q (device)
+        pristine, input_desc = workloads.prescribed_spectrum_device(n, "geo", 1e5, seed, a_device=f"cuda:{local}")
+    pristine_np = None
     a = torch.empty_like(pristine)
     ab = torch.empty((n, b + 1), dtype=torch.float32, device=a.device) if rank == 0 else None
     w = torch.empty((n - b, n), dtype=torch.float32, device=a.device) if rank == 0 else None
@@ -410,10 +482,16 @@ def main():
         del a_host
     cpu = None
     if rank == 0 and not args.no_cpu_baseline:
-        a_np = workloads.random_symmetric(n, seed)
+        a_np = pristine.cpu().numpy()   # the same input bits
         cpu = cpu_oracle_sample(n, b, a_np, args.cpu_sample_s)
         cpu.pop("seconds_extrapolated", None)
         del a_np
+    lapack = None
+    if rank == 0 and not args.no_cpu_baseline and args.lapack_n > 0:
+        try:
+            lapack = lapack_sy2sb_baseline(min(args.lapack_n, n), b, n, seed)
+        except Exception as e:  # pragma: no cover
+            lapack = {"error": str(e)}
 
     if rank == 0:
         line = {
@@ -430,7 +508,7 @@ def main():
             "vs_baseline": None,
             "dtype": "f32" if mode == "3xtf32" else "f16",
             "data": "synthetic",
-            "config": {"workload": f"{cfg_name}: n={n} random symmetric U[-1,1) (seed {seed}), b={b}, nb={nb}, "
+            "config": {"workload": f"{cfg_name}: n={n} {input_desc}, b={b}, nb={nb}, "
                                    f"{'FP16-in/FP32-acc' if mode == 'fp16' else '3xTF32'}",
                        "n": n, "b": b, "nb": nb, "mode": mode,
                        "parallelism": f"sbr_reduce_dist over {world} GPUs: per-panel pass sharded by lower "
@@ -442,6 +520,7 @@ def main():
             "roofline": roof,
             "breakdown": breakdown,
             "cpu_baseline": cpu,
+            "lapack_baseline": lapack,
             "e2e": e2e,
             "form_q": formq,
             "gpu_launches": launches,

@@ -43,7 +43,7 @@ extern "C" {
 #endif
 
 #define SBR_OK 0
-#define SBR_ERR_NONFINITE 1  /* input holds Inf/NaN (detected before any update)   */
+#define SBR_ERR_NONFINITE 1  /* input holds Inf/NaN, or the band overflowed fp32   */
 #define SBR_ERR_CUDA 2       /* CUDA runtime/driver error; see sbr_status_string    */
 #define SBR_ERR_NCCL 3       /* reserved for the multi-GPU path                     */
 #define SBR_ERR_NOMEM 4      /* device workspace allocation failed                  */
@@ -97,11 +97,19 @@ int sbr_workspace_query(sbr_handle_t h, int64_t n, int b, int nb, int mode, size
  *           If NULL, W lives in handle workspace (per block) and is dropped. (arg 10)
  *   ldw   : >= n if W != NULL.                                (arg 11)
  * Trivial case n <= b+1: AB = band of A, W untouched, no reflectors.
- * Returns 0, -i, SBR_ERR_NONFINITE, SBR_ERR_CUDA, SBR_ERR_NOMEM, or SBR_ERR_UNSUPPORTED when
- * a panel taller than the TSQR fallback's capacity (148 x 256 rows at b <= 32, n >~ 37900)
- * is numerically rank deficient for CholeskyQR (the results are then invalid).  Synchronises
- * the stream once at the start (4-byte read of the input's finiteness flag), and once more at
- * the end only when such tall panels occurred (4-byte read of the fallback flag). */
+ * FP16 mode range handling (a0, reading C10): the reduction runs on 2^k A with the
+ * exact power of two 2^k chosen on the device so that ||A||_F 2^k lies in [2^12, 2^13) -- every
+ * fp16 operand then stays below 2^15 and typical entries far from fp16's subnormals.  The
+ * fp32 master (A's lower triangle) is scaled in place; on exit the band (in A and in AB) is
+ * unscaled by 2^-k, Y and W are scale free.  The 3xTF32 mode takes the same scale (its fp32
+ * panel norms and products would under/overflow near the ends of the fp32 range).
+ * Returns (argument checks, enqueue failures) 0, -i, SBR_ERR_CUDA, SBR_ERR_NOMEM, or an error
+ * LATCHED by an earlier call on this handle.  The call never synchronises the host: errors
+ * detected on the device -- SBR_ERR_NONFINITE (Inf/NaN in the referenced input, or a
+ * non-finite band entry, i.e. fp16 range exceeded after scaling) and SBR_ERR_UNSUPPORTED (a
+ * panel taller than the TSQR fallback's capacity, 148 x 256 rows at b <= 32, n >~ 37900, was
+ * numerically rank deficient for CholeskyQR) -- are latched and returned by sbr_sync or by
+ * the next call on the handle; the outputs of that reduction are then invalid. */
 int sbr_reduce(sbr_handle_t h, int mode, int64_t n, int b, int nb,
                float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw);
 
@@ -166,7 +174,8 @@ int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb,
 int sbr_rank(sbr_handle_t h);     /* 0 for sbr_create handles; -1 if h is NULL */
 int sbr_nranks(sbr_handle_t h);   /* 1 for sbr_create handles; -1 if h is NULL */
 
-/* Wait for all work enqueued on the handle's stream. */
+/* Wait for all work enqueued on the handle's stream; returns the first error latched by a
+ * finished reduction (SBR_ERR_NONFINITE / SBR_ERR_UNSUPPORTED, see sbr_reduce) or 0. */
 int sbr_sync(sbr_handle_t h);
 
 /* Human-readable text for a status code (static storage; includes the last

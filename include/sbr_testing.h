@@ -79,6 +79,17 @@ int sbr_test_syr2k_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_zform_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
                         const float* X, int64_t ldx, float* Z, int64_t ldz);
 
+/* Number of CholeskyQR panels that declined (rank deficient / not orthonormal after three
+ * rounds, so the paper's TSQR factored them) since the handle's workspace was allocated or
+ * the last call with reset != 0.  Synchronises.  Returns 0, -1 (h), -3 (count NULL). */
+int sbr_test_panel_declines(sbr_handle_t h, int reset, int64_t* count);
+
+/* Experiment knobs (timing experiments only; process-wide, 0 = production behaviour):
+ *   knob 0 (pass experiment bits): 1 = skip the pass's L W MMAs, 2 = skip its L^T W MMAs
+ *   (results are WRONG: for timing the stream alone), 4 = normal L2 policy for the OA stream.
+ * Returns 0, or -1 for an unknown knob. */
+int sbr_test_set_knob(int knob, int value);
+
 #ifdef __cplusplus
 }
 #endif

@@ -64,6 +64,8 @@ SIGNATURES = {
     "sbr_test_pass_partition": (_i, [_i64, _i, _i, _i, ctypes.POINTER(_i64), ctypes.POINTER(_i64),
                                      ctypes.POINTER(_i64)]),
     "sbr_test_pass_tiles": (_i, [_i64, _i, _i64, _i64, _p]),
+    "sbr_test_set_knob": (_i, [_i, _i]),
+    "sbr_test_panel_declines": (_i, [_h, _i, ctypes.POINTER(_i64)]),
 }
 
 _LIB = None

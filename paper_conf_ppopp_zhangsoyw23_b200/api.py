@@ -106,7 +106,8 @@ class Handle:
         Returns ``(ab, w)``: ``ab`` (n, b+1) with ``ab[j, d] = B[j+d, j]``; ``w``
         (n-b, n) with ``w[c, r] = W(r, c)`` (None if ``want_w`` is False).  A is
         overwritten with the sy2sb layout (see the package docstring).  Enqueued on
-        the handle's stream; no host synchronisation except the input check.
+        the handle's stream without host synchronisation: device-detected errors (non-finite
+        input, fp16 range) are latched and raised by :meth:`sync` or the next call.
         """
         import torch
 
@@ -115,8 +116,8 @@ class Handle:
             raise ValueError("A must be a contiguous square float32 CUDA tensor")
         if ab is None:
             ab = torch.empty((n, b + 1), dtype=torch.float32, device=A.device)
-        if want_w and w is None and n > b:
-            w = torch.empty((max(n - b, 1), n), dtype=torch.float32, device=A.device)
+        if want_w and w is None and n > b:   # zeros: entries the reduction does not reference stay 0
+            w = torch.zeros((max(n - b, 1), n), dtype=torch.float32, device=A.device)
         if not want_w:
             w = None
         check(lib().sbr_reduce(self._h, _mode(mode), n, int(b), int(nb), _ptr(A), n, _ptr(ab), b + 1,
@@ -205,6 +206,12 @@ class Handle:
         check(lib().sbr_kernel_stats(self._h, kid, ctypes.byref(n), ctypes.byref(ms), ctypes.byref(by),
                                      ctypes.byref(fl)), "kernel_stats")
         return {"launches": n.value, "ms": ms.value, "bytes": by.value, "flops": fl.value}
+
+    def panel_declines(self, reset: bool = True) -> int:
+        """Test hook: CholeskyQR panels that declined (TSQR fallback) since the last reset."""
+        c = ctypes.c_int64()
+        check(lib().sbr_test_panel_declines(self._h, int(bool(reset)), ctypes.byref(c)), "panel_declines")
+        return int(c.value)
 
     def launch_count(self) -> int:
         return int(lib().sbr_launch_count(self._h))

@@ -53,6 +53,18 @@ SBR_DEV void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 
 bool pdl_enabled();   // SBR_PDL=0 disables (ablation)
 
+// cudaFuncSetAttribute is per device context: set (fn, attr) = value once per device
+// (cached under a mutex keyed by the current device), so a handle on a second device in
+// the same process gets its own attributes.  k_misc.cu.
+cudaError_t func_attr(const void* fn, cudaFuncAttribute attr, int value);
+// occupancy-derived co-resident CTAs per SM of (fn, threads, smem) on the current device (cached)
+int func_blocks_per_sm(const void* fn, int threads, size_t smem);
+int current_device_sms();
+
+// test-only experiment knobs (sbr_testing.h sbr_test_set_knob); 0 unless a test set them
+enum Knob { KNOB_PASS_EXPER = 0, KNOB_COUNT = 8 };
+int knob(Knob k);
+
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
                               Args&&... args) {

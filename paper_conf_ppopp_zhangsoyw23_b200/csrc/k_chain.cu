@@ -156,12 +156,8 @@ template <int CL, int NG>
 static cudaError_t launch_kxb_t(const KxbArgs& a, cudaStream_t st) {
   auto kern = kxb_kernel<CL, NG>;
   if (CL > 8) {
-    static bool attr = false;
-    if (!attr) {
-      const cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-      if (e != cudaSuccess) return e;
-      attr = true;
-    }
+    const cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    if (e != cudaSuccess) return e;
   }
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((a.k + KXB_QT - 1) / KXB_QT, CL);

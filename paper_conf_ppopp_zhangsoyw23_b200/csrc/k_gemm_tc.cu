@@ -286,11 +286,9 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   auto kern = gemm_tc_kernel<MODE, TF>;
   constexpr int BK = TF ? 32 : 64;
   constexpr int G_BN = GCfg<TF>::BN, G_SMEM = GCfg<TF>::SMEM;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, G_SMEM);
+  {
+    cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, G_SMEM);
     if (e != cudaSuccess) return e;
-    attr = true;
   }
   CUtensorMap mA0, mA1, mB0, mB1;
   cudaError_t e;

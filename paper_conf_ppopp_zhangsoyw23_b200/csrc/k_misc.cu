@@ -1,9 +1,61 @@
 // k_misc.cu -- small kernels: input generator, finiteness check, band extraction,
 // symmetric mirrors, the k x b correction of the lazy panel update.
+#include <map>
+#include <mutex>
+#include <tuple>
+
 #include "common.cuh"
 #include "kernels.h"
 
 namespace sbr {
+
+namespace {
+std::mutex g_attr_mu;
+std::map<std::tuple<const void*, int, int>, int> g_attr;   // (fn, attr, device) -> value set
+std::map<std::tuple<const void*, int, size_t, int>, int> g_occ;   // (fn, threads, smem, device) -> blocks/SM
+int g_knobs[KNOB_COUNT] = {};
+}  // namespace
+
+cudaError_t func_attr(const void* fn, cudaFuncAttribute attr, int value) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  std::lock_guard<std::mutex> lk(g_attr_mu);
+  const auto key = std::make_tuple(fn, (int)attr, dev);
+  auto it = g_attr.find(key);
+  if (it != g_attr.end() && it->second == value) return cudaSuccess;
+  e = cudaFuncSetAttribute(fn, attr, value);
+  if (e == cudaSuccess) g_attr[key] = value;
+  return e;
+}
+
+int func_blocks_per_sm(const void* fn, int threads, size_t smem) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(g_attr_mu);
+  const auto key = std::make_tuple(fn, threads, smem, dev);
+  auto it = g_occ.find(key);
+  if (it != g_occ.end()) return it->second;
+  int per = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, fn, threads, smem) != cudaSuccess) {
+    cudaGetLastError();
+    per = 0;
+  }
+  g_occ[key] = per;
+  return per;
+}
+
+int current_device_sms() {
+  int dev = 0, n = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+  return n;
+}
+
+int knob(Knob k) { return (k >= 0 && k < KNOB_COUNT) ? g_knobs[k] : 0; }
+void set_knob(int k, int v) {
+  if (k >= 0 && k < KNOB_COUNT) g_knobs[k] = v;
+}
 
 bool pdl_enabled() {
   static int v = -1;
@@ -40,20 +92,83 @@ cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaS
   return cudaGetLastError();
 }
 
-__global__ void check_finite_kernel(int64_t n, const float* A, int64_t lda, unsigned* flag) {
+// a0 scan (reading C10): finiteness of the referenced lower triangle (flag[0] |= 1) and
+// ||A||_F^2 in fp64 (off-diagonal entries twice), one fp64 atomic per block.
+__global__ void prep_scan_kernel(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2) {
   const int64_t j = blockIdx.y;
+  double s = 0.0;
+  bool bad = false;
   for (int64_t i = j + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
-    if (!isfinite(A[i + j * lda])) { atomicOr(flag, 1u); return; }
+    const float v = A[i + j * lda];
+    if (!isfinite(v)) bad = true;
+    s += (i == j ? 1.0 : 2.0) * (double)v * (double)v;
+  }
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(flag, 1u);
+  __shared__ double red[32];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    s = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : 0.0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (threadIdx.x == 0 && s != 0.0) atomicAdd(fro2, s);
   }
 }
 
-cudaError_t check_finite(int64_t n, const float* A, int64_t lda, unsigned* flag, cudaStream_t st) {
-  cudaError_t e = cudaMemsetAsync(flag, 0, sizeof(unsigned), st);
+// Exact power-of-two scale (reading C10): 2^k with ||A||_F 2^k in [2^12, 2^13).  Every
+// trailing matrix of the reduction is orthogonally similar to a principal part of A, so its
+// entries are <= ||A||_2 <= ||A||_F; X = OA W and Z stay within a few times that: all fp16
+// operands stay below 2^15 < 65504, and typical entries (||A||_F / n) far above fp16's
+// subnormal range.  The 3xTF32 mode takes the same scale (tf32 has fp32's exponent range,
+// but the fp32 panel norms and products of an input near the ends of that range would
+// under- or overflow).  k = 0 for a zero or non-finite input.
+__global__ void choose_scale_kernel(const double* fro2, const unsigned* flag, int fp16_mode, int* kexp) {
+  int k = 0;
+  const double f2 = *fro2;
+  if (!flag[0] && f2 > 0.0 && isfinite(f2)) {   // both modes (fp16_mode kept for the record)
+    int e = 0;
+    frexp(sqrt(f2), &e);   // ||A||_F in [2^(e-1), 2^e)
+    k = max(-250, min(250, 13 - e));
+  }
+  *kexp = k;
+}
+
+cudaError_t prep_scale(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2, int* kexp,
+                       bool fp16_mode, cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(fro2, 0, sizeof(double), st);
   if (e != cudaSuccess) return e;
   for (int64_t j0 = 0; j0 < n; j0 += 65535) {
     const int64_t nc = std::min<int64_t>(65535, n - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 16), (unsigned)nc);
-    check_finite_kernel<<<grid, 256, 0, st>>>(n - j0, A + j0 + j0 * lda, lda, flag);
+    prep_scan_kernel<<<grid, 256, 0, st>>>(n - j0, A + j0 + j0 * lda, lda, flag, fro2);
+  }
+  choose_scale_kernel<<<1, 1, 0, st>>>(fro2, flag, fp16_mode ? 1 : 0, kexp);
+  return cudaGetLastError();
+}
+
+// a * 2^k, exact whenever the result is a normal float (two factors keep each within range)
+// (|k| <= 252; 2^j built from its exponent bits, j in [-126, 126])
+SBR_DEV float scale_pow2(float a, int k) {
+  const int k1 = k / 2, k2 = k - k1;
+  return (a * __int_as_float((k1 + 127) << 23)) * __int_as_float((k2 + 127) << 23);
+}
+
+// 3xTF32 mode: the lower triangle of A scaled in place by 2^k (no-op for k = 0)
+__global__ void scale_lower_kernel(int64_t n, int64_t j0, float* A, int64_t lda, const int* kexp) {
+  const int k = *kexp;
+  if (k == 0) return;
+  const int64_t j = j0 + blockIdx.y;
+  for (int64_t i = j + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    A[i + j * lda] = scale_pow2(A[i + j * lda], k);
+}
+
+cudaError_t scale_lower(int64_t n, float* A, int64_t lda, const int* kexp, cudaStream_t st) {
+  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, n - j0);
+    dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 32), (unsigned)nc);
+    scale_lower_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, kexp);
   }
   return cudaGetLastError();
 }
@@ -70,17 +185,34 @@ cudaError_t note_unhandled(const int* fail, unsigned* sticky, cudaStream_t st) {
   return launch_pdl(note_unhandled_kernel, dim3(1), dim3(32), 0, st, fail, sticky);
 }
 
-__global__ void extract_band_kernel(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab) {
+// Band out (a7): AB = 2^-k (band of A), written back into A's band unscaled too (A's Y part is
+// scale free); a non-finite band entry (fp16 range exceeded despite the scaling) latches flag[2].
+__global__ void extract_band_kernel(int64_t n, int b, float* A, int64_t lda, float* AB, int64_t ldab,
+                                    const int* kexp, unsigned* flag) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
   const int d = threadIdx.x;
-  if (j >= n || d > b) return;
-  AB[d + j * ldab] = (j + d < n) ? A[(j + d) + j * lda] : 0.f;
+  const int k = kexp ? *kexp : 0;
+  bool bad = false;
+  if (j < n && d <= b) {
+    float v = 0.f;
+    if (j + d < n) {
+      v = A[(j + d) + j * lda];
+      if (k != 0) {
+        v = scale_pow2(v, -k);
+        A[(j + d) + j * lda] = v;
+      }
+      bad = !isfinite(v);
+    }
+    AB[d + j * ldab] = v;
+  }
+  if (flag && __syncthreads_or(bad) && threadIdx.x == 0 && threadIdx.y == 0) atomicOr(flag + 2, 1u);
 }
 
-cudaError_t extract_band(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab, cudaStream_t st) {
+cudaError_t extract_band(int64_t n, int b, float* A, int64_t lda, float* AB, int64_t ldab, const int* kexp,
+                         unsigned* flag, cudaStream_t st) {
   const int dx = b + 1;
   const int dy = max(1, 256 / dx);
-  extract_band_kernel<<<(unsigned)((n + dy - 1) / dy), dim3(dx, dy), 0, st>>>(n, b, A, lda, AB, ldab);
+  extract_band_kernel<<<(unsigned)((n + dy - 1) / dy), dim3(dx, dy), 0, st>>>(n, b, A, lda, AB, ldab, kexp, flag);
   return cudaGetLastError();
 }
 
@@ -133,23 +265,33 @@ cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaS
   return cudaMemset2DAsync(A, lda * sizeof(float), 0, rows * sizeof(float), cols, st);
 }
 
-// fp16 shadow of the lower triangle: strict lower as is, HALF the diagonal, zero above
-// (so that a diagonal tile T satisfies T + T^T = L; see k_pass_tc.cu).
-__global__ void shadow_init_kernel(int64_t n, int64_t j0, const float* A, int64_t lda, __half* Sh, int64_t ldsh) {
+// a0: fp16 shadow of the lower triangle of 2^k A: strict lower as is, HALF the diagonal, zero
+// above (so that a diagonal tile T satisfies T + T^T = L; see k_pass_tc.cu).  With k != 0 the
+// fp32 master's lower triangle is scaled in place too (exact: powers of two; reading C10).
+__global__ void shadow_init_kernel(int64_t n, int64_t j0, float* A, int64_t lda, __half* Sh, int64_t ldsh,
+                                   const int* kexp) {
   const int64_t j = j0 + blockIdx.y;
+  const int k = kexp ? *kexp : 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     float v = 0.f;
-    if (i > j) v = A[i + j * lda];
-    else if (i == j) v = 0.5f * A[i + j * lda];
+    if (i >= j) {
+      v = A[i + j * lda];
+      if (k != 0) {
+        v = scale_pow2(v, k);
+        A[i + j * lda] = v;
+      }
+      if (i == j) v *= 0.5f;
+    }
     Sh[i + j * ldsh] = __float2half_rn(v);
   }
 }
 
-cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int64_t ldsh, cudaStream_t st) {
+cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ldsh, const int* kexp,
+                        cudaStream_t st) {
   for (int64_t j0 = 0; j0 < n; j0 += 65535) {
     const int64_t nc = std::min<int64_t>(65535, n - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 32), (unsigned)nc);
-    shadow_init_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, Sh, ldsh);
+    shadow_init_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, Sh, ldsh, kexp);
   }
   return cudaGetLastError();
 }

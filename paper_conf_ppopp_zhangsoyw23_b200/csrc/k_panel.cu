@@ -634,15 +634,17 @@ template <int B, int CPW>
 static cudaError_t launch_panel_t(PanelArgs& a, int max_ctas, cudaStream_t st) {
   constexpr size_t smem = panel_smem<B>();
   auto kern = panel_tsqr_kernel<B, CPW>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  {
+    cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    attr_set = true;
   }
   constexpr int capN = 32 * P_SN, capL = 32 * P_SL;
   const int L = (a.m <= capN) ? 1 : (a.m + capL - 1) / capL;   // 1: single node, direct QR
-  if (L > max_ctas) return cudaErrorInvalidValue;  // one CTA per leaf must be co-resident
+  a.over_capacity = 0;
+  if (L > max_ctas) {   // one CTA per leaf must be co-resident: reported through over_capacity
+    a.over_capacity = 1;
+    return cudaSuccess;
+  }
   a.arity = std::max(2, capN / a.b);
   a.nlev = 0;
   int nodes = L;
@@ -696,16 +698,14 @@ PanelWs panel_ws_sizes(int64_t m_max, int b) {
 }
 
 int panel_max_ctas(int b) {
-  int dev = 0, nsm = 0, per = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  const int nsm = current_device_sms();
   const void* k;
   size_t smem;
   if (b <= 16) { k = (const void*)panel_tsqr_kernel<16, 1>; smem = panel_smem<16>(); }
   else if (b <= 32) { k = (const void*)panel_tsqr_kernel<32, 1>; smem = panel_smem<32>(); }
   else { k = (const void*)panel_tsqr_kernel<64, 2>; smem = panel_smem<64>(); }
-  cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k, P_NW * 32, smem);
+  func_attr(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  const int per = func_blocks_per_sm(k, P_NW * 32, smem);
   return std::max(1, per) * nsm;
 }
 

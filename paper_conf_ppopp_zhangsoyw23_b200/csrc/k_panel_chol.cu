@@ -52,6 +52,7 @@ constexpr size_t PCW_BYTES = PCW_LU + sizeof(float) * (2 * 64 * 64 + 2 * 64);
 
 size_t panel_chol_ws_bytes() { return PCW_BYTES; }
 int* panel_chol_fail(void* ws) { return reinterpret_cast<int*>((char*)ws + PCW_CTL) + 3; }
+unsigned* panel_chol_declines(void* ws) { return reinterpret_cast<unsigned*>((char*)ws + PCW_CTL) + 4; }
 
 template <int B>
 struct CholSmem {
@@ -328,10 +329,11 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   // ---- zero the other parity's Gram sets and barrier counter (used by the next launch)
   {
     double* other = reinterpret_cast<double*>(ws + PCW_SETS) + (size_t)(par ^ 1u) * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
-    const int64_t tot = (int64_t)PC_NSET * PC_NCOPY * PC_SETSTRIDE;
+    // only the B x B head of each (set, copy) is ever accumulated (index p + q B)
+    const int64_t tot = (int64_t)PC_NSET * PC_NCOPY * B * B;
     const int64_t per = (tot + G - 1) / G;
     const int64_t lo = (int64_t)blockIdx.x * per, hi = std::min<int64_t>(tot, lo + per);
-    for (int64_t e = lo + threadIdx.x; e < hi; e += blockDim.x) other[e] = 0.0;
+    for (int64_t e = lo + threadIdx.x; e < hi; e += blockDim.x) other[(e / (B * B)) * PC_SETSTRIDE + e % (B * B)] = 0.0;
     if (blockIdx.x == 0 && threadIdx.x == 0) ctl[par ^ 1u] = 0u;
   }
   __syncthreads();
@@ -401,6 +403,9 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       __threadfence();
       atomicAdd(ctr, 1u);
     }
+    // Gpart is read by the bulk reduction until thread 0's wait_group: no warp may reuse it
+    // (the LU's Lcol/Urow alias it) before that
+    __syncthreads();
   };
   auto gram_read = [&](int set) {   // after the barrier: sum the copies into Gk (upper)
     const double* Gs = sets + (size_t)set * PC_NCOPY * PC_SETSTRIDE;
@@ -542,7 +547,10 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   stamp(3);
   gram_read(0);
   if (!chol(0.0)) {                    // not numerically SPD: leave the panel to TSQR
-    if (blockIdx.x == 0 && threadIdx.x == 0) *fail = 1;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      *fail = 1;
+      atomicAdd(ctl + 4, 1u);   // declines since the workspace was zeroed (sbr_test_panel_declines)
+    }
     return;
   }
   stamp(4);
@@ -587,7 +595,10 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     if (blockIdx.x == 0 || stream) racc_update(false);
   }
   if (!done) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) *fail = 1;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      *fail = 1;
+      atomicAdd(ctl + 4, 1u);   // declines since the workspace was zeroed (sbr_test_panel_declines)
+    }
     return;
   }
   stamp(9);
@@ -719,19 +730,13 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
 template <int B>
 static cudaError_t launch_chol_t(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st) {
   constexpr size_t smem = CholSmem<B>::BYTES;
-  static int per_sm = -1, nsm = 0;
-  if (per_sm < 0) {
-    cudaError_t e = cudaFuncSetAttribute(panel_chol_kernel<B, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         (int)smem);
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(panel_chol_kernel<B, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, panel_chol_kernel<B, false>, PC_THREADS, smem);
-    if (per_sm < 1) per_sm = 1;
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-  }
+  cudaError_t e = func_attr((const void*)panel_chol_kernel<B, false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)smem);
+  if (e != cudaSuccess) return e;
+  e = func_attr((const void*)panel_chol_kernel<B, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  const int per_sm = std::max(1, func_blocks_per_sm((const void*)panel_chol_kernel<B, false>, PC_THREADS, smem));
+  const int nsm = current_device_sms();
   const int cap = per_sm * nsm;
   // >= 64 rows per CTA (CTA 0 must hold the b top rows); panels beyond cap x pc_maxr rows are
   // streamed in row chunks (see the kernel)

@@ -150,7 +150,7 @@ __global__ void __launch_bounds__(256, 1)
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
     if (lane == 0) {
-      // OA tiles are read once per pass: evict_first (SBR_PASS_EXPER bit 2 = normal, ablation)
+      // OA tiles are read once per pass: evict_first (experiment knob bit 2 = normal, ablation)
       const uint64_t lpol = (exper & 4) ? l2_policy_evict_normal() : l2_policy_evict_first();
       int st = 0; uint32_t ph = 0;            // L ring
       int ws = 0; uint32_t wph = 0;           // W_I ring
@@ -213,7 +213,7 @@ __global__ void __launch_bounds__(256, 1)
         mbar_wait(&l_full[st], ph);
         tc_fence_after();
         const uint32_t lt = aL + st * Cfg::LT;
-        if (!(exper & 1))   // (exper: timing experiments only, SBR_PASS_EXPER; 0 in production)
+        if (!(exper & 1))   // (exper: timing experiments only, test knob; 0 in production)
 #pragma unroll
         for (int s = 0; s < 8; ++s) {  // X_I += L W_J : A MN-major (LBO = 16 KB between 64-row atoms)
           const uint64_t a = sdesc_sw128(lt + (s >> 2) * 8192 + (s & 3) * 2048, 16384, 1024);
@@ -341,11 +341,9 @@ template <int BN, int C, int NS>
 static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   using Cfg = PassCfg<BN, C, NS>;
   auto kern = pass_tc_kernel<BN, C, NS>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+  {
+    cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
     if (e != cudaSuccess) return e;
-    attr = true;
   }
   CUtensorMap mapL, mapW;
   cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 128);
@@ -358,7 +356,7 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
   const int64_t T = T1 - T0;
   if (T <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
-  static const int exper = getenv("SBR_PASS_EXPER") ? atoi(getenv("SBR_PASS_EXPER")) : 0;
+  const int exper = knob(KNOB_PASS_EXPER);   // timing experiments only (sbr_test_set_knob); 0 in production
   return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mapL, mapW, (int)p.r0, (int)p.M, NT, T0, T, p.b,
                     p.X, p.ldx, exper);
 }

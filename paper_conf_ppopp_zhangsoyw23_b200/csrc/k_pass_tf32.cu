@@ -342,11 +342,9 @@ int64_t pass_tf32_tiles(int64_t M) {
 cudaError_t launch_pass_tf32(const PassTf32Launch& p, cudaStream_t st) {
   if (p.b < 1 || p.b > 32) return cudaErrorInvalidValue;
   auto kern = pass_tf32_kernel;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, P3_SMEM);
+  {
+    cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, P3_SMEM);
     if (e != cudaSuccess) return e;
-    attr = true;
   }
   const int NT = (int)((p.M + 127) / 128);
   const int jstrip = p.S ? (int)std::min<int64_t>((p.sw + 127) / 128, NT) : 0;

@@ -153,11 +153,9 @@ template <int BN>
 static cudaError_t launch_nn_t(const SkinnyNN& p, cudaStream_t st) {
   using Cfg = NnCfg<BN>;
   auto kern = skinny_nn_kernel<BN>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+  {
+    cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
     if (e != cudaSuccess) return e;
-    attr = true;
   }
   CUtensorMap mA0, mA1, mB0, mB1;
   cudaError_t e;
@@ -308,11 +306,9 @@ template <int BN>
 static cudaError_t launch_tn_t(const SkinnyTN& p, cudaStream_t st) {
   using Cfg = TnCfg<BN>;
   auto kern = skinny_tn_kernel<BN>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+  {
+    cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
     if (e != cudaSuccess) return e;
-    attr = true;
   }
   if (p.K1 <= 0 || p.rows <= 0) return cudaSuccess;
   CUtensorMap mA0, mA1, mB;

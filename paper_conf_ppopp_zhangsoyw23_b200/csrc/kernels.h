@@ -35,6 +35,7 @@ struct PanelArgs {
   int64_t* trace;  // optional: CTA 0 phase timestamps (globaltimer ns), 10 entries
   const int* run_if;  // TSQR only: if non-NULL, do nothing unless *run_if != 0 (CholQR fallback)
   double orth_tol;    // CholeskyQR acceptance: max|Q^T Q - I| (fp64) <= orth_tol (0: default 1e-9)
+  int over_capacity;  // set by launch_panel: the TSQR tree needs more co-resident CTAs than exist (no launch)
   // tree (filled by launch_panel)
   int nlev, arity;
   int nodes[kPanelMaxLev];
@@ -54,6 +55,7 @@ int panel_max_ctas(int b);
 // On return the TSQR fallback must be launched with run_if = panel_chol_fail(ws).
 size_t panel_chol_ws_bytes();
 int* panel_chol_fail(void* ws);
+unsigned* panel_chol_declines(void* ws);   // count of declined CholeskyQR panels (device)
 cudaError_t launch_panel_chol(PanelArgs& a, void* ws, unsigned launch, cudaStream_t st);
 
 // ---- SIMT building blocks (fp32) ----
@@ -77,10 +79,17 @@ cudaError_t tn_small(int64_t rows, int b, const float* A, int64_t lda, const flo
 
 // ---- misc ----
 cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaStream_t st);
-cudaError_t check_finite(int64_t n, const float* A, int64_t lda, unsigned* flag, cudaStream_t st);
+// a0: flag[0] |= 1 if the lower triangle holds Inf/NaN; *kexp = k of the scale 2^k
+// (||A||_F 2^k in [2^12, 2^13)); fro2: one double of scratch
+cudaError_t prep_scale(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2, int* kexp,
+                       bool fp16_mode, cudaStream_t st);
+// 3xTF32 mode: A's lower triangle *= 2^k in place (the FP16 mode does it in shadow_init)
+cudaError_t scale_lower(int64_t n, float* A, int64_t lda, const int* kexp, cudaStream_t st);
 cudaError_t note_unhandled(const int* fail, unsigned* sticky, cudaStream_t st);
-cudaError_t extract_band(int64_t n, int b, const float* A, int64_t lda, float* AB, int64_t ldab,
-                         cudaStream_t st);
+// band out, unscaled by 2^-k (kexp may be NULL: k = 0); A's band rewritten unscaled; a non-finite
+// band entry sets flag[2] (flag may be NULL)
+cudaError_t extract_band(int64_t n, int b, float* A, int64_t lda, float* AB, int64_t ldab, const int* kexp,
+                         unsigned* flag, cudaStream_t st);
 cudaError_t mirror_lower_block(int b, float* A, int64_t lda, cudaStream_t st);
 cudaError_t lazy_small_p(int k, int b, const float* Xc, int64_t ldx, const float* WtX, int64_t ldwx,
                          const float* Yc, int64_t ldy, float* P, cudaStream_t st);
@@ -235,7 +244,10 @@ cudaError_t f32cm_to_f16rm(int64_t rows, int cols, const float* src, int64_t lds
                            cudaStream_t st);
 cudaError_t build_lazy_b(int k, int b, const __half* Yh, int64_t ldyh, int64_t c, const float* P, __half* Bl,
                          int64_t ldbl, cudaStream_t st);
-cudaError_t shadow_init(int64_t n, const float* A, int64_t lda, __half* Sh, int64_t ldsh, cudaStream_t st);
+// fp16 shadow of 2^k A (lower; half diagonal; zero upper); with k != 0 also scales A's lower
+// triangle in place (kexp may be NULL: k = 0)
+cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ldsh, const int* kexp,
+                        cudaStream_t st);
 cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
                        int64_t ldd, cudaStream_t st);
 

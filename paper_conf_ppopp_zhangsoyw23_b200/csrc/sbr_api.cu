@@ -19,6 +19,7 @@
 #include <vector>
 
 #include "../../include/sbr.h"
+#include "common.cuh"
 #include "kernels.h"
 #include "nccl_rt.h"
 
@@ -91,6 +92,13 @@ struct sbr_ctx {
   nccl::Comm comm = nullptr;
   bool force_coll = false;   // SBR_DIST_COLLECTIVES=1: issue the exchanges even with one rank (tests)
   bool tf32_tc = true;       // SBR_TF32_TC=0: 3xTF32 mode on the SIMT fp32 kernels (ablation)
+  // latched device-detected errors (§8(b)): each sbr_reduce copies its status words (flag[0..3])
+  // into a pinned slot and records an event; sbr_sync and the next calls report them
+  static constexpr int kSlots = 4;
+  unsigned* pinned = nullptr;          // kSlots x 4 words
+  cudaEvent_t slot_ev[kSlots] = {};
+  bool slot_busy[kSlots] = {};
+  int slot_next = 0;
   // sbr_test_panel_trace: per-panel CholeskyQR phase stamps of the next sbr_reduce (16 int64 per panel)
   int64_t* ptrace = nullptr;
   int ptrace_cap = 0, ptrace_used = 0;
@@ -144,6 +152,62 @@ void drain_stats(sbr_ctx* h) {
     h->ev_pool.push_back(p.e1);
   }
   h->pending.clear();
+}
+
+// status words of a finished reduction -> sbr.h code (0 if none)
+int status_of(const unsigned* w) {
+  if (w[0] || w[2]) return SBR_ERR_NONFINITE;   // non-finite input / fp16 range exceeded
+  if (w[1]) return SBR_ERR_UNSUPPORTED;          // declined CholeskyQR panel beyond the TSQR capacity
+  return SBR_OK;
+}
+
+// Report latched errors of finished reductions (wait = block until all slots complete).
+int poll_latched(sbr_ctx* h, bool wait) {
+  int rc = SBR_OK;
+  for (int i = 0; i < sbr_ctx::kSlots; ++i) {
+    if (!h->slot_busy[i]) continue;
+    const cudaError_t q = wait ? cudaEventSynchronize(h->slot_ev[i]) : cudaEventQuery(h->slot_ev[i]);
+    if (q == cudaErrorNotReady) {
+      cudaGetLastError();
+      continue;
+    }
+    h->slot_busy[i] = false;
+    const int r = status_of(h->pinned + 4 * i);
+    if (r != SBR_OK && rc == SBR_OK) {
+      rc = r;
+      if (r == SBR_ERR_UNSUPPORTED) {
+        std::lock_guard<std::mutex> lk(g_err_mu);
+        g_last_err = "a panel taller than the TSQR capacity was rank deficient for CholeskyQR";
+      }
+    }
+  }
+  return rc;
+}
+
+// Enqueue the copy of this reduction's status words into a free pinned slot.
+int latch_status(sbr_ctx* h, cudaStream_t st) {
+  if (!h->pinned) {
+    if (cudaHostAlloc((void**)&h->pinned, sizeof(unsigned) * 4 * sbr_ctx::kSlots, cudaHostAllocDefault) !=
+        cudaSuccess) {
+      cudaGetLastError();
+      return SBR_ERR_NOMEM;
+    }
+    for (int i = 0; i < sbr_ctx::kSlots; ++i) cudaEventCreateWithFlags(&h->slot_ev[i], cudaEventDisableTiming);
+  }
+  const int i = h->slot_next;
+  h->slot_next = (i + 1) % sbr_ctx::kSlots;
+  if (h->slot_busy[i]) {   // more reductions in flight than slots: the oldest must finish first
+    const int r = poll_latched(h, true);
+    if (r != SBR_OK) return r;
+  }
+  cudaError_t e = cudaMemcpyAsync(h->pinned + 4 * i, h->flag, sizeof(unsigned) * 4, cudaMemcpyDeviceToHost, st);
+  if (e == cudaSuccess) e = cudaEventRecord(h->slot_ev[i], st);
+  if (e != cudaSuccess) {
+    set_err("latch status", e);
+    return SBR_ERR_CUDA;
+  }
+  h->slot_busy[i] = true;
+  return SBR_OK;
 }
 
 #define SBR_NC(expr, what)                                             \
@@ -292,26 +356,30 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   // broadcast of Y (fp16) and W^T X.  With nranks == 1 this is exactly sbr_reduce.
   const bool lead = h->rank == 0;
   const bool dist = h->comm != nullptr && (h->nranks > 1 || h->force_coll);
+  {   // errors latched by earlier reductions on this handle are returned by the next call (§8(b))
+    const int lr = poll_latched(h, false);
+    if (lr != SBR_OK) return lr;
+  }
   if (n <= b + 1) {
     if (!lead) return SBR_OK;
     Scope sc(h, SBR_K_OTHER, 0, 0);
-    SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
+    SBR_CK(extract_band(n, b, A, lda, AB, ldab, nullptr, nullptr, st), "extract_band");
     h->launches++;
     return SBR_OK;
   }
   int rc = ensure_ws(h, n, b, nb, mode, nullptr);
   if (rc != SBR_OK) return rc;
+  // status words flag[0..3] (input non-finite, declined tall panel, non-finite band), then the
+  // a0 scan: finiteness + ||A||_F -> the FP16 mode's power-of-two scale 2^k (kexp, device)
+  unsigned* flag = h->flag;
+  double* fro2 = reinterpret_cast<double*>(h->flag + 8);
+  int* kexp = reinterpret_cast<int*>(h->flag + 10);
+  SBR_CK(cudaMemsetAsync(flag, 0, sizeof(unsigned) * 4, st), "zero status");
   {
-    Scope sc(h, SBR_K_OTHER, 2.0 * n * n, 0);
-    SBR_CK(check_finite(n, A, lda, h->flag, st), "check_finite");
-    h->launches += (n + 65534) / 65535;
+    Scope sc(h, SBR_K_OTHER, 2.0 * n * n, 2.0 * n * n);
+    SBR_CK(prep_scale(n, A, lda, flag, fro2, kexp, mode == SBR_FP16_FP32ACC, st), "prep_scale");
+    h->launches += (n + 65534) / 65535 + 1;
   }
-  unsigned flag = 0;
-  SBR_CK(cudaMemcpyAsync(&flag, h->flag, sizeof(unsigned), cudaMemcpyDeviceToHost, st), "flag D2H");
-  SBR_CK(cudaStreamSynchronize(st), "sync");
-  if (flag) return SBR_ERR_NONFINITE;
-  SBR_CK(cudaMemsetAsync(h->flag + 1, 0, sizeof(unsigned), st), "zero sticky");
-  bool unguarded = false;   // some panel ran CholeskyQR without a TSQR fallback
 
   const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
   const int64_t ldn = n;        // ld of the block buffers
@@ -321,7 +389,12 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   const bool tc32 = !tc16 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0;
   if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper)
     Scope sc(h, SBR_K_OTHER, 6.0 * n * n, 0);
-    SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, st), "shadow_init");
+    SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, kexp, st), "shadow_init");
+    h->launches += (n + 65534) / 65535;
+  }
+  if (!tc16) {  // a0 in 3xTF32 mode: the master scaled in place (FP16: inside shadow_init)
+    Scope sc(h, SBR_K_OTHER, 8.0 * n * n / 2, 0);
+    SBR_CK(scale_lower(n, A, lda, kexp, st), "scale_lower");
     h->launches += (n + 65534) / 65535;
   }
   if (tc16) {  // fp16 W copies: pad columns (b < BN) must read as zero in the pass
@@ -444,8 +517,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         if (h->ptrace && h->ptrace_used < h->ptrace_cap) pa.trace = h->ptrace + 16 * (int64_t)h->ptrace_used++;
         bool chol = false;
         if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
-          const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
+          const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches, st);
           if (ce == cudaSuccess) {
+            h->chol_launches++;   // the Gram-set / barrier parity advances only with a launched kernel
             pa.run_if = h->pfail;
             h->launches += 1;
             chol = true;
@@ -455,22 +529,19 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         }
         pa.trace = nullptr;   // the phase trace is CholeskyQR's (the TSQR fallback has its own stamps)
         const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
-        if (te == cudaErrorInvalidValue && chol) {
+        SBR_CK(te, "panel");
+        if (pa.over_capacity && chol) {
           // panel taller than the TSQR tree can hold (one co-resident CTA per 256-row leaf): no
           // fallback; a declined CholeskyQR is recorded and reported after the reduction
-          cudaGetLastError();
           SBR_CK(note_unhandled(h->pfail, h->flag + 1, st), "note_unhandled");
-          unguarded = true;
-        } else if (te == cudaErrorInvalidValue) {
-          cudaGetLastError();
+        } else if (pa.over_capacity) {
           std::lock_guard<std::mutex> lk(g_err_mu);
           g_last_err = "panel of " + std::to_string(m) + " x " + std::to_string(b) +
                        " exceeds the panel kernels' capacity (CholeskyQR: 148 CTAs x rows in smem)";
           return SBR_ERR_UNSUPPORTED;
         } else {
-          SBR_CK(te, "panel");
+          h->launches += 1;
         }
-        h->launches += 1;
       }
       if (tc16) {
         if (t >= 1 && lead) {
@@ -713,20 +784,10 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   }
   if (lead) {
     Scope sc(h, SBR_K_OTHER, 8.0 * (b + 1) * n, 0);
-    SBR_CK(extract_band(n, b, A, lda, AB, ldab, st), "extract_band");
+    SBR_CK(extract_band(n, b, A, lda, AB, ldab, kexp, flag, st), "extract_band");
     h->launches += 1;
   }
-  if (unguarded) {   // one 4-byte read at the end, only for panels beyond the TSQR capacity
-    unsigned sticky = 0;
-    SBR_CK(cudaMemcpyAsync(&sticky, h->flag + 1, sizeof(unsigned), cudaMemcpyDeviceToHost, st), "sticky D2H");
-    SBR_CK(cudaStreamSynchronize(st), "sync");
-    if (sticky) {
-      std::lock_guard<std::mutex> lk(g_err_mu);
-      g_last_err = "a panel taller than the TSQR capacity was rank deficient for CholeskyQR";
-      return SBR_ERR_UNSUPPORTED;
-    }
-  }
-  return SBR_OK;
+  return latch_status(h, st);   // errors found on the device are reported by sbr_sync / the next call
 }
 
 }  // namespace
@@ -861,6 +922,9 @@ int sbr_destroy(sbr_handle_t h) {
   if (h->e2e) cudaFree(h->e2e);
   if (h->fq) cudaFree(h->fq);
   if (h->ptrace) cudaFree(h->ptrace);
+  if (h->pinned) cudaFreeHost(h->pinned);
+  for (auto e : h->slot_ev)
+    if (e) cudaEventDestroy(e);
   delete h;
   return SBR_OK;
 }
@@ -929,7 +993,7 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A
            "D2H W");
   }
   SBR_CK(cudaStreamSynchronize(st), "sync");
-  return SBR_OK;
+  return poll_latched(h, true);   // the call returns after the results are on the host: report now
 }
 
 int sbr_get_unique_id(void* id) {
@@ -999,7 +1063,7 @@ int sbr_nranks(sbr_handle_t h) { return h ? h->nranks : -1; }
 int sbr_sync(sbr_handle_t h) {
   if (!h) return -1;
   SBR_CK(cudaStreamSynchronize(h->stream), "sync");
-  return SBR_OK;
+  return poll_latched(h, true);
 }
 
 const char* sbr_status_string(int status) {
@@ -1125,7 +1189,7 @@ int sbr_test_pass_fp16_part(sbr_handle_t h, int64_t M, int b, int rank, int nran
   const int64_t ldsh = (M + 7) / 8 * 8;
   DevBuf sh(sizeof(__half) * ldsh * M), wh(sizeof(__half) * ldwh * 64);
   if (!sh.p || !wh.p) return SBR_ERR_NOMEM;
-  SBR_CK(shadow_init(M, OA, ldoa, (__half*)sh.p, ldsh, st), "shadow");
+  SBR_CK(shadow_init(M, const_cast<float*>(OA), ldoa, (__half*)sh.p, ldsh, nullptr, st), "shadow");   // k = 0: read only
   SBR_CK(to_half_cm(M, b, pass_bn(b), W, ldw, (__half*)wh.p, ldwh, st), "W->fp16");
   SBR_CK(zero_matrix(M, b, X, ldx, st), "zero X");
   PassLaunch pl{};
@@ -1352,8 +1416,9 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
   pa.trace = trace_host ? (int64_t*)tr.p : nullptr;
   bool chol = false;
   if (h->panel_mode == 0 && m > 512) {
-    const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches++, st);
+    const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches, st);
     if (ce == cudaSuccess) {
+      h->chol_launches++;
       pa.run_if = h->pfail;
       chol = true;
     } else if (ce != cudaErrorNotSupported) {
@@ -1361,14 +1426,13 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
     }
   }
   const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
-  if (te == cudaErrorInvalidValue && chol) {   // taller than the TSQR tree: CholeskyQR only (as sbr_reduce)
-    cudaGetLastError();
+  SBR_CK(te, "panel");
+  if (pa.over_capacity && !chol) return SBR_ERR_UNSUPPORTED;
+  if (pa.over_capacity && chol) {   // taller than the TSQR tree: CholeskyQR only (as sbr_reduce)
     int failed = 0;
     SBR_CK(cudaMemcpyAsync(&failed, h->pfail, sizeof(int), cudaMemcpyDeviceToHost, st), "fail D2H");
     SBR_CK(cudaStreamSynchronize(st), "sync");
     if (failed) return SBR_ERR_UNSUPPORTED;
-  } else {
-    SBR_CK(te, "panel");
   }
   if (trace_host) {
     SBR_CK(cudaMemcpyAsync(trace_host, tr.p, sizeof(int64_t) * 16, cudaMemcpyDeviceToHost, st), "trace D2H");
@@ -1399,6 +1463,29 @@ extern "C" int sbr_test_panel_trace(sbr_handle_t h, int cap, int64_t* host, int*
       SBR_CK(cudaMemcpy(host, h->ptrace, sizeof(int64_t) * 16 * (size_t)h->ptrace_used, cudaMemcpyDeviceToHost),
              "trace D2H");
   }
+  return SBR_OK;
+}
+
+// Declined CholeskyQR panels (TSQR fallback taken) since the last call with reset != 0.
+extern "C" int sbr_test_panel_declines(sbr_handle_t h, int reset, int64_t* count) {
+  if (!h) return -1;
+  if (!count) return -3;
+  *count = 0;
+  if (!h->chol_ws) return SBR_OK;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  unsigned v = 0;
+  SBR_CK(cudaMemcpyAsync(&v, panel_chol_declines(h->chol_ws), sizeof(unsigned), cudaMemcpyDeviceToHost, h->stream),
+         "declines D2H");
+  SBR_CK(cudaStreamSynchronize(h->stream), "sync");
+  *count = v;
+  if (reset) SBR_CK(cudaMemsetAsync(panel_chol_declines(h->chol_ws), 0, sizeof(unsigned), h->stream), "reset");
+  return SBR_OK;
+}
+
+namespace sbr { void set_knob(int k, int v); }
+extern "C" int sbr_test_set_knob(int k, int value) {
+  if (k < 0 || k >= sbr::KNOB_COUNT) return -1;
+  sbr::set_knob(k, value);
   return SBR_OK;
 }
 

@@ -95,9 +95,11 @@ def test_trivial_and_error_cases():
     bad = torch.from_numpy(a_host).cuda()
     bad[3, 2] = float("nan")      # both triangles (only the lower one is referenced)
     bad[2, 3] = float("nan")
+    h.reduce(bad, 2, 4)                 # no host sync: the device latches the error ...
     with pytest.raises(SbrError) as ei:
-        h.reduce(bad, 2, 4)
+        h.sync()                        # ... and sbr_sync reports it (include/sbr.h)
     assert ei.value.status == 1
+    h.sync()                            # reported once
     with pytest.raises(SbrError) as ei:
         h.reduce(torch.from_numpy(a_host).cuda(), 2, 3)   # nb % b != 0
     assert ei.value.status == -5

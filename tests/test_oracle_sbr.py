@@ -186,3 +186,22 @@ def test_blocks_from_output_roundtrip():
         w_out[c0 + b:, c0:c0 + k] = wj
     blocks = metrics.blocks_from_output(a_out, w_out, n, b, nb)
     np.testing.assert_allclose(metrics.q_from_blocks(n, b, blocks), w["Q"], atol=1e-13)
+
+
+@needs_sy2sb
+def test_only_lower_triangle_referenced():
+    """Reading C14 pinned against LAPACK: dsytrd_sy2sb(UPLO='L') reads only the lower triangle,
+    so an input with garbage above the diagonal must give the same band in the oracle as in
+    LAPACK -- a mirrored upper triangle (or a transposed read) would fail."""
+    n, b = 90, 6
+    a = workloads.random_symmetric(n, 1234).astype(np.float64)
+    junk = a.copy()
+    iu = np.triu_indices(n, 1)
+    junk[iu] = np.random.default_rng(5).standard_normal(len(iu[0])) * 100.0
+    o = sbr.sbr_unblocked(junk, b)
+    ab, _, _ = sytrd_sy2sb(junk, b)
+    ref = sbr.lapack_band_to_dense(ab)
+    assert np.abs(o["B"] - ref).max() <= 1e-12 * np.linalg.norm(np.tril(a))
+    w = sbr.sbr_wy_blocked(junk, b, 18)
+    assert np.abs(w["B"] - ref).max() <= 1e-12 * np.linalg.norm(np.tril(a))
+    np.testing.assert_array_equal(sbr.symmetrize_lower(junk), sbr.symmetrize_lower(np.tril(junk)))

@@ -36,3 +36,20 @@ def test_prescribed_spectrum():
         assert np.isclose(lam.max(), 1.0) and np.isclose(lam.min(), 1e-3)
         got = np.linalg.eigvalsh(a.astype(np.float64))
         assert np.max(np.abs(np.sort(got) - np.sort(lam))) < 1e-6
+
+
+def test_hadamard_prescribed_spectrum_cpu():
+    """Config-5 recipe (randomised Hadamard Q) on CPU at small n: bit-symmetric,
+    dense, spectrum = the prescribed one to fp32 accuracy."""
+    import numpy as np
+
+    import workloads
+
+    n = 512
+    a, desc = workloads.prescribed_spectrum_device(n, "geo", 1e5, 11, a_device="cpu", haar_max=16)
+    a = a.numpy()
+    assert "Hadamard" in desc
+    np.testing.assert_array_equal(a, a.T)
+    assert np.count_nonzero(a) > 0.99 * n * n
+    lam = np.linalg.eigvalsh(a.astype(np.float64))
+    assert np.max(np.abs(lam - np.sort(workloads.spectrum(n, "geo", 1e5)))) <= 1e-6

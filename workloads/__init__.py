@@ -37,6 +37,8 @@ __all__ = [
     "spectrum",
     "prescribed_spectrum",
     "SPECTRUM_KINDS",
+    "haar_orthogonal",
+    "prescribed_spectrum_device",
 ]
 
 
@@ -141,3 +143,55 @@ def prescribed_spectrum(n: int, kind: str = "geo", kappa: float = 1e5, seed: int
     low = np.tril(a)
     a = low + np.tril(low, -1).T
     return a.astype(np.float32), lam
+
+
+def prescribed_spectrum_device(n: int, kind: str = "geo", kappa: float = 1e5, seed: int = BASE_SEED,
+                               a_device: str = "cuda:0", haar_max: int = 16384):
+    """Prescribed-spectrum input on the device (torch fp32 (n, n), bit-symmetric) and a one-line
+    description.  n <= haar_max: the host recipe ``prescribed_spectrum`` (Haar Q).  Larger n
+    (config 5): Q = H D1 H D2 H D3 / n^{3/2} -- H the n x n Walsh-Hadamard matrix
+    (fast transform), D_i seeded random +-1 diagonals -- so A = Q diag(lam) Q^T is dense, exactly
+    orthogonally similar to diag(lam) in exact arithmetic, and built in O(n^2 log n) on the GPU
+    (fp32; n a power of two).  Input generation only: none of the method's arithmetic."""
+    import torch
+
+    if n <= haar_max:
+        a, _ = prescribed_spectrum(n, kind, kappa, seed)
+        return torch.from_numpy(a).to(a_device), f"prescribed spectrum SVD_{kind} kappa={kappa:g}, Haar Q (seed {seed})"
+    if n & (n - 1):
+        raise ValueError("the Hadamard recipe needs n a power of two")
+    lam = torch.from_numpy(spectrum(n, kind, kappa)).to(device=a_device, dtype=torch.float32)
+    g = torch.Generator(device="cpu").manual_seed(seed)
+    d = [(torch.randint(0, 2, (n,), generator=g).to(a_device, torch.float32) * 2 - 1) for _ in range(3)]
+
+    def fwht_rows_(x):   # x (n, m): x <- H x (unnormalised), in place, column block by block
+        h = 1
+        while h < n:
+            v = x.view(n // (2 * h), 2, h, -1)
+            a = v[:, 0].clone()
+            v[:, 0].add_(v[:, 1])
+            v[:, 1].neg_().add_(a)
+            del a
+            h *= 2
+        return x
+
+    def apply_q_(x):     # x <- Q x, column blocks of 4096 to bound the temporaries
+        for c0 in range(0, x.shape[1], 4096):
+            blk = x[:, c0:c0 + 4096]
+            t = blk.contiguous()
+            for di in (d[2], d[1], d[0]):
+                t.mul_(di[:, None])
+                fwht_rows_(t)
+            t.mul_(float(n) ** -1.5)
+            blk.copy_(t)
+        return x
+
+    t = torch.diag(lam)                  # T = Q diag(lam)
+    apply_q_(t)
+    a = t.t().contiguous()               # diag(lam) Q^T
+    del t
+    apply_q_(a)                          # A = Q diag(lam) Q^T
+    low = torch.tril(a)
+    a = low + torch.tril(low, -1).t()
+    return a.contiguous(), (f"prescribed spectrum SVD_{kind} kappa={kappa:g}, randomised Hadamard "
+                            f"Q = H D1 H D2 H D3 / n^1.5 (seed {seed})")
