@@ -52,7 +52,7 @@ def parse():
     p.add_argument("--profile-steps", type=int, default=2)
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--cpu-sample-s", type=float, default=15.0)
-    p.add_argument("--lapack-n", type=int, default=4096,
+    p.add_argument("--lapack-n", type=int, default=16384,
                    help="n of the LAPACK ssytrd_sy2sb/dsytrd_sy2sb host baseline (0: skip)")
     return p.parse_args()
 

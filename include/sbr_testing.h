@@ -40,11 +40,12 @@ int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_t ldp, float* Y, float* W, int64_t ldyw,
                    int64_t* trace);
 
-/* Diagnostic: per-panel CholeskyQR phase stamps inside sbr_reduce.  cap > 0 arms recording
- * for the next cap panels (device buffer owned by the handle, 16 int64 globaltimer stamps in
- * ns per panel, CTA 0's view, stamp 0 taken before the PDL wait); host != NULL copies the
- * stamps recorded so far (count * 16 int64) after synchronising the handle's stream and
- * stores the panel count in *count (NULL count with non-NULL host: -4). */
+/* Diagnostic: per-panel phase stamps inside sbr_reduce (the CholeskyQR panel kernel, or the
+ * fused chain kernel of the FP16 mode).  cap > 0 arms recording for the next cap panels
+ * (device buffer owned by the handle, 32 int64 globaltimer slots in ns per panel, CTA 0's
+ * view, stamp 0 taken before the PDL wait); host != NULL copies the stamps recorded so far
+ * (count * 32 int64) after synchronising the handle's stream and stores the panel count in
+ * *count (NULL count with non-NULL host: -4). */
 int sbr_test_panel_trace(sbr_handle_t h, int cap, int64_t* host, int* count);
 
 /* Same as sbr_test_pass_fp16 but only the share of `rank` of `nranks` (the tiles

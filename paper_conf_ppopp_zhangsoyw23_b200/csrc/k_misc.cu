@@ -92,6 +92,10 @@ cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaS
   return cudaGetLastError();
 }
 
+// kexp sentinel: the input held Inf/NaN; the lower triangle is zeroed instead of scaled, so the
+// reduction that follows runs on finite data (its outputs are invalid; the error is latched)
+constexpr int kScaleZero = -(1 << 30);
+
 // a0 scan (reading C10): finiteness of the referenced lower triangle (flag[0] |= 1) and
 // ||A||_F^2 in fp64 (off-diagonal entries twice), one fp64 atomic per block.
 __global__ void prep_scan_kernel(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2) {
@@ -127,6 +131,10 @@ __global__ void prep_scan_kernel(int64_t n, const float* A, int64_t lda, unsigne
 __global__ void choose_scale_kernel(const double* fro2, const unsigned* flag, int fp16_mode, int* kexp) {
   int k = 0;
   const double f2 = *fro2;
+  if (flag[0]) {   // non-finite input: the reduction runs on zeros (error latched, outputs invalid)
+    *kexp = kScaleZero;
+    return;
+  }
   if (!flag[0] && f2 > 0.0 && isfinite(f2)) {   // both modes (fp16_mode kept for the record)
     int e = 0;
     frexp(sqrt(f2), &e);   // ||A||_F in [2^(e-1), 2^e)
@@ -161,7 +169,7 @@ __global__ void scale_lower_kernel(int64_t n, int64_t j0, float* A, int64_t lda,
   if (k == 0) return;
   const int64_t j = j0 + blockIdx.y;
   for (int64_t i = j + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
-    A[i + j * lda] = scale_pow2(A[i + j * lda], k);
+    A[i + j * lda] = k == kScaleZero ? 0.f : scale_pow2(A[i + j * lda], k);
 }
 
 cudaError_t scale_lower(int64_t n, float* A, int64_t lda, const int* kexp, cudaStream_t st) {
@@ -191,7 +199,7 @@ __global__ void extract_band_kernel(int64_t n, int b, float* A, int64_t lda, flo
                                     const int* kexp, unsigned* flag) {
   const int64_t j = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
   const int d = threadIdx.x;
-  const int k = kexp ? *kexp : 0;
+  const int k = (kexp && *kexp != kScaleZero) ? *kexp : 0;
   bool bad = false;
   if (j < n && d <= b) {
     float v = 0.f;
@@ -277,7 +285,7 @@ __global__ void shadow_init_kernel(int64_t n, int64_t j0, float* A, int64_t lda,
     if (i >= j) {
       v = A[i + j * lda];
       if (k != 0) {
-        v = scale_pow2(v, k);
+        v = k == kScaleZero ? 0.f : scale_pow2(v, k);
         A[i + j * lda] = v;
       }
       if (i == j) v *= 0.5f;

@@ -239,6 +239,31 @@ cudaError_t launch_kxb(const KxbArgs& a, cudaStream_t st);
 cudaError_t launch_postpass(int64_t M, int b, const float* X, int64_t ldx, const float* W, int64_t ldw, __half* Xh,
                             int64_t ldxh, float* WtXtt, int64_t ldwtx, cudaStream_t st);
 
+// The fused per-panel chain of the FP16 mode (k_chain_fused.cu): ONE cooperative launch per
+// panel t does the previous pass's tail (Xh, W^T X diagonal block), the lazy update, the panel
+// QR (CholeskyQR + reconstruction, Householder fallback), and the W merge.  b = 32 only.
+struct ChainFusedLaunch {
+  int t, k;                        // panel index in the block, k = t b
+  int64_t M, tb;                   // block-local order, t b
+  float* A; int64_t lda, r0;       // master, OA origin r0
+  float* Yb; int64_t ldy;          // block Y fp32 (OA rows)
+  float* Wt; int64_t ldw;          // this panel's W columns (OA rows)
+  const float* Xb; int64_t ldx;    // X (M x p b)
+  __half* Xh;                      // fp16 row-major X (ld ldk)
+  float* WtX; int64_t ldwx;
+  float* Gf; float* Hf;            // k x 32 fp32 scratch each
+  __half* Ph; __half* Yh; __half* Wrh; int64_t ldk;
+  __half* Wh; int64_t ldwh;        // fp16 column-major W_t (pass operand)
+  void* ws; unsigned launch;       // chain_fused_ws_bytes(), zeroed once; launch counter (parity)
+  unsigned* declines;
+  double orth_tol;
+  int grid;                        // CTAs (= SMs; all co-resident)
+  int64_t* trace;                  // optional phase stamps (16 int64, CTA 0)
+};
+size_t chain_fused_ws_bytes();
+bool chain_fused_supported(int b, int64_t M, int num_sms);
+cudaError_t launch_chain_fused(const ChainFusedLaunch& L, cudaStream_t st);
+
 // fp16 conversions
 cudaError_t f32cm_to_f16rm(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd,
                            cudaStream_t st);

@@ -70,6 +70,9 @@ struct sbr_ctx {
   float* GH = nullptr;     // per-block G_t / H_t (k x b, ld nb, panel t at offset t*nb*b), zeroed per block
   __half* Ph = nullptr;    // fp16 P^T (b x k, row-major) of the lazy update
   void* chol_ws = nullptr;  // CholeskyQR panel workspace (Gram sets, barrier, LU), zeroed at allocation
+  void* fused_ws = nullptr; // fused chain kernel workspace (two launch parities), zeroed at allocation
+  unsigned fused_launches = 0;
+  bool fused = false;       // SBR_FUSED=1: the fused per-panel chain kernel (k_chain_fused.cu)
   int* pfail = nullptr;
   unsigned chol_launches = 0;
   int panel_mode = 0;      // 0: CholeskyQR3 + TSQR fallback, 1: TSQR only (SBR_PANEL=tsqr)
@@ -258,7 +261,8 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
                oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take(panel_chol_ws_bytes() / sizeof(float) + 64),
-               oGH = take((size_t)2 * nb * nb), oPh = take((size_t)64 * ldk / 2 + 8);
+               oGH = take((size_t)2 * nb * nb), oPh = take((size_t)64 * ldk / 2 + 8),
+               oFz = take(chain_fused_ws_bytes() / sizeof(float) + 64);
   const int64_t tlo = (nb + 31) / 32 * 32, ldts = 2 * tlo, ldws = (M + 3) / 4 * 4;
   size_t oYS = 0, oZS = 0, oGS = 0, oWS = 0;
   if (mode == SBR_3XTF32) {
@@ -322,6 +326,9 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->WS = mode == SBR_3XTF32 ? (float*)(base + oWS) : nullptr;
   h->pfail = panel_chol_fail(h->chol_ws);
   if (cudaMemset(h->chol_ws, 0, panel_chol_ws_bytes()) != cudaSuccess) return SBR_ERR_CUDA;
+  h->fused_ws = base + oFz;
+  h->fused_launches = 0;
+  if (cudaMemset(h->fused_ws, 0, chain_fused_ws_bytes()) != cudaSuccess) return SBR_ERR_CUDA;
   h->ldbl = 2 * ldk + 128;
   h->ldwh = ldwh;
   h->ldsh = ldsh;
@@ -344,6 +351,8 @@ int validate(sbr_ctx* h, int mode, int64_t n, int b, int nb, const float* A, int
   if (W && ldw < n) return -11;
   return SBR_OK;
 }
+
+bool panel_mode_default(const sbr_ctx* h) { return h->panel_mode == 0; }
 
 // Algorithm 1 on device buffers (arguments already validated).
 int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB, int64_t ldab,
@@ -383,10 +392,14 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
 
   const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
   const int64_t ldn = n;        // ld of the block buffers
-  const bool tc16 = (mode == SBR_FP16_FP32ACC);  // tcgen05 kind::f16 path
+  // the TMA-fed tensor-core kernels need 16-byte aligned tile origins (OA origin r0 = c0 + b):
+  // FP16 operands need b, nb multiples of 8, fp32 (3xTF32) multiples of 4; other (b, nb) run on
+  // the fp32 SIMT kernels (more accurate than either mode's operands)
+  const bool tc16 = (mode == SBR_FP16_FP32ACC) && b % 8 == 0 && nb % 8 == 0;  // tcgen05 kind::f16 path
   // 3xTF32 on tcgen05 kind::tf32 (pass + Z + SYR2K); the SIMT fp32 kernels remain for A that
   // TMA cannot address (lda % 4 != 0) and for the SBR_TF32_TC=0 ablation
-  const bool tc32 = !tc16 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0;
+  const bool tc32 = mode == SBR_3XTF32 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0 && b % 4 == 0 &&
+                    nb % 4 == 0;
   if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper)
     Scope sc(h, SBR_K_OTHER, 6.0 * n * n, 0);
     SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, kexp, st), "shadow_init");
@@ -421,7 +434,82 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       SBR_CK(cudaMemsetAsync(h->WtX, 0, sizeof(float) * nb * nb, st), "zero WtX");
       SBR_CK(cudaMemsetAsync(h->GH, 0, sizeof(float) * 2 * nb * nb, st), "zero G/H");
     }
-    for (int t = 0; t < p; ++t) {
+    // fused FP16 chain (k_chain_fused.cu): one cooperative launch per panel + the pass
+    const bool fused = tc16 && h->fused && !dist && panel_mode_default(h) && nb <= 1024 &&
+                       chain_fused_supported(b, M, h->nsm);
+    for (int t = 0; fused && t < p; ++t) {
+      const int64_t tb = (int64_t)t * b;
+      float* Wt = Wb + tb * ldwb;
+      {
+        Scope sc(h, SBR_K_PANEL, 4.0 * (M - tb) * b * 4 + (t ? 8.0 * M * b + 4.0 * (M - tb) * t * b * 5 : 0),
+                 4.0 * (M - tb) * b * b * 2 + (t ? 10.0 * M * t * b * b : 0));
+        ChainFusedLaunch L{};
+        L.t = t;
+        L.k = t * b;
+        L.M = M;
+        L.tb = tb;
+        L.A = A;
+        L.lda = lda;
+        L.r0 = r0;
+        L.Yb = h->Yb;
+        L.ldy = ldn;
+        L.Wt = Wt;
+        L.ldw = ldwb;
+        L.Xb = h->Xb;
+        L.ldx = M;
+        L.Xh = h->Xh;
+        L.WtX = h->WtX;
+        L.ldwx = nb;
+        L.Gf = h->GH;
+        L.Hf = h->GH + (size_t)nb * nb;
+        L.Ph = h->Ph;
+        L.Yh = h->Yh;
+        L.Wrh = h->Wrh;
+        L.ldk = h->ldk;
+        L.Wh = h->Wh;
+        L.ldwh = h->ldwh;
+        L.ws = h->fused_ws;
+        L.launch = h->fused_launches;
+        L.declines = panel_chol_declines(h->chol_ws);
+        L.orth_tol = 1e-6;
+        L.grid = h->nsm;
+        if (h->ptrace && h->ptrace_used < h->ptrace_cap) L.trace = h->ptrace + 32 * (int64_t)h->ptrace_used++;
+        const cudaError_t fe = launch_chain_fused(L, st);
+        if (fe != cudaSuccess) {   // the parity chain is broken: re-zero the workspace
+          cudaGetLastError();
+          cudaMemsetAsync(h->fused_ws, 0, chain_fused_ws_bytes(), st);
+          h->fused_launches = 0;
+          SBR_CK(fe, "chain_fused");
+        }
+        h->fused_launches++;
+        h->launches += 1;
+      }
+      {  // ---- a4: pass X_t = OA W_t
+        Scope sc(h, SBR_K_PASS, (1.0 * M * M + 6.0 * M * b), 2.0 * M * M * b);
+        PassLaunch pl{};
+        pl.shadow = h->Sh;
+        pl.n = n;
+        pl.ld_shadow = h->ldsh;
+        pl.Wh = h->Wh;
+        pl.M = M;
+        pl.ld_wh = h->ldwh;
+        pl.r0 = r0;
+        pl.b = b;
+        pl.X = h->Xb + tb * M;
+        pl.ldx = M;
+        pl.num_sms = h->nsm;
+        pl.seg_rows = 8;
+        SBR_CK(launch_pass_tc(pl, st), "pass_tc");
+        h->launches += 1;
+      }
+      if (t == p - 1) {  // the last panel's pass tail (the next fused launch does it otherwise)
+        Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
+        SBR_CK(launch_postpass(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb, st),
+               "postpass");
+        h->launches += 1;
+      }
+    }
+    for (int t = 0; !fused && t < p; ++t) {
       const int64_t g = c0 + (int64_t)t * b;
       const int64_t tb = (int64_t)t * b;
       const int64_t m = M - tb;
@@ -514,7 +602,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         // mode's operands -- FP16 mode rounds every GEMM operand to fp16 (u = 4.9e-4), 3xTF32 keeps
         // fp32 (u = 6e-8)
         pa.orth_tol = tc16 ? 1e-6 : 1e-8;
-        if (h->ptrace && h->ptrace_used < h->ptrace_cap) pa.trace = h->ptrace + 16 * (int64_t)h->ptrace_used++;
+        if (h->ptrace && h->ptrace_used < h->ptrace_cap) pa.trace = h->ptrace + 32 * (int64_t)h->ptrace_used++;
         bool chol = false;
         if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
           const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches, st);
@@ -811,6 +899,8 @@ int sbr_create(sbr_handle_t* out, int device, void* stream) {
   if (pm && strcmp(pm, "tsqr") == 0) h->panel_mode = 1;
   const char* tt = getenv("SBR_TF32_TC");  // "0": 3xTF32 mode on the SIMT fp32 kernels (ablation)
   if (tt && strcmp(tt, "0") == 0) h->tf32_tc = false;
+  const char* fz = getenv("SBR_FUSED");    // "1": the fused FP16 chain kernel, "0": the per-kernel chain
+  if (fz) h->fused = strcmp(fz, "1") == 0;
   *out = h;
   return SBR_OK;
 }
@@ -1450,8 +1540,8 @@ extern "C" int sbr_test_panel_trace(sbr_handle_t h, int cap, int64_t* host, int*
   if (cap > 0) {
     if (h->ptrace) cudaFree(h->ptrace);
     h->ptrace = nullptr;
-    SBR_CK(cudaMalloc(&h->ptrace, sizeof(int64_t) * 16 * (size_t)cap), "trace alloc");
-    SBR_CK(cudaMemsetAsync(h->ptrace, 0, sizeof(int64_t) * 16 * (size_t)cap, h->stream), "trace memset");
+    SBR_CK(cudaMalloc(&h->ptrace, sizeof(int64_t) * 32 * (size_t)cap), "trace alloc");
+    SBR_CK(cudaMemsetAsync(h->ptrace, 0, sizeof(int64_t) * 32 * (size_t)cap, h->stream), "trace memset");
     h->ptrace_cap = cap;
     h->ptrace_used = 0;
   }
@@ -1460,7 +1550,7 @@ extern "C" int sbr_test_panel_trace(sbr_handle_t h, int cap, int64_t* host, int*
     SBR_CK(cudaStreamSynchronize(h->stream), "sync");
     *count = h->ptrace_used;
     if (h->ptrace_used > 0)
-      SBR_CK(cudaMemcpy(host, h->ptrace, sizeof(int64_t) * 16 * (size_t)h->ptrace_used, cudaMemcpyDeviceToHost),
+      SBR_CK(cudaMemcpy(host, h->ptrace, sizeof(int64_t) * 32 * (size_t)h->ptrace_used, cudaMemcpyDeviceToHost),
              "trace D2H");
   }
   return SBR_OK;

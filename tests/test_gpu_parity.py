@@ -86,16 +86,16 @@ def test_trivial_and_error_cases():
     from paper_conf_ppopp_zhangsoyw23_b200 import SbrError
 
     h = sbr.Handle(0)
-    a_host = workloads.random_symmetric(10, 3)
+    a_host = workloads.random_symmetric(40, 3)
     a = torch.from_numpy(a_host).cuda()
-    ab, _ = h.reduce(a, 9, 9, mode="fp16")          # n <= b+1: AB = band of A
+    ab, _ = h.reduce(a, 39, 39, mode="fp16")        # n <= b+1: AB = band of A
     torch.cuda.synchronize()
     got = sbr.band_to_dense(ab.double()).cpu().numpy()
-    np.testing.assert_array_equal(got, osbr.band_part(a_host.astype(np.float64), 9))
+    np.testing.assert_array_equal(got, osbr.band_part(a_host.astype(np.float64), 39))
     bad = torch.from_numpy(a_host).cuda()
     bad[3, 2] = float("nan")      # both triangles (only the lower one is referenced)
     bad[2, 3] = float("nan")
-    h.reduce(bad, 2, 4)                 # no host sync: the device latches the error ...
+    h.reduce(bad, 8, 16)                # no host sync: the device latches the error ...
     with pytest.raises(SbrError) as ei:
         h.sync()                        # ... and sbr_sync reports it (include/sbr.h)
     assert ei.value.status == 1

@@ -23,9 +23,9 @@ lib = _lib.lib()
 _lib.check(lib.sbr_test_panel_trace(h._h, npan + 8, None, None), "arm")
 A = A0.clone(); torch.cuda.synchronize()
 h.reduce(A, b, nb, mode="fp16")
-buf = (ctypes.c_int64 * (16 * (npan + 8)))(); cnt = ctypes.c_int(0)
+buf = (ctypes.c_int64 * (32 * (npan + 8)))(); cnt = ctypes.c_int(0)
 _lib.check(lib.sbr_test_panel_trace(h._h, 0, buf, ctypes.byref(cnt)), "read")
-T = np.frombuffer(buf, dtype=np.int64)[: 16 * cnt.value].reshape(cnt.value, 16)[:, :12].astype(np.float64)
+T = np.frombuffer(buf, dtype=np.int64)[: 32 * cnt.value].reshape(cnt.value, 32)[:, :12].astype(np.float64)
 print(f"n={n}: {cnt.value} CholeskyQR panels traced")
 rel = (T - T[:, :1]) / 1e3
 rel[T == 0] = np.nan
