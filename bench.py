@@ -9,10 +9,12 @@ over one synthetic n x n input resident in HBM.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 
-One process per GPU (torchrun for N>1).  N>1 reduces ONE matrix across the ranks with
-sbr_reduce_dist (strong scaling, "scaling": "strong"): the per-panel pass is sharded by
-lower tiles with an NCCL broadcast of W_t and all-reduce of X_t per panel (DESIGN.md
-"Multi-GPU"); every rank times its own steps and the max over ranks is reported.
+One process per GPU (torchrun for N>1; a plain `--gpus N` re-launches itself under
+torch.distributed.run).  N>1 reduces ONE matrix across the ranks with sbr_reduce_dist (strong
+scaling, "scaling": "strong"): 1D block-cyclic nb-column blocks, the owner of each block
+factors its panels and NCCL-broadcasts W_t, every rank streams the pass tiles and applies the
+SYR2K on its own columns; every rank times its own steps and the max
+over ranks is reported.
 ``--impl reference`` times the CPU oracle (this tier has no reference implementation; the
 oracle is the reference arm).
 """
@@ -285,8 +287,21 @@ def run_reference(args, rank, world):
     print(json.dumps(line), flush=True)
 
 
+def respawn_distributed(args):
+    """`python bench.py --gpus N` without a torchrun environment: re-launch under
+    torch.distributed.run with N local ranks (127.0.0.1) and exit with its status."""
+    import subprocess
+
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", os.environ.get("SBR_BENCH_PORT", "29517"),
+           os.path.abspath(__file__)] + sys.argv[1:]
+    sys.exit(subprocess.call(cmd))
+
+
 def main():
     args = parse()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        respawn_distributed(args)
     rank, world, local = dist_setup()
     if args.impl == "reference":
         run_reference(args, rank, world)
@@ -320,14 +335,18 @@ def main():
         input_desc = f"random symmetric U[-1,1) (seed {seed})"
     else:   # prescribed spectrum, SVD_Geo kappa = 1e5: Haar Q (host) or randomised Hadamard Q (device)
         pristine, input_desc = workloads.prescribed_spectrum_device(n, "geo", 1e5, seed, a_device=f"cuda:{local}")
-    pristine_np = None
+    if world > 1:   # 1D block-cyclic: this rank keeps only its nb-blocks of columns
+        cols = torch.from_numpy(sbr.local_columns(n, nb, rank, world)).to(pristine.device)
+        pristine = pristine.index_select(0, cols).contiguous()
+        torch.cuda.empty_cache()
     a = torch.empty_like(pristine)
     ab = torch.empty((n, b + 1), dtype=torch.float32, device=a.device) if rank == 0 else None
-    w = torch.empty((n - b, n), dtype=torch.float32, device=a.device) if rank == 0 else None
+    w = torch.zeros((a.shape[0], n), dtype=torch.float32, device=a.device) if world > 1 else \
+        torch.empty((n - b, n), dtype=torch.float32, device=a.device)
 
     def run_step():
         if world > 1:
-            h.reduce_dist(a, b, nb, mode=mode, ab=ab, w=w)
+            h.reduce_dist(a, n, b, nb, mode=mode, ab=ab, w=w)
         else:
             h.reduce(a, b, nb, mode=mode, ab=ab, w=w)
 
@@ -440,7 +459,7 @@ def main():
     if args.e2e_steps > 0 and world > 1:
         # every rank copies the pinned host input in, the ranks reduce it together, rank 0
         # reads the band back; wall clock with a barrier on both sides, max over ranks
-        a_host = torch.empty((n, n), dtype=torch.float32, pin_memory=True)
+        a_host = torch.empty(tuple(pristine.shape), dtype=torch.float32, pin_memory=True)   # this rank's columns
         a_host.copy_(pristine.cpu())
         ab_host = torch.empty((n, b + 1), dtype=torch.float32, pin_memory=True)
         e2e_ms = []
@@ -458,9 +477,10 @@ def main():
             e2e_ms.append(float(dt.item()))
         e2e_ms = e2e_ms[1:]
         e2e = {"value": eff_tflops(n, statistics.median(e2e_ms) / 1e3), "unit": "TFLOP/s",
-               "h2d_bytes_per_step": 4 * n * n * world, "d2h_bytes_per_step": 4 * n * (b + 1),
+               "h2d_bytes_per_step": 4 * n * n, "d2h_bytes_per_step": 4 * n * (b + 1),
                "ms_per_step": statistics.median(e2e_ms), "steps": args.e2e_steps,
-               "note": "Handle.reduce_dist: pinned host A -> every rank, reduce across ranks, band -> host"}
+               "note": "Handle.reduce_dist: each rank's pinned host columns -> its GPU, reduce across ranks, "
+                       "band -> host (rank 0)"}
         del a_host
     elif args.e2e_steps > 0:
         a_host = torch.empty((n, n), dtype=torch.float32, pin_memory=True)
@@ -511,8 +531,9 @@ def main():
             "config": {"workload": f"{cfg_name}: n={n} {input_desc}, b={b}, nb={nb}, "
                                    f"{'FP16-in/FP32-acc' if mode == 'fp16' else '3xTF32'}",
                        "n": n, "b": b, "nb": nb, "mode": mode,
-                       "parallelism": f"sbr_reduce_dist over {world} GPUs: per-panel pass sharded by lower "
-                                      f"tiles, NCCL broadcast W_t + all-reduce X_t" if world > 1 else "single",
+                       "parallelism": f"sbr_reduce_dist over {world} GPUs: 1D block-cyclic nb-column blocks "
+                                      f"(owner factors its panels; pass and SYR2K on own columns; NCCL "
+                                      f"broadcast W_t / Y, all-reduce X_t)" if world > 1 else "single",
                        "l2": f"inputs {4 * n * n / 2**30:.1f} GiB >> 126 MB L2 (no flush needed)"},
             "frac_of_peak": {"fp16_spec_2250": value / world / 2250.0,
                              "fp16_measured": value / world / peaks.get("bf16_tflops", 1642.5),

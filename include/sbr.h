@@ -145,32 +145,49 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb,
 int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
                float* Q, int64_t ldq);
 
-/* ---- Multi-GPU (one process per GPU, NCCL over NVLink/NVSwitch) ----
+/* ---- Multi-GPU (north star: 1D block-cyclic columns) ----
+ *
+ * Data distribution: the columns of A are split into nb-wide blocks J (global columns
+ * [J nb, (J+1) nb)); rank r holds the blocks with J % nranks == r, in order, as an n x ncols_loc
+ * column-major array A_local (local column of global column g: (J / nranks) nb + (g - J nb));
+ * ncols_loc = sbr_local_cols(n, nb, r, nranks).  The fp16 shadow of the trailing matrix is
+ * sharded the same way, so device memory per rank is about 6 n^2 / nranks bytes plus the
+ * replicated block buffers (Y, X, Z: n x nb each).
  *
  * sbr_get_unique_id: rank 0 creates the 128-byte NCCL unique id (host call, no device work)
  *   and distributes it to the other ranks out of band (e.g. torch.distributed).  Returns 0
  *   or SBR_ERR_NCCL (libnccl.so.2 not loadable; it is dlopen'ed, the single-GPU path never
  *   needs it).
  * sbr_create_dist: like sbr_create, plus an NCCL communicator of `nranks` ranks built from
- *   `unique_id` (collective: every rank must call it).  Returns 0, -1 (h NULL), -2 (device),
- *   -4 (unique_id NULL), -5 (rank), -6 (nranks), SBR_ERR_CUDA, SBR_ERR_NCCL.
- * sbr_reduce_dist: the reduction of ONE matrix across the communicator (strong scaling).
- *   Every rank passes the same input A (full n x n, device; each rank keeps a full copy so
- *   the trailing updates need no data exchange).  Rank 0 runs the sequential per-panel chain
- *   (panel QR, reconstruction, lazy update, W merge) and returns AB, Y (in A) and W exactly
- *   as sbr_reduce; on the other ranks AB and W may be NULL and A is left in an unspecified
- *   state.  Per b-panel every rank streams its 1/nranks share of the lower tiles of OA for
- *   X_t = OA W_t; the partial X_t are summed by an NCCL all-reduce (M x b fp32) after W_t
- *   (fp16, M x b) is broadcast from rank 0; per nb-block rank 0 broadcasts Y (fp16) and
- *   W^T X and every rank applies the trailing update.  All calls are stream-ordered on the
- *   handle's stream and collective (every rank must call with the same n, b, nb, mode).
- *   FP16 mode only when nranks > 1 (else SBR_ERR_UNSUPPORTED).  Same argument errors as
- *   sbr_reduce; SBR_ERR_NCCL on a communication error.
+ *   `unique_id` (collective: every rank must call it; one process per GPU).  Returns 0, -1 (h
+ *   NULL), -2 (device), -4 (unique_id NULL), -5 (rank), -6 (nranks), SBR_ERR_CUDA, SBR_ERR_NCCL.
+ * sbr_create_dist_local: the same reduction with `nranks` handles in ONE process (one host
+ *   thread per rank, any devices, the same one included), exchanging through device memory
+ *   with host barriers instead of NCCL: every rank passes the same `group` key.  It runs the
+ *   same kernels and call sequence as NCCL ranks (used to test the sharded reduction on one
+ *   GPU).  1 <= nranks <= 16.  Same returns as sbr_create_dist.
+ * sbr_local_cols: ncols_loc of `rank` (host only); -1 on invalid arguments.
+ * sbr_reduce_dist: the reduction of ONE matrix across the ranks (strong scaling), collective:
+ *   every rank calls it with the same n, b, nb, mode and its A_local (lda >= n).  The owner of
+ *   block J (J % nranks) factors that block's panels (its columns only: the lazy panel
+ *   updates, TSQR/CholeskyQR + reconstruction and W merges) and broadcasts W_t
+ *   (fp16) per panel; every rank streams the pass tiles of ITS column blocks and the partial
+ *   X_t = OA W_t are summed by an all-reduce (M x b fp32); per block the owner broadcasts Y
+ *   (fp16) and W^T X and every rank applies the trailing SYR2K to its own columns (Eq. 1-3).
+ *   On return: A_local holds the owned columns in sbr_reduce's output layout (band + Y below
+ *   it), W_local (may be NULL, ldw >= n) the owned blocks' W columns (same local columns), and
+ *   AB (rank 0; may be NULL elsewhere) the whole band, assembled over the ranks.  With
+ *   nranks > 1: FP16 mode, b % 8 == 0 and nb a multiple of 128 x the pass's tile columns per
+ *   group (1024 for b <= 32, 512 for b = 64), else SBR_ERR_UNSUPPORTED.  Same argument
+ *   errors as sbr_reduce; SBR_ERR_NCCL on a communication error (a failing rank can leave
+ *   the others blocked in a collective: treat it as fatal for the group).
  * With nranks == 1, sbr_reduce_dist is sbr_reduce. */
 int sbr_get_unique_id(void* unique_id_128_bytes);
 int sbr_create_dist(sbr_handle_t* h, int device, void* stream, const void* unique_id, int rank, int nranks);
+int sbr_create_dist_local(sbr_handle_t* h, int device, void* stream, int group, int rank, int nranks);
+int64_t sbr_local_cols(int64_t n, int nb, int rank, int nranks);
 int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb,
-                    float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw);
+                    float* A_local, int64_t lda, float* AB, int64_t ldab, float* W_local, int64_t ldw);
 int sbr_rank(sbr_handle_t h);     /* 0 for sbr_create handles; -1 if h is NULL */
 int sbr_nranks(sbr_handle_t h);   /* 1 for sbr_create handles; -1 if h is NULL */
 

@@ -80,6 +80,13 @@ int sbr_test_syr2k_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_zform_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
                         const float* X, int64_t ldx, float* Z, int64_t ldz);
 
+/* Host only: the pass tiles rank `rank` of `nranks` streams under sbr_reduce_dist for the block
+ * at column c0 (n, b, nb as the reduction): the 128-aligned tile grid with origin c0 (global
+ * rows / columns c0 + 128 I ..; OA rows start b rows into tile 0), column-block ownership
+ * (J % nranks), lower tiles I >= J.  Writes up to cap pairs IJ[2k] = I, IJ[2k+1] = J in walk
+ * order and returns the count (-1: invalid arguments / unsupported nb). */
+int64_t sbr_test_pass_owned_tiles(int64_t n, int b, int nb, int64_t c0, int rank, int nranks, int* IJ, int64_t cap);
+
 /* Number of CholeskyQR panels that declined (rank deficient / not orthonormal after three
  * rounds, so the paper's TSQR factored them) since the handle's workspace was allocated or
  * the last call with reset != 0.  Synchronises.  Returns 0, -1 (h), -3 (count NULL). */

@@ -15,8 +15,9 @@ tail is ``A[c, c+b+1:]``.  ``ab`` has torch shape (n, b+1): ``ab[j, d] = B[j+d, 
 ``w[c, r] = W(r, c)``.
 """
 from .api import (Handle, reduce, reduce_host, generate_symmetric, band_to_dense, get_unique_id,  # noqa: F401
-                  pass_partition, pass_tiles)
+                  pass_partition, pass_tiles, local_cols, local_columns, pass_owned_tiles)
 from ._lib import lib, LIB_PATH, SbrError  # noqa: F401
 
 __all__ = ["Handle", "reduce", "reduce_host", "generate_symmetric", "band_to_dense", "get_unique_id",
-           "pass_partition", "pass_tiles", "lib", "LIB_PATH", "SbrError"]
+           "pass_partition", "pass_tiles", "local_cols", "local_columns", "pass_owned_tiles", "lib", "LIB_PATH",
+           "SbrError"]

@@ -47,6 +47,8 @@ SIGNATURES = {
     "sbr_version": (ctypes.c_char_p, []),
     "sbr_get_unique_id": (_i, [_p]),
     "sbr_create_dist": (_i, [ctypes.POINTER(ctypes.c_void_p), _i, _p, _p, _i, _i]),
+    "sbr_create_dist_local": (_i, [ctypes.POINTER(ctypes.c_void_p), _i, _p, _i, _i, _i]),
+    "sbr_local_cols": (_i64, [_i64, _i, _i, _i]),
     "sbr_reduce_dist": (_i, [_h, _i, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_form_q": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_rank": (_i, [_h]),
@@ -65,6 +67,7 @@ SIGNATURES = {
                                      ctypes.POINTER(_i64)]),
     "sbr_test_pass_tiles": (_i, [_i64, _i, _i64, _i64, _p]),
     "sbr_test_set_knob": (_i, [_i, _i]),
+    "sbr_test_pass_owned_tiles": (_i64, [_i64, _i, _i, _i64, _i, _i, _p, _i64]),
     "sbr_test_panel_declines": (_i, [_h, _i, ctypes.POINTER(_i64)]),
 }
 

@@ -41,6 +41,29 @@ def pass_partition(M: int, b: int, rank: int, nranks: int):
     return t0.value, t1.value, tot.value
 
 
+def local_cols(n: int, nb: int, rank: int, nranks: int) -> int:
+    """Columns rank ``rank`` holds under the 1D block-cyclic distribution (sbr_local_cols)."""
+    return int(lib().sbr_local_cols(int(n), int(nb), int(rank), int(nranks)))
+
+
+def local_columns(n: int, nb: int, rank: int, nranks: int):
+    """Global column indices of the rank's local columns, in local order (numpy int64)."""
+    import numpy as np
+
+    cols = [np.arange(c0, min(n, c0 + nb)) for c0 in range(rank * nb, n, nranks * nb)]
+    return np.concatenate(cols) if cols else np.zeros(0, dtype=np.int64)
+
+
+def pass_owned_tiles(n: int, b: int, nb: int, c0: int, rank: int, nranks: int):
+    """Host-only: (I, J) tiles of the distributed pass that ``rank`` streams for block origin c0."""
+    cnt = int(lib().sbr_test_pass_owned_tiles(n, b, nb, c0, rank, nranks, None, 0))
+    if cnt < 0:
+        raise ValueError("unsupported arguments")
+    buf = (ctypes.c_int * (2 * cnt + 1))()
+    lib().sbr_test_pass_owned_tiles(n, b, nb, c0, rank, nranks, buf, cnt)
+    return [(buf[2 * k], buf[2 * k + 1]) for k in range(cnt)]
+
+
 def pass_tiles(M: int, b: int, t0: int, t1: int):
     """Host-only: list of (I, J) lower 128x128 tiles [t0, t1) in the pass's order."""
     n = max(0, t1 - t0)
@@ -55,7 +78,9 @@ class Handle:
     an NCCL communicator (one process per GPU) for :meth:`reduce_dist`."""
 
     def __init__(self, device: int = 0, stream=None, unique_id: bytes | None = None, rank: int = 0,
-                 nranks: int = 1):
+                 nranks: int = 1, local_group: int | None = None):
+        """``unique_id``: NCCL communicator (one process per GPU).  ``local_group``: the in-process
+        communicator -- ``nranks`` handles of one process (one thread each) with the same key."""
         import torch
 
         self.device = int(device)
@@ -63,7 +88,10 @@ class Handle:
             stream = torch.cuda.current_stream(self.device)
         self._stream = stream
         h = ctypes.c_void_p()
-        if unique_id is None:
+        if local_group is not None:
+            check(lib().sbr_create_dist_local(ctypes.byref(h), self.device, ctypes.c_void_p(stream.cuda_stream),
+                                              int(local_group), int(rank), int(nranks)), "sbr_create_dist_local")
+        elif unique_id is None:
             check(lib().sbr_create(ctypes.byref(h), self.device, ctypes.c_void_p(stream.cuda_stream)), "sbr_create")
         else:
             uid = ctypes.create_string_buffer(bytes(unique_id), 128)
@@ -140,28 +168,31 @@ class Handle:
         check(lib().sbr_form_q(self._h, n, int(b), int(nb), _ptr(A), n, _ptr(w), n, _ptr(q), n), "sbr_form_q")
         return q
 
-    def reduce_dist(self, A, b: int, nb: int, mode="fp16", want_w: bool = True, ab=None, w=None):
-        """One matrix across the handle's communicator (collective; see sbr_reduce_dist).
+    def reduce_dist(self, A_local, n: int, b: int, nb: int, mode="fp16", want_w: bool = True, ab=None, w=None):
+        """One n x n matrix across the handle's ranks (collective; include/sbr.h sbr_reduce_dist).
 
-        Every rank passes the same (n, n) float32 CUDA tensor; rank 0 gets ``(ab, w)`` as
-        :meth:`reduce` returns them, other ranks get ``(None, None)``."""
+        ``A_local``: this rank's columns -- a contiguous float32 CUDA tensor of torch shape
+        (ncols_loc, n) whose row lc is global column ``local_columns(n, nb, rank, nranks)[lc]``
+        (``A[cols]`` for a symmetric torch matrix ``A``).  Returns ``(ab, w_local)``: the band
+        (rank 0; None elsewhere, torch shape (n, b+1)) and this rank's W columns (same local
+        layout as ``A_local``; None if ``want_w`` is False)."""
         import torch
 
-        n = int(A.shape[0])
-        if A.dim() != 2 or A.shape[1] != n or A.dtype != torch.float32 or not A.is_cuda or not A.is_contiguous():
-            raise ValueError("A must be a contiguous square float32 CUDA tensor")
+        n = int(n)
+        ncl = local_cols(n, nb, self.rank, self.nranks)
+        if (A_local.dim() != 2 or tuple(A_local.shape) != (ncl, n) or A_local.dtype != torch.float32
+                or not A_local.is_cuda or not A_local.is_contiguous()):
+            raise ValueError(f"A_local must be a contiguous ({ncl}, {n}) float32 CUDA tensor")
         lead = self.rank == 0
         if lead and ab is None:
-            ab = torch.empty((n, b + 1), dtype=torch.float32, device=A.device)
-        if lead and want_w and w is None and n > b:
-            w = torch.empty((max(n - b, 1), n), dtype=torch.float32, device=A.device)
-        if not lead or not want_w:
-            w = None if not lead else w
+            ab = torch.empty((n, b + 1), dtype=torch.float32, device=A_local.device)
+        if want_w and w is None and ncl > 0:
+            w = torch.zeros((ncl, n), dtype=torch.float32, device=A_local.device)
         if not want_w:
             w = None
-        check(lib().sbr_reduce_dist(self._h, _mode(mode), n, int(b), int(nb), _ptr(A), n,
+        check(lib().sbr_reduce_dist(self._h, _mode(mode), n, int(b), int(nb), _ptr(A_local), n,
                                     _ptr(ab) if lead else None, b + 1, _ptr(w), n), "sbr_reduce_dist")
-        return (ab, w) if lead else (None, None)
+        return (ab if lead else None), w
 
     def reduce_host(self, A, b: int, nb: int, mode="fp16", outputs: int = _lib.SBR_OUT_BAND, ab=None, w=None):
         """End-to-end variant on HOST buffers (torch CPU tensors, ideally pinned, or numpy).

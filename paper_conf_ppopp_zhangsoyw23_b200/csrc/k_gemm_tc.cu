@@ -62,6 +62,21 @@ SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
   }
 }
 
+// Multi-GPU column ownership of the SYR2K output (sbr_reduce_dist): output column rel (relative to
+// the trailing region) is global column org + rel, owned by rank (g / nbo) % P; the owned tiles
+// (BN columns, inside one block) update C / shadow at local column (g / nbo / P) nbo + g % nbo
+// (C and shadow then point at the region's first ROW, column 0).  P = 1: every tile, column rel.
+struct GemmOwn {
+  int P = 1, rank = 0;
+  int64_t org = 0, nbo = 1;
+  SBR_DEV bool owned(int64_t rel) const { return P <= 1 || ((org + rel) / nbo) % P == rank; }
+  SBR_DEV int64_t lcol(int64_t rel) const {
+    if (P <= 1) return rel;
+    const int64_t g = org + rel;
+    return (g / nbo / P) * nbo + g % nbo;
+  }
+};
+
 constexpr int G_EPI_WARPS = 8;  // two warps per TMEM lane quarter, each half of the 256 columns
 constexpr int G_THREADS = 128 + 32 * G_EPI_WARPS;
 
@@ -78,7 +93,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
                    const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
                    const GemmSegs segs, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles,
                    float* C, int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, const float* __restrict__ X,
-                   int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off) {
+                   int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off, const GemmOwn own) {
   using Cfg = GCfg<TF>;
   constexpr int BK = TF ? 32 : 64;   // K elements per 128-byte row chunk
   constexpr int G_BN = Cfg::BN, G_NS = Cfg::NS, G_STAGE = Cfg::STAGE;
@@ -114,6 +129,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
         int I, Jc;
         gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+        if (!own.owned((int64_t)Jc * G_BN)) continue;
         for (int kc = 0; kc < nk; ++kc) {
           const int sg = kc / kpb, kin = (kc % kpb) * BK;
           mbar_wait(&empty[st], ph ^ 1);
@@ -135,6 +151,11 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       // accumulation groups: fp16 one per tile; 3xTF32 every FLUSH k-chunks (drained by the epilogue)
       const int ch = TF ? Cfg::FLUSH : nk;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+        if (own.P > 1) {
+          int I, Jc;
+          gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+          if (!own.owned((int64_t)Jc * G_BN)) continue;
+        }
         for (int kc = 0; kc < nk; ++kc) {
           if (kc % ch == 0) {
             mbar_wait(&acc_empty[ab], aph ^ 1);
@@ -173,6 +194,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
       gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+      if (!own.owned((int64_t)Jc * G_BN)) continue;
       float acc[64];
 #pragma unroll
       for (int c = 0; c < 64; ++c) acc[c] = 0.f;
@@ -195,7 +217,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       if (row >= Mrows) continue;
       const int64_t col0 = (int64_t)Jc * G_BN + chalf * 64;
       if (MODE == 0 || MODE == 3) {   // SYR2K: lower elements; GEMM_SUB: all of C
-        float* cp = C + row + col0 * ldc;
+        float* cp = C + row + own.lcol(col0) * ldc;
 #pragma unroll
         for (int c = 0; c < 64; ++c)
           if (MODE == 0 ? (col0 + c <= row) : (col0 + c < Ncols)) __stcs(cp + c * ldc, __ldcs(cp + c * ldc) - acc[c]);
@@ -225,6 +247,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
       gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+      if (!own.owned((int64_t)Jc * G_BN)) continue;
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();
       const int64_t row = (int64_t)I * G_BM + rit;
@@ -238,7 +261,9 @@ __global__ void __launch_bounds__(G_THREADS, 1)
         tmem_ld32(tmem + ab * G_BN + cc * 32 + lane_off, v);
         if (row >= Mrows) continue;
         if (MODE == 0) {
-          float* cp = C + row + col0 * ldc;
+          const int64_t lc0 = own.lcol(col0);
+          float* cp = C + row + lc0 * ldc;
+          __half* sp = shadow + row + lc0 * ldsh;
           float old[32];
 #pragma unroll
           for (int c = 0; c < 32; ++c) old[c] = (col0 + c <= row) ? __ldcs(cp + c * ldc) : 0.f;   // all loads first
@@ -248,7 +273,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
             if (col <= row) {
               const float nv = old[c] - v[c];
               __stcs(cp + c * ldc, nv);
-              shadow[row + col * ldsh] = __float2half_rn(col == row ? 0.5f * nv : nv);
+              sp[c * ldsh] = __float2half_rn(col == row ? 0.5f * nv : nv);
             }
           }
         } else {
@@ -331,9 +356,17 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   }
   if (ntiles == 0) return cudaSuccess;
   const int grid = std::min(ntiles, p.num_sms);
+  GemmOwn own;
+  if (p.own_P > 1) {
+    if (MODE != 0 || p.nbo % G_BN != 0 || p.own_org % p.nbo != 0) return cudaErrorInvalidValue;
+    own.P = p.own_P;
+    own.rank = p.own_rank;
+    own.org = p.own_org;
+    own.nbo = p.nbo;
+  }
   return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
                     (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
-                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off);
+                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off, own);
 }
 
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, false>(p, st); }

@@ -96,18 +96,19 @@ cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaS
 // reduction that follows runs on finite data (its outputs are invalid; the error is latched)
 constexpr int kScaleZero = -(1 << 30);
 
-// a0 scan (reading C10): finiteness of the referenced lower triangle (flag[0] |= 1) and
-// ||A||_F^2 in fp64 (off-diagonal entries twice), one fp64 atomic per block.
-__global__ void prep_scan_kernel(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2) {
-  const int64_t j = blockIdx.y;
+// a0 scan (reading C10): over the local columns j (global column cm.g(j)), the referenced lower
+// triangle: scan[0] += ||.||_F^2 (fp64, off-diagonal entries twice), scan[1] += count of Inf/NaN.
+__global__ void prep_scan_kernel(int64_t n, int64_t j0, const float* A, int64_t lda, ColMap cm, double* scan) {
+  const int64_t j = j0 + blockIdx.y;
+  const int64_t g = cm.g(j);
   double s = 0.0;
   bool bad = false;
-  for (int64_t i = j + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+  for (int64_t i = g + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     const float v = A[i + j * lda];
     if (!isfinite(v)) bad = true;
-    s += (i == j ? 1.0 : 2.0) * (double)v * (double)v;
+    else s += (i == g ? 1.0 : 2.0) * (double)v * (double)v;
   }
-  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicOr(flag, 1u);
+  if (__syncthreads_or(bad) && threadIdx.x == 0) atomicAdd(scan + 1, 1.0);
   __shared__ double red[32];
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
@@ -117,7 +118,7 @@ __global__ void prep_scan_kernel(int64_t n, const float* A, int64_t lda, unsigne
     s = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : 0.0;
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    if (threadIdx.x == 0 && s != 0.0) atomicAdd(fro2, s);
+    if (threadIdx.x == 0 && s != 0.0) atomicAdd(scan, s);
   }
 }
 
@@ -128,14 +129,15 @@ __global__ void prep_scan_kernel(int64_t n, const float* A, int64_t lda, unsigne
 // subnormal range.  The 3xTF32 mode takes the same scale (tf32 has fp32's exponent range,
 // but the fp32 panel norms and products of an input near the ends of that range would
 // under- or overflow).  k = 0 for a zero or non-finite input.
-__global__ void choose_scale_kernel(const double* fro2, const unsigned* flag, int fp16_mode, int* kexp) {
+__global__ void choose_scale_kernel(const double* scan, unsigned* flag, int* kexp) {
   int k = 0;
-  const double f2 = *fro2;
-  if (flag[0]) {   // non-finite input: the reduction runs on zeros (error latched, outputs invalid)
+  const double f2 = scan[0];
+  if (scan[1] != 0.0) {   // non-finite input: the reduction runs on zeros (error latched, outputs invalid)
+    flag[0] = 1u;
     *kexp = kScaleZero;
     return;
   }
-  if (!flag[0] && f2 > 0.0 && isfinite(f2)) {   // both modes (fp16_mode kept for the record)
+  if (f2 > 0.0 && isfinite(f2)) {   // both modes
     int e = 0;
     frexp(sqrt(f2), &e);   // ||A||_F in [2^(e-1), 2^e)
     k = max(-250, min(250, 13 - e));
@@ -143,16 +145,20 @@ __global__ void choose_scale_kernel(const double* fro2, const unsigned* flag, in
   *kexp = k;
 }
 
-cudaError_t prep_scale(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2, int* kexp,
-                       bool fp16_mode, cudaStream_t st) {
-  cudaError_t e = cudaMemsetAsync(fro2, 0, sizeof(double), st);
+cudaError_t prep_scan(int64_t n, int64_t ncols, const float* A, int64_t lda, ColMap cm, double* scan,
+                      cudaStream_t st) {
+  cudaError_t e = cudaMemsetAsync(scan, 0, 2 * sizeof(double), st);
   if (e != cudaSuccess) return e;
-  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
-    const int64_t nc = std::min<int64_t>(65535, n - j0);
+  for (int64_t j0 = 0; j0 < ncols; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, ncols - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 16), (unsigned)nc);
-    prep_scan_kernel<<<grid, 256, 0, st>>>(n - j0, A + j0 + j0 * lda, lda, flag, fro2);
+    prep_scan_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, cm, scan);
   }
-  choose_scale_kernel<<<1, 1, 0, st>>>(fro2, flag, fp16_mode ? 1 : 0, kexp);
+  return cudaGetLastError();
+}
+
+cudaError_t choose_scale(const double* scan, unsigned* flag, int* kexp, cudaStream_t st) {
+  choose_scale_kernel<<<1, 1, 0, st>>>(scan, flag, kexp);
   return cudaGetLastError();
 }
 
@@ -164,19 +170,20 @@ SBR_DEV float scale_pow2(float a, int k) {
 }
 
 // 3xTF32 mode: the lower triangle of A scaled in place by 2^k (no-op for k = 0)
-__global__ void scale_lower_kernel(int64_t n, int64_t j0, float* A, int64_t lda, const int* kexp) {
+__global__ void scale_lower_kernel(int64_t n, int64_t j0, float* A, int64_t lda, ColMap cm, const int* kexp) {
   const int k = *kexp;
   if (k == 0) return;
   const int64_t j = j0 + blockIdx.y;
-  for (int64_t i = j + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+  const int64_t g = cm.g(j);
+  for (int64_t i = g + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
     A[i + j * lda] = k == kScaleZero ? 0.f : scale_pow2(A[i + j * lda], k);
 }
 
-cudaError_t scale_lower(int64_t n, float* A, int64_t lda, const int* kexp, cudaStream_t st) {
-  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
-    const int64_t nc = std::min<int64_t>(65535, n - j0);
+cudaError_t scale_lower(int64_t n, int64_t ncols, float* A, int64_t lda, ColMap cm, const int* kexp, cudaStream_t st) {
+  for (int64_t j0 = 0; j0 < ncols; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, ncols - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 32), (unsigned)nc);
-    scale_lower_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, kexp);
+    scale_lower_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, cm, kexp);
   }
   return cudaGetLastError();
 }
@@ -195,19 +202,21 @@ cudaError_t note_unhandled(const int* fail, unsigned* sticky, cudaStream_t st) {
 
 // Band out (a7): AB = 2^-k (band of A), written back into A's band unscaled too (A's Y part is
 // scale free); a non-finite band entry (fp16 range exceeded despite the scaling) latches flag[2].
-__global__ void extract_band_kernel(int64_t n, int b, float* A, int64_t lda, float* AB, int64_t ldab,
-                                    const int* kexp, unsigned* flag) {
-  const int64_t j = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
+// Local column lc (global cm.g(lc)) of A fills AB column cm.g(lc).
+__global__ void extract_band_kernel(int64_t n, int64_t ncols, int b, float* A, int64_t lda, ColMap cm, float* AB,
+                                    int64_t ldab, const int* kexp, unsigned* flag) {
+  const int64_t lc = (int64_t)blockIdx.x * blockDim.y + threadIdx.y;
   const int d = threadIdx.x;
   const int k = (kexp && *kexp != kScaleZero) ? *kexp : 0;
   bool bad = false;
-  if (j < n && d <= b) {
+  if (lc < ncols && d <= b) {
+    const int64_t j = cm.g(lc);
     float v = 0.f;
     if (j + d < n) {
-      v = A[(j + d) + j * lda];
+      v = A[(j + d) + lc * lda];
       if (k != 0) {
         v = scale_pow2(v, -k);
-        A[(j + d) + j * lda] = v;
+        A[(j + d) + lc * lda] = v;
       }
       bad = !isfinite(v);
     }
@@ -217,10 +226,12 @@ __global__ void extract_band_kernel(int64_t n, int b, float* A, int64_t lda, flo
 }
 
 cudaError_t extract_band(int64_t n, int b, float* A, int64_t lda, float* AB, int64_t ldab, const int* kexp,
-                         unsigned* flag, cudaStream_t st) {
+                         unsigned* flag, cudaStream_t st, int64_t ncols, ColMap cm) {
+  if (ncols < 0) ncols = n;
   const int dx = b + 1;
   const int dy = max(1, 256 / dx);
-  extract_band_kernel<<<(unsigned)((n + dy - 1) / dy), dim3(dx, dy), 0, st>>>(n, b, A, lda, AB, ldab, kexp, flag);
+  extract_band_kernel<<<(unsigned)((ncols + dy - 1) / dy), dim3(dx, dy), 0, st>>>(n, ncols, b, A, lda, cm, AB, ldab,
+                                                                                 kexp, flag);
   return cudaGetLastError();
 }
 
@@ -277,29 +288,31 @@ cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaS
 // above (so that a diagonal tile T satisfies T + T^T = L; see k_pass_tc.cu).  With k != 0 the
 // fp32 master's lower triangle is scaled in place too (exact: powers of two; reading C10).
 __global__ void shadow_init_kernel(int64_t n, int64_t j0, float* A, int64_t lda, __half* Sh, int64_t ldsh,
-                                   const int* kexp) {
+                                   const int* kexp, ColMap cm) {
   const int64_t j = j0 + blockIdx.y;
+  const int64_t g = cm.g(j);
   const int k = kexp ? *kexp : 0;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     float v = 0.f;
-    if (i >= j) {
+    if (i >= g) {
       v = A[i + j * lda];
       if (k != 0) {
         v = k == kScaleZero ? 0.f : scale_pow2(v, k);
         A[i + j * lda] = v;
       }
-      if (i == j) v *= 0.5f;
+      if (i == g) v *= 0.5f;
     }
     Sh[i + j * ldsh] = __float2half_rn(v);
   }
 }
 
 cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ldsh, const int* kexp,
-                        cudaStream_t st) {
-  for (int64_t j0 = 0; j0 < n; j0 += 65535) {
-    const int64_t nc = std::min<int64_t>(65535, n - j0);
+                        cudaStream_t st, int64_t ncols, ColMap cm) {
+  if (ncols < 0) ncols = n;
+  for (int64_t j0 = 0; j0 < ncols; j0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, ncols - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 32), (unsigned)nc);
-    shadow_init_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, Sh, ldsh, kexp);
+    shadow_init_kernel<<<grid, 256, 0, st>>>(n, j0, A, lda, Sh, ldsh, kexp, cm);
   }
   return cudaGetLastError();
 }

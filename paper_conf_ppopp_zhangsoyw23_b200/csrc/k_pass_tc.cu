@@ -38,23 +38,37 @@ struct PassCfg {
 // (balanced to one tile), so a launch ends when the slowest SM has streamed T/grid tiles.
 // The three roles walk the same range with this iterator.
 #define SBR_HD __host__ __device__ __forceinline__
+// Multi-GPU (sbr_reduce_dist, 1D block-cyclic columns): only the groups whose tile columns lie in
+// this rank's column blocks are walked -- group g covers global column block blk0 + g / gpb,
+// owned by rank (blk0 + g / gpb) % P (P = 1: every group).
+struct PassOwn {
+  int P = 1, rank = 0, blk0 = 0, gpb = 1;
+  SBR_HD bool owned(int g) const { return P <= 1 || (blk0 + g / gpb) % P == rank; }
+};
+
 struct PassWalk {
   int NT, C;
   int g, J0, ceff, I, J;
   int64_t left;
   bool gfirst, rfirst;
+  PassOwn own;
   SBR_HD int jend() const { return min(J0 + ceff, I + 1); }
   SBR_HD static int64_t group_tiles(int NT, int C, int g) {
     const int J0 = g * C, ce = min(C, NT - J0);
     return (int64_t)ce * (ce + 1) / 2 + (int64_t)(NT - J0 - ce) * ce;
   }
-  SBR_HD void start(int NT_, int C_, int64_t t0, int64_t count) {
+  SBR_HD int64_t owned_tiles(int g) const { return own.owned(g) ? group_tiles(NT, C, g) : 0; }
+  SBR_HD void start(int NT_, int C_, int64_t t0, int64_t count, PassOwn own_ = PassOwn()) {
     NT = NT_;
     C = C_;
+    own = own_;
     left = count;
     g = 0;
+    gfirst = rfirst = true;
+    if (count <= 0) return;   // nothing to walk (e.g. a rank that owns no column of this OA)
     for (;;) {
-      const int64_t gt = group_tiles(NT, C, g);
+      if (g * C >= NT) break;
+      const int64_t gt = owned_tiles(g);
       if (t0 < gt) break;
       t0 -= gt;
       ++g;
@@ -91,7 +105,9 @@ struct PassWalk {
       return;
     }
     gfirst = true;
-    ++g;
+    do {
+      ++g;
+    } while (g * C < NT && !own.owned(g));
     J0 = g * C;
     ceff = min(C, NT - J0);
     I = J = J0;
@@ -101,7 +117,12 @@ struct PassWalk {
 template <int BN, int C, int NS>
 __global__ void __launch_bounds__(256, 1)
     pass_tc_kernel(const __grid_constant__ CUtensorMap mapL, const __grid_constant__ CUtensorMap mapW, int r0, int M,
-                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx, int exper) {
+                   int NT, int64_t T0, int64_t T, int b, float* X, int64_t ldx, int exper, int off, PassOwn own,
+                   int nbo) {
+  // tile I covers shadow rows / columns r0 + 128 I .. (r0 = the first tile's origin) and OA rows
+  // 128 I - off ..; W rows are stored with `off` zero rows in front (W row 128 J = OA row 128 J - off).
+  // Multi-GPU: the shadow holds this rank's columns only: local column of global column g =
+  // (g / nbo / P) nbo + g % nbo.
   using Cfg = PassCfg<BN, C, NS>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -146,6 +167,12 @@ __global__ void __launch_bounds__(256, 1)
   const uint32_t t_col = tmem;                 // C column accumulators: cols [jj*BN, jj*BN+BN)
   const uint32_t t_row = tmem + C * BN;        // 2 row accumulators
   PassWalk w;
+  auto lcolJ = [&](int Jt) -> int {   // shadow column coordinate of tile column Jt
+    const int g = r0 + Jt * 128;
+    if (own.P <= 1) return g;
+    const int blk = g / nbo;
+    return (blk / own.P) * nbo + g % nbo;
+  };
 
   if (warp == 0) {
     // ------------------------------------------------ TMA producer
@@ -155,7 +182,7 @@ __global__ void __launch_bounds__(256, 1)
       int st = 0; uint32_t ph = 0;            // L ring
       int ws = 0; uint32_t wph = 0;           // W_I ring
       uint32_t jph = 0;
-      for (w.start(NT, C, t_beg, t_end - t_beg); w.valid(); w.next()) {
+      for (w.start(NT, C, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
         if (w.gfirst) {
           mbar_wait(wj_empty, jph ^ 1);
           jph ^= 1;
@@ -174,7 +201,7 @@ __global__ void __launch_bounds__(256, 1)
         mbar_expect_tx(&l_full[st], Cfg::LT);
         uint8_t* dst = sL + st * Cfg::LT;
         for (int rb = 0; rb < 2; ++rb)   // box = 64 rows x 128 columns (same smem image as 2 boxes of 64)
-          tma_load_2d_hint(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, r0 + w.J * 128, lpol);
+          tma_load_2d_hint(dst + rb * 16384, &mapL, &l_full[st], r0 + w.I * 128 + rb * 64, lcolJ(w.J), lpol);
         if (++st == NS) { st = 0; ph ^= 1; }
         if (w.rlast()) {
           if (++ws == 2) { ws = 0; wph ^= 1; }
@@ -193,7 +220,7 @@ __global__ void __launch_bounds__(256, 1)
       const uint32_t aL = smem_u32(sL), aWj = smem_u32(sWj), aWi = smem_u32(sWi);
       uint32_t cinit = 0;
       bool rowfirst = true;
-      for (w.start(NT, C, t_beg, t_end - t_beg); w.valid(); w.next()) {
+      for (w.start(NT, C, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
         if (w.gfirst) {
           mbar_wait(wj_full, jph);
           jph ^= 1;
@@ -253,18 +280,18 @@ __global__ void __launch_bounds__(256, 1)
     int rb = 0; uint32_t rph = 0;
     uint32_t cph = 0;
     uint32_t touched = 0;
-    for (w.start(NT, C, t_beg, t_end - t_beg); w.valid(); w.next()) {
+    for (w.start(NT, C, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
       if (w.gfirst) touched = 0;
       touched |= 1u << (w.J - w.J0);
       if (w.rlast()) {
         mbar_wait(&racc_full[rb], rph);
         tc_fence_after();
-        const int64_t row = (int64_t)w.I * 128 + row_in_tile;
+        const int64_t row = (int64_t)w.I * 128 + row_in_tile - off;
 #pragma unroll
         for (int c0 = 0; c0 < BN; c0 += 32) {
           float v[32];
           tmem_ld32(t_row + rb * BN + c0 + lane_off, v);
-          if (row < M) {
+          if (row >= 0 && row < M) {
 #pragma unroll
             for (int c = 0; c < 32; ++c)
               if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
@@ -280,12 +307,12 @@ __global__ void __launch_bounds__(256, 1)
         tc_fence_after();
         for (int jj = 0; jj < w.ceff; ++jj) {
           if (!((touched >> jj) & 1u)) continue;
-          const int64_t row = (int64_t)(w.J0 + jj) * 128 + row_in_tile;
+          const int64_t row = (int64_t)(w.J0 + jj) * 128 + row_in_tile - off;
 #pragma unroll
           for (int c0 = 0; c0 < BN; c0 += 32) {
             float v[32];
             tmem_ld32(t_col + jj * BN + c0 + lane_off, v);
-            if (row < M) {
+            if (row >= 0 && row < M) {
 #pragma unroll
               for (int c = 0; c < 32; ++c)
                 if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
@@ -306,9 +333,10 @@ __global__ void __launch_bounds__(256, 1)
 }
 
 // ---------------------------------------------------------------- host
-static int64_t pass_total_tiles(int NT, int C) {
+static int64_t pass_total_tiles(int NT, int C, PassOwn own = PassOwn()) {
   int64_t T = 0;
-  for (int g = 0; g * C < NT; ++g) T += PassWalk::group_tiles(NT, C, g);
+  for (int g = 0; g * C < NT; ++g)
+    if (own.owned(g)) T += PassWalk::group_tiles(NT, C, g);
   return T;
 }
 
@@ -325,6 +353,29 @@ void pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t
   *total = T;
   *t0 = T * rank / nranks;
   *t1 = T * (rank + 1) / nranks;
+}
+
+// multi-GPU: the tiles `rank` walks for a block with 128-aligned grid origin r0g, OA offset `off`
+// (OA rows start off rows into tile 0), ownership width nbo -- host mirror of the kernel's walk
+int64_t pass_owned_tiles(int64_t M, int b, int64_t r0g, int off, int64_t nbo, int P, int rank, int* IJ, int64_t cap) {
+  const int C = pass_group_cols(b);
+  const int NT = (int)((M + off + 127) / 128);
+  PassOwn own;
+  own.P = P;
+  own.rank = rank;
+  own.blk0 = (int)(r0g / nbo);
+  own.gpb = (int)(nbo / (128 * C));
+  if (P > 1 && (own.gpb < 1 || nbo % (128 * C) != 0 || r0g % 128 != 0)) return -1;
+  const int64_t T = pass_total_tiles(NT, C, own);
+  PassWalk w;
+  int64_t k = 0;
+  for (w.start(NT, C, 0, T, own); w.valid(); w.next(), ++k) {
+    if (IJ && k < cap) {
+      IJ[2 * k] = w.I;
+      IJ[2 * k + 1] = w.J;
+    }
+  }
+  return k;
 }
 
 void pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ) {
@@ -346,19 +397,27 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
     if (e != cudaSuccess) return e;
   }
   CUtensorMap mapL, mapW;
-  cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.n, p.ld_shadow, 64, 128);
+  cudaError_t e = make_tmap_2d(&mapL, p.shadow, true, p.n, p.shadow_cols > 0 ? p.shadow_cols : p.n, p.ld_shadow, 64, 128);
   if (e != cudaSuccess) return e;
-  e = make_tmap_2d(&mapW, p.Wh, true, p.M, BN, p.ld_wh, 64, BN);
+  e = make_tmap_2d(&mapW, p.Wh, true, p.M + p.off, BN, p.ld_wh, 64, BN);
   if (e != cudaSuccess) return e;
-  const int NT = (int)((p.M + 127) / 128);
-  const int64_t Tall = pass_total_tiles(NT, C);
+  const int NT = (int)((p.M + p.off + 127) / 128);
+  PassOwn own;
+  if (p.own_P > 1) {   // column-block ownership (sbr_reduce_dist): groups of C tile columns, nbo / (128 C) per block
+    own.P = p.own_P;
+    own.rank = p.own_rank;
+    own.blk0 = (int)(p.r0 / p.nbo);
+    own.gpb = (int)(p.nbo / (128 * C));
+    if (own.gpb < 1 || p.nbo % (128 * C) != 0 || p.r0 % 128 != 0) return cudaErrorInvalidValue;
+  }
+  const int64_t Tall = pass_total_tiles(NT, C, own);
   const int64_t T0 = Tall * p.rank / p.nranks, T1 = Tall * (p.rank + 1) / p.nranks;
   const int64_t T = T1 - T0;
   if (T <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
   const int exper = knob(KNOB_PASS_EXPER);   // timing experiments only (sbr_test_set_knob); 0 in production
   return launch_pdl(kern, dim3(grid), dim3(256), Cfg::SMEM, st, mapL, mapW, (int)p.r0, (int)p.M, NT, T0, T, p.b,
-                    p.X, p.ldx, exper);
+                    p.X, p.ldx, exper, p.off, own, p.nbo);
 }
 
 static int pass_variant() {   // SBR_PASS_CFG (tuning experiments only): 0 = C8/NS4, 1 = C4/NS5, 2 = C2/NS6
@@ -384,5 +443,7 @@ cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st) {
 }
 
 int pass_bn(int b) { return b <= 16 ? 16 : b <= 32 ? 32 : 64; }
+
+int pass_dist_align(int b) { return 128 * pass_group_cols(b); }
 
 }  // namespace sbr

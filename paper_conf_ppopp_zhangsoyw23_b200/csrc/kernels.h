@@ -79,17 +79,27 @@ cudaError_t tn_small(int64_t rows, int b, const float* A, int64_t lda, const flo
 
 // ---- misc ----
 cudaError_t gen_symmetric(uint64_t seed, int64_t n, float* A, int64_t lda, cudaStream_t st);
-// a0: flag[0] |= 1 if the lower triangle holds Inf/NaN; *kexp = k of the scale 2^k
-// (||A||_F 2^k in [2^12, 2^13)); fro2: one double of scratch
-cudaError_t prep_scale(int64_t n, const float* A, int64_t lda, unsigned* flag, double* fro2, int* kexp,
-                       bool fp16_mode, cudaStream_t st);
+// Local -> global column map of a rank's 1D block-cyclic storage (sbr_reduce_dist): local column
+// lc holds global column ((lc / nbo) P + rank) nbo + lc % nbo.  P = 1: identity.
+struct ColMap {
+  int P = 1, rank = 0;
+  int64_t nbo = 1;
+  __host__ __device__ int64_t g(int64_t lc) const { return P <= 1 ? lc : ((lc / nbo) * P + rank) * nbo + lc % nbo; }
+};
+// a0: scan[0] = ||A_lower||_F^2 over the local columns, scan[1] = count of non-finite entries (2
+// doubles, summed over ranks by the caller if distributed); then choose_scale: flag[0] = 1 if any
+// Inf/NaN (k = a sentinel: the matrix is zeroed), else *kexp = k of 2^k with ||A||_F 2^k in
+// [2^12, 2^13)
+cudaError_t prep_scan(int64_t n, int64_t ncols, const float* A, int64_t lda, ColMap cm, double* scan,
+                      cudaStream_t st);
+cudaError_t choose_scale(const double* scan, unsigned* flag, int* kexp, cudaStream_t st);
 // 3xTF32 mode: A's lower triangle *= 2^k in place (the FP16 mode does it in shadow_init)
-cudaError_t scale_lower(int64_t n, float* A, int64_t lda, const int* kexp, cudaStream_t st);
+cudaError_t scale_lower(int64_t n, int64_t ncols, float* A, int64_t lda, ColMap cm, const int* kexp, cudaStream_t st);
 cudaError_t note_unhandled(const int* fail, unsigned* sticky, cudaStream_t st);
 // band out, unscaled by 2^-k (kexp may be NULL: k = 0); A's band rewritten unscaled; a non-finite
 // band entry sets flag[2] (flag may be NULL)
 cudaError_t extract_band(int64_t n, int b, float* A, int64_t lda, float* AB, int64_t ldab, const int* kexp,
-                         unsigned* flag, cudaStream_t st);
+                         unsigned* flag, cudaStream_t st, int64_t ncols = -1, ColMap cm = ColMap());
 cudaError_t mirror_lower_block(int b, float* A, int64_t lda, cudaStream_t st);
 cudaError_t lazy_small_p(int k, int b, const float* Xc, int64_t ldx, const float* WtX, int64_t ldwx,
                          const float* Yc, int64_t ldy, float* P, cudaStream_t st);
@@ -120,13 +130,22 @@ struct PassLaunch {
   int64_t ldx;
   int num_sms;
   int seg_rows;
-  int rank = 0, nranks = 1;   // tile share of this launch (sbr_reduce_dist): [T*rank/nranks, T*(rank+1)/nranks)
+  int rank = 0, nranks = 1;   // tile share of this launch: [T*rank/nranks, T*(rank+1)/nranks) of the walked tiles
+  // multi-GPU column ownership (sbr_reduce_dist): the shadow holds the columns of blocks J % own_P
+  // == own_rank only (shadow_cols of them, local column = (g / nbo / own_P) nbo + g % nbo); r0 is
+  // then the 128-aligned origin of the tile grid and `off` the OA row of its first row (W stored
+  // with `off` zero rows in front, X rows = tile rows - off)
+  int own_P = 1, own_rank = 0;
+  int64_t nbo = 0, shadow_cols = 0;
+  int off = 0;
 };
 cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st);
 // host mirror of the pass's tile order (k_pass_tc.cu PassWalk): share of `rank`, and the (I, J) list
 void pass_partition(int64_t M, int b, int rank, int nranks, int64_t* t0, int64_t* t1, int64_t* total);
 void pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int* IJ);
 int pass_bn(int b);
+int pass_dist_align(int b);
+int64_t pass_owned_tiles(int64_t M, int b, int64_t r0g, int off, int64_t nbo, int P, int rank, int* IJ, int64_t cap);   // column-block width multiple the distributed pass needs (128 x tile columns per group)
 
 // 3xTF32 pass (k_pass_tf32.cu): X (M x b, b <= 32, column-major, zeroed by the caller) +=
 // OA WS with OA = A[r0:, r0:] (fp32 master, lower referenced, lda % 4 == 0) except tile
@@ -163,6 +182,12 @@ struct GemmTcLaunch {
   int64_t lo_off = 0;
   float* Zs = nullptr;
   int64_t zlo_off = -1;   // lo offset of the Zs output (default lo_off)
+  // SYR2K column ownership (sbr_reduce_dist): output column rel is global column own_org + rel,
+  // updated only if ((own_org + rel) / nbo) % own_P == own_rank, at LOCAL column
+  // (g / nbo / own_P) nbo + g % nbo of C / shadow (which then point at the region's first row,
+  // column 0).  own_P = 1: every tile; C / shadow point at the region's origin.
+  int own_P = 1, own_rank = 0;
+  int64_t own_org = 0, nbo = 1;
 };
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st);
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st);
@@ -272,7 +297,7 @@ cudaError_t build_lazy_b(int k, int b, const __half* Yh, int64_t ldyh, int64_t c
 // fp16 shadow of 2^k A (lower; half diagonal; zero upper); with k != 0 also scales A's lower
 // triangle in place (kexp may be NULL: k = 0)
 cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ldsh, const int* kexp,
-                        cudaStream_t st);
+                        cudaStream_t st, int64_t ncols = -1, ColMap cm = ColMap());
 cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
                        int64_t ldd, cudaStream_t st);
 

@@ -60,6 +60,9 @@ int comm_destroy(Comm c) { return g_api.commDestroy(c); }
 int all_reduce_sum_f32(float* buf, size_t count, Comm c, cudaStream_t st) {
   return g_api.allReduce(buf, buf, count, kFloat32, kSum, c, st);
 }
+int all_reduce_sum(void* buf, size_t count, int dtype, Comm c, cudaStream_t st) {
+  return g_api.allReduce(buf, buf, count, dtype, kSum, c, st);
+}
 int broadcast(void* buf, size_t count, int dtype, int root, Comm c, cudaStream_t st) {
   return g_api.broadcast(buf, buf, count, dtype, root, c, st);
 }

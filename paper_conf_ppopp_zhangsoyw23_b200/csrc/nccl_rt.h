@@ -25,6 +25,7 @@ int get_unique_id(UniqueId* id);
 int comm_init_rank(Comm* c, int nranks, const UniqueId& id, int rank);
 int comm_destroy(Comm c);
 int all_reduce_sum_f32(float* buf, size_t count, Comm c, cudaStream_t st);   // in place
+int all_reduce_sum(void* buf, size_t count, int dtype, Comm c, cudaStream_t st);   // in place
 int broadcast(void* buf, size_t count, int dtype, int root, Comm c, cudaStream_t st);   // in place
 
 }  // namespace nccl

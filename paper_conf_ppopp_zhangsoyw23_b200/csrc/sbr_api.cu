@@ -14,6 +14,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <mutex>
 #include <string>
 #include <vector>
@@ -21,6 +22,7 @@
 #include "../../include/sbr.h"
 #include "common.cuh"
 #include "kernels.h"
+#include "comm.h"
 #include "nccl_rt.h"
 
 using namespace sbr;
@@ -57,6 +59,8 @@ struct sbr_ctx {
   size_t ws_bytes = 0;
   int64_t ws_n = -1;
   int ws_b = -1, ws_nb = -1, ws_mode = -1;
+  int64_t ws_shcols = -1;
+  float* ABd = nullptr;     // multi-GPU: (b+1) x n band assembled over the ranks
   float *Yb = nullptr, *Xb = nullptr, *Zb = nullptr, *Wws = nullptr, *Strip = nullptr, *WtX = nullptr,
         *Pb = nullptr, *Gb = nullptr;
   float *pv = nullptr, *ptau = nullptr, *pr = nullptr, *pq = nullptr, *pmisc = nullptr;
@@ -92,8 +96,7 @@ struct sbr_ctx {
   int64_t launches = 0;
   // multi-GPU (sbr_create_dist): this process's rank in an NCCL communicator of nranks
   int rank = 0, nranks = 1;
-  nccl::Comm comm = nullptr;
-  bool force_coll = false;   // SBR_DIST_COLLECTIVES=1: issue the exchanges even with one rank (tests)
+  sbr::Comm* comm = nullptr;   // NCCL or in-process ("local") communicator (comm.h)
   bool tf32_tc = true;       // SBR_TF32_TC=0: 3xTF32 mode on the SIMT fp32 kernels (ablation)
   // latched device-detected errors (§8(b)): each sbr_reduce copies its status words (flag[0..3])
   // into a pinned slot and records an event; sbr_sync and the next calls report them
@@ -223,6 +226,15 @@ int latch_status(sbr_ctx* h, cudaStream_t st) {
     }                                                                  \
   } while (0)
 
+#define SBR_CM(expr, what)                                                  \
+  do {                                                                      \
+    if ((expr) != 0) {                                                      \
+      std::lock_guard<std::mutex> lk(g_err_mu);                             \
+      g_last_err = std::string(what) + ": " + h->comm->err();               \
+      return SBR_ERR_NCCL;                                                  \
+    }                                                                       \
+  } while (0)
+
 #define SBR_CK(expr, what)                 \
   do {                                     \
     cudaError_t _e = (expr);               \
@@ -234,7 +246,15 @@ int latch_status(sbr_ctx* h, cudaStream_t st) {
 
 size_t align_up(size_t x) { return (x + 255) & ~size_t(255); }
 
-int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out) {
+// columns of the nb-blocks J with J % P == rank (1D block-cyclic, sbr_reduce_dist)
+int64_t local_cols(int64_t n, int nb, int P, int rank) {
+  int64_t c = 0;
+  for (int64_t c0 = (int64_t)rank * nb; c0 < n; c0 += (int64_t)P * nb) c += std::min<int64_t>(nb, n - c0);
+  return c;
+}
+
+int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out, int64_t shadow_cols = -1) {
+  if (shadow_cols < 0) shadow_cols = n;
   const int64_t M = n - b;
   const PanelWs pw = panel_ws_sizes(M, b);
   size_t off = 0;
@@ -249,20 +269,21 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
                oP = take((size_t)nb * 64), oG = take((size_t)nb * 64), oPv = take(pw.v), oPt = take(pw.tau),
                oPr = take(pw.r), oPq = take(pw.q), oPm = take(pw.misc), oF = take(64);
   // fp16 operands of the tensor-core path (sizes in floats = halves / 2)
-  const int64_t ldwh = (M + 7) / 8 * 8;       // TMA strides must be multiples of 16 bytes
+  // W copies: room for up to 128 zero rows in front (the multi-GPU pass's 128-aligned tile grid)
+  const int64_t ldwh = (M + 128 + 7) / 8 * 8;   // TMA strides must be multiples of 16 bytes
   // fp16 shadow: ld a multiple of 128 and a row offset `shoff` chosen so that every block's OA
   // origin (row/col c0 + b, c0 = J*nb) starts on a 256-byte boundary -- the pass streams
   // 128x128 tiles of it and unaligned tiles drag in neighbouring lines (L2 256 B promotion).
   const int64_t shoff = (nb % 128 == 0 && (128 - b % 128) % 8 == 0) ? (128 - b % 128) % 128 : 0;
   const int64_t ldsh = (n + shoff + 127) / 128 * 128;
   const int64_t ldk = (nb + 7) / 8 * 8;
-  const size_t oSh = take(((size_t)ldsh * n + shoff) / 2 + 128), oYh = take((size_t)n * ldk / 2 + 8),
+  const size_t oSh = take(((size_t)ldsh * shadow_cols + shoff) / 2 + 128), oYh = take((size_t)n * ldk / 2 + 8),
                oZh = take((size_t)n * ldk / 2 + 8), oWh = take((size_t)ldwh * 64 / 2 + 8),
                oWtXh = take((size_t)nb * ldk / 2 + 8), oXh = take((size_t)n * ldk / 2 + 8),
                oWrh = take((size_t)n * ldk / 2 + 8), oBl = take((size_t)64 * (2 * ldk + 128) / 2 + 8),
                oGh = take((size_t)ldk * 64 / 2 + 8), oHb = take((size_t)nb * 64), oGram = take(panel_chol_ws_bytes() / sizeof(float) + 64),
                oGH = take((size_t)2 * nb * nb), oPh = take((size_t)64 * ldk / 2 + 8),
-               oFz = take(chain_fused_ws_bytes() / sizeof(float) + 64);
+               oFz = take(chain_fused_ws_bytes() / sizeof(float) + 64), oABd = take((size_t)(b + 1) * n + 64);
   const int64_t tlo = (nb + 31) / 32 * 32, ldts = 2 * tlo, ldws = (M + 3) / 4 * 4;
   size_t oYS = 0, oZS = 0, oGS = 0, oWS = 0;
   if (mode == SBR_3XTF32) {
@@ -273,7 +294,8 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   }
   if (bytes_out) *bytes_out = off;
   if (!h) return SBR_OK;
-  if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb && h->ws_mode == mode)
+  if (h->ws && h->ws_bytes >= off && h->ws_n == n && h->ws_b == b && h->ws_nb == nb && h->ws_mode == mode &&
+      h->ws_shcols == shadow_cols)
     return SBR_OK;
   if (h->ws) {
     cudaFree(h->ws);
@@ -289,7 +311,9 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out)
   h->ws_b = b;
   h->ws_nb = nb;
   h->ws_mode = mode;
+  h->ws_shcols = shadow_cols;
   char* base = (char*)h->ws;
+  h->ABd = (float*)(base + oABd);
   h->Yb = (float*)(base + oY);
   h->Xb = (float*)(base + oX);
   h->Zb = (float*)(base + oZ);
@@ -358,38 +382,54 @@ bool panel_mode_default(const sbr_ctx* h) { return h->panel_mode == 0; }
 int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB, int64_t ldab,
                   float* W, int64_t ldw) {
   cudaStream_t st = h->stream;
-  // sbr_reduce_dist: every rank holds the full matrix; rank 0 ("lead") runs the sequential
-  // per-panel chain (a1-a3, a5) and owns the outputs, every rank streams its share of the
-  // per-panel pass (a4) and applies the trailing update (a6).  Exchanges per panel: broadcast
-  // of W_t (fp16, what the pass consumes) and all-reduce of the partial X_t; per block:
-  // broadcast of Y (fp16) and W^T X.  With nranks == 1 this is exactly sbr_reduce.
-  const bool lead = h->rank == 0;
-  const bool dist = h->comm != nullptr && (h->nranks > 1 || h->force_coll);
+  // sbr_reduce_dist (north star): 1D block-cyclic columns -- rank r holds the
+  // columns of the nb-blocks J with J % P == r (fp32 master A and fp16 shadow), local column
+  // (J / P) nb + (g - J nb).  The owner of block J factors all of its panels (the chain needs
+  // only its own columns) and broadcasts W_t (fp16) per panel; every rank streams the pass tiles
+  // of ITS columns and the partial X_t are summed by an all-reduce; per block the owner
+  // broadcasts Y (fp16) and W^T X, and every rank applies the trailing SYR2K to its own
+  // columns.  The band is assembled over the ranks at the end (rank 0 returns it).
+  const bool dist = h->comm != nullptr && h->nranks > 1;
+  const int P = dist ? h->nranks : 1, rank = dist ? h->rank : 0;
+  const bool lead = rank == 0;   // returns the band
+  ColMap cm;
+  cm.P = P;
+  cm.rank = rank;
+  cm.nbo = nb;
+  const int64_t ncols_loc = dist ? local_cols(n, nb, P, rank) : n;
+  auto owner = [&](int64_t c0) { return (int)((c0 / nb) % P); };
+  auto blk_ptr = [&](float* base, int64_t ld, int64_t c0) -> float* {   // global column indexing inside block c0 / nb
+    if (!dist || !base) return base;
+    const int64_t J = c0 / nb;
+    return base + ((J / P) * nb - J * nb) * ld;
+  };
   {   // errors latched by earlier reductions on this handle are returned by the next call (§8(b))
     const int lr = poll_latched(h, false);
     if (lr != SBR_OK) return lr;
   }
-  if (n <= b + 1) {
-    if (!lead) return SBR_OK;
+  if (n <= b + 1 && !dist) {
     Scope sc(h, SBR_K_OTHER, 0, 0);
     SBR_CK(extract_band(n, b, A, lda, AB, ldab, nullptr, nullptr, st), "extract_band");
     h->launches++;
     return SBR_OK;
   }
-  int rc = ensure_ws(h, n, b, nb, mode, nullptr);
+  int rc = ensure_ws(h, n, b, nb, mode, nullptr, ncols_loc);
   if (rc != SBR_OK) return rc;
   // status words flag[0..3] (input non-finite, declined tall panel, non-finite band), then the
-  // a0 scan: finiteness + ||A||_F -> the FP16 mode's power-of-two scale 2^k (kexp, device)
+  // a0 scan: finiteness + ||A||_F -> the power-of-two scale 2^k (kexp, device)
   unsigned* flag = h->flag;
-  double* fro2 = reinterpret_cast<double*>(h->flag + 8);
-  int* kexp = reinterpret_cast<int*>(h->flag + 10);
+  double* scan = reinterpret_cast<double*>(h->flag + 8);
+  int* kexp = reinterpret_cast<int*>(h->flag + 12);
   SBR_CK(cudaMemsetAsync(flag, 0, sizeof(unsigned) * 4, st), "zero status");
   {
-    Scope sc(h, SBR_K_OTHER, 2.0 * n * n, 2.0 * n * n);
-    SBR_CK(prep_scale(n, A, lda, flag, fro2, kexp, mode == SBR_FP16_FP32ACC, st), "prep_scale");
-    h->launches += (n + 65534) / 65535 + 1;
+    Scope sc(h, SBR_K_OTHER, 2.0 * n * ncols_loc, 2.0 * n * ncols_loc);
+    SBR_CK(prep_scan(n, ncols_loc, A, lda, cm, scan, st), "prep_scan");
+    if (dist) SBR_CM(h->comm->all_reduce_sum_f64(scan, 2, st), "all-reduce ||A||_F");
+    SBR_CK(choose_scale(scan, flag, kexp, st), "choose_scale");
+    h->launches += (ncols_loc + 65534) / 65535 + 1;
   }
-
+  if (n <= b + 1) goto band_out;
+  {
   const int64_t ncols = n - b;  // reflector columns 0 .. n-b-1
   const int64_t ldn = n;        // ld of the block buffers
   // the TMA-fed tensor-core kernels need 16-byte aligned tile origins (OA origin r0 = c0 + b):
@@ -400,26 +440,38 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   // TMA cannot address (lda % 4 != 0) and for the SBR_TF32_TC=0 ablation
   const bool tc32 = mode == SBR_3XTF32 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0 && b % 4 == 0 &&
                     nb % 4 == 0;
-  if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper)
-    Scope sc(h, SBR_K_OTHER, 6.0 * n * n, 0);
-    SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, kexp, st), "shadow_init");
-    h->launches += (n + 65534) / 65535;
+  if (dist && !tc16) {   // checked by sbr_reduce_dist
+    std::lock_guard<std::mutex> lk(g_err_mu);
+    g_last_err = "sbr_reduce_dist: FP16 mode with b, nb multiples of 8 only";
+    return SBR_ERR_UNSUPPORTED;
+  }
+  if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper) -- this rank's columns
+    Scope sc(h, SBR_K_OTHER, 6.0 * n * ncols_loc, 0);
+    SBR_CK(shadow_init(n, A, lda, h->Sh, h->ldsh, kexp, st, ncols_loc, cm), "shadow_init");
+    h->launches += (ncols_loc + 65534) / 65535;
   }
   if (!tc16) {  // a0 in 3xTF32 mode: the master scaled in place (FP16: inside shadow_init)
-    Scope sc(h, SBR_K_OTHER, 8.0 * n * n / 2, 0);
-    SBR_CK(scale_lower(n, A, lda, kexp, st), "scale_lower");
-    h->launches += (n + 65534) / 65535;
+    Scope sc(h, SBR_K_OTHER, 8.0 * n * ncols_loc / 2, 0);
+    SBR_CK(scale_lower(n, ncols_loc, A, lda, cm, kexp, st), "scale_lower");
+    h->launches += (ncols_loc + 65534) / 65535;
   }
-  if (tc16) {  // fp16 W copies: pad columns (b < BN) must read as zero in the pass
+  if (tc16) {  // fp16 W copies: pad columns (b < BN) and the pad rows in front must read as zero in the pass
     SBR_CK(cudaMemsetAsync(h->Wh, 0, sizeof(__half) * h->ldwh * 64, st), "zero Wh");
   }
+  // multi-GPU pass grid: 128-aligned tile origin c0 (nb % 1024 == 0), OA rows start `off` = b rows
+  // into it; the W copies the pass reads carry `off` zero rows in front (the chain writes Whc)
+  const int off = dist ? b : 0;
+  __half* const Whc = h->Wh + off;
   for (int64_t c0 = 0; c0 < ncols; c0 += nb) {
     const int64_t r0 = c0 + b, M = n - r0;
     const int kJ = (int)std::min<int64_t>(nb, ncols - c0);
     const int p = (kJ + b - 1) / b;
-    float* Wb = W ? W + r0 + c0 * ldw : h->Wws;
+    const int own = owner(c0);
+    const bool leadJ = own == rank;               // this rank factors block J's panels
+    float* const AJ = blk_ptr(A, lda, c0);        // global column indexing inside block J (its owner only)
+    float* Wb = W ? blk_ptr(W, ldw, c0) + r0 + c0 * ldw : h->Wws;
     const int64_t ldwb = W ? ldw : ldn;
-    float* OA = A + r0 + r0 * lda;
+    float* OA = AJ + r0 + r0 * lda;
     const int sw = std::min<int64_t>((int64_t)(p - 1) * b, M);  // OA columns rewritten during the block
     if (sw > 0 && !tc16) {  // tc32: whole 128-column tiles of the strip
       const int64_t swc = tc32 ? std::min<int64_t>((sw + 127) / 128 * 128, M) : sw;
@@ -435,12 +487,44 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       SBR_CK(cudaMemsetAsync(h->GH, 0, sizeof(float) * 2 * nb * nb, st), "zero G/H");
     }
     // fused FP16 chain (k_chain_fused.cu): one cooperative launch per panel + the pass
-    const bool fused = tc16 && h->fused && !dist && panel_mode_default(h) && nb <= 1024 &&
-                       chain_fused_supported(b, M, h->nsm);
+    const bool fused = tc16 && h->fused && panel_mode_default(h) && nb <= 1024 && chain_fused_supported(b, M, h->nsm);
+    // ---- a4 for panel t on every rank: W_t from the owner (dist), the pass over this rank's
+    //      tiles (the 128-aligned grid of its column blocks when distributed), X_t summed
+    auto pass_t = [&](int64_t tb) -> int {
+      if (dist) SBR_CM(h->comm->broadcast(h->Wh, (size_t)h->ldwh * pass_bn(b) * sizeof(__half), own, st),
+                       "broadcast W_t");
+      {
+        Scope sc(h, SBR_K_PASS, (1.0 * M * M + 6.0 * M * b) / P, 2.0 * M * M * b / P);
+        PassLaunch pl{};
+        pl.shadow = h->Sh;
+        pl.n = n;
+        pl.ld_shadow = h->ldsh;
+        pl.Wh = h->Wh;
+        pl.M = M;
+        pl.ld_wh = h->ldwh;
+        pl.r0 = dist ? c0 : r0;
+        pl.off = off;
+        pl.b = b;
+        pl.X = h->Xb + tb * M;
+        pl.ldx = M;
+        pl.num_sms = h->nsm;
+        pl.seg_rows = 8;
+        if (dist) {
+          pl.own_P = P;
+          pl.own_rank = rank;
+          pl.nbo = nb;
+          pl.shadow_cols = ncols_loc;
+        }
+        SBR_CK(launch_pass_tc(pl, st), "pass_tc");
+        h->launches += 1;
+      }
+      if (dist) SBR_CM(h->comm->all_reduce_sum_f32(h->Xb + tb * M, (size_t)M * b, st), "all-reduce X_t");
+      return SBR_OK;
+    };
     for (int t = 0; fused && t < p; ++t) {
       const int64_t tb = (int64_t)t * b;
       float* Wt = Wb + tb * ldwb;
-      {
+      if (leadJ) {
         Scope sc(h, SBR_K_PANEL, 4.0 * (M - tb) * b * 4 + (t ? 8.0 * M * b + 4.0 * (M - tb) * t * b * 5 : 0),
                  4.0 * (M - tb) * b * b * 2 + (t ? 10.0 * M * t * b * b : 0));
         ChainFusedLaunch L{};
@@ -448,7 +532,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         L.k = t * b;
         L.M = M;
         L.tb = tb;
-        L.A = A;
+        L.A = AJ;
         L.lda = lda;
         L.r0 = r0;
         L.Yb = h->Yb;
@@ -466,7 +550,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         L.Yh = h->Yh;
         L.Wrh = h->Wrh;
         L.ldk = h->ldk;
-        L.Wh = h->Wh;
+        L.Wh = Whc;
         L.ldwh = h->ldwh;
         L.ws = h->fused_ws;
         L.launch = h->fused_launches;
@@ -484,25 +568,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         h->fused_launches++;
         h->launches += 1;
       }
-      {  // ---- a4: pass X_t = OA W_t
-        Scope sc(h, SBR_K_PASS, (1.0 * M * M + 6.0 * M * b), 2.0 * M * M * b);
-        PassLaunch pl{};
-        pl.shadow = h->Sh;
-        pl.n = n;
-        pl.ld_shadow = h->ldsh;
-        pl.Wh = h->Wh;
-        pl.M = M;
-        pl.ld_wh = h->ldwh;
-        pl.r0 = r0;
-        pl.b = b;
-        pl.X = h->Xb + tb * M;
-        pl.ldx = M;
-        pl.num_sms = h->nsm;
-        pl.seg_rows = 8;
-        SBR_CK(launch_pass_tc(pl, st), "pass_tc");
-        h->launches += 1;
-      }
-      if (t == p - 1) {  // the last panel's pass tail (the next fused launch does it otherwise)
+      if (int prc = pass_t(tb)) return prc;
+      if (t == p - 1 && leadJ) {  // the last panel's pass tail (the next fused launch does it otherwise)
         Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
         SBR_CK(launch_postpass(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb, st),
                "postpass");
@@ -520,8 +587,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       if (t >= 1) {  // ---- a5: lazy update of panel t's columns (Alg.1 l.8-10)
         const int64_t c = tb - b;  // OA column of the panel's first column
         const int64_t rows = M - c;
-        float* Ablk = A + g + g * lda;
-        if (tc16 && !lead) {
+        float* Ablk = AJ + g + g * lda;
+        if (tc16 && !leadJ) {
           // not this rank's step
         } else if (tc16) {  // P = W^T R (SIMT), then GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
           Scope sc(h, SBR_K_LAZY, 2.0 * rows * 2.0 * k + 8.0 * rows * b, 4.0 * rows * k * b);
@@ -574,10 +641,10 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           h->launches += 4;
         }
       }
-      if (lead) {  // ---- a1/a2: TSQR + reconstruction
+      if (leadJ) {  // ---- a1/a2: TSQR + reconstruction
         Scope sc(h, SBR_K_PANEL, 4.0 * m * b * 4, 4.0 * m * b * b * 2);
         PanelArgs pa{};
-        pa.P = A + (g + b) + g * lda;
+        pa.P = AJ + (g + b) + g * lda;
         pa.ldp = lda;
         pa.m = (int)m;
         pa.b = b;
@@ -589,7 +656,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.M = M;
         pa.Yh = tc16 ? h->Yh + tb : nullptr;
         pa.ldyh = h->ldk;
-        pa.Wh = tc16 ? h->Wh : nullptr;        // W^0 (fp16, column-major): pass operand / merge B
+        pa.Wh = tc16 ? Whc : nullptr;          // W^0 (fp16, column-major): pass operand / merge B
         pa.ldwh = h->ldwh;
         pa.Wrh = (tc16 && t == 0) ? h->Wrh : nullptr;   // W_0 = W^0 (row-major): later merges
         pa.ldwrh = h->ldk;
@@ -632,7 +699,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         }
       }
       if (tc16) {
-        if (t >= 1 && lead) {
+        if (t >= 1 && leadJ) {
           // ---- a3 on tcgen05: G = Y^T W0, H = X^T W0 (one pass over Y, X); W^T X_t = H - (W^T X) G;
           //      W_t = W0 - W G, written as fp32 + fp16 (column-major for the pass, row-major for later merges)
           Scope sc(h, SBR_K_WMERGE, 2.0 * (M - tb) * 2.0 * k + 2.0 * M * k + 12.0 * M * b,
@@ -643,7 +710,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           q.K1 = k;
           q.a_rows = M;
           q.lda = h->ldk;
-          q.B = h->Wh;
+          q.B = Whc;
           q.b_rows = M;
           q.ldb = h->ldwh;
           q.row0 = tb;
@@ -685,40 +752,16 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           mq.ldc = ldwb;
           mq.D = Wt;
           mq.ldd = ldwb;
-          mq.Hcm = h->Wh;
+          mq.Hcm = Whc;
           mq.ldhc = h->ldwh;
           mq.Hrm = h->Wrh + tb;
           mq.ldhr = h->ldk;
           SBR_CK(launch_skinny_nn(mq, st), "W merge");
           h->launches += 3;
         }
-        if (dist) {  // W_t (fp16, column-major) from the lead to every rank
-          SBR_NC(nccl::broadcast(h->Wh, (size_t)h->ldwh * b, nccl::kFloat16, 0, h->comm, st), "broadcast W_t");
-        }
-        {  // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA); X_t zeroed at block start
-          Scope sc(h, SBR_K_PASS, (1.0 * M * M + 6.0 * M * b) / h->nranks, 2.0 * M * M * b / h->nranks);
-          PassLaunch pl{};
-          pl.shadow = h->Sh;
-          pl.n = n;
-          pl.ld_shadow = h->ldsh;
-          pl.Wh = h->Wh;
-          pl.M = M;
-          pl.ld_wh = h->ldwh;
-          pl.r0 = r0;
-          pl.b = b;
-          pl.X = h->Xb + tb * M;
-          pl.ldx = M;
-          pl.num_sms = h->nsm;
-          pl.seg_rows = 8;
-          pl.rank = h->rank;
-          pl.nranks = h->nranks;
-          SBR_CK(launch_pass_tc(pl, st), "pass_tc");
-          h->launches += 1;
-        }
-        if (dist) {  // partial passes -> X_t on every rank
-          SBR_NC(nccl::all_reduce_sum_f32(h->Xb + tb * M, (size_t)M * b, h->comm, st), "all-reduce X_t");
-        }
-        if (lead) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block)
+        // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA); X_t zeroed at block start
+        if (int prc = pass_t(tb)) return prc;
+        if (leadJ) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block)
           Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
           SBR_CK(launch_postpass(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb,
                                  st),
@@ -779,9 +822,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int64_t s = (int64_t)p * b - b;
     const int64_t Mt = M - s;
     const int kk = p * b;
-    if (Mt > 0 && tc16 && dist) {   // the lead's Y (fp16) and W^T X for every rank's trailing update
-      SBR_NC(nccl::broadcast(h->Yh, (size_t)M * h->ldk, nccl::kFloat16, 0, h->comm, st), "broadcast Y");
-      SBR_NC(nccl::broadcast(h->WtX, (size_t)nb * nb, nccl::kFloat32, 0, h->comm, st), "broadcast W^T X");
+    if (Mt > 0 && tc16 && dist) {   // the owner's Y (fp16) and W^T X for every rank's trailing update
+      SBR_CM(h->comm->broadcast(h->Yh, (size_t)M * h->ldk * sizeof(__half), own, st), "broadcast Y");
+      SBR_CM(h->comm->broadcast(h->WtX, (size_t)nb * nb * sizeof(float), own, st), "broadcast W^T X");
     }
     if (Mt > 0 && tc16) {
       Scope sc(h, SBR_K_SYR2K, 10.0 * Mt * Mt / 2 + 2.0 * Mt * kk * 4 + 4.0 * Mt * kk,
@@ -815,11 +858,17 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       gs.ld_a = gs.ld_b = h->ldk;
       gs.arow0 = gs.brow0 = s;
       gs.Mrows = gs.Ncols = Mt;
-      gs.C = A + (r0 + s) + (r0 + s) * lda;
+      gs.C = A + (r0 + s) + (dist ? 0 : (r0 + s) * lda);   // distributed: local columns via the ownership map
       gs.ldc = lda;
-      gs.shadow = h->Sh + (r0 + s) + (r0 + s) * h->ldsh;
+      gs.shadow = h->Sh + (r0 + s) + (dist ? 0 : (r0 + s) * h->ldsh);
       gs.ld_shadow = h->ldsh;
       gs.num_sms = h->nsm;
+      if (dist) {   // this rank's columns of the trailing region only
+        gs.own_P = P;
+        gs.own_rank = rank;
+        gs.own_org = r0 + s;
+        gs.nbo = nb;
+      }
       SBR_CK(launch_syr2k_tc(gs, st), "syr2k_tc");
       h->launches += 3;
     } else if (Mt > 0 && tc32) {   // a6 in 3xTF32 on tcgen05: split Y, W^T X; Z (split) ; SYR2K
@@ -870,9 +919,22 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       h->launches += 2;
     }
   }
-  if (lead) {
+  }
+band_out:
+  if (!dist) {
     Scope sc(h, SBR_K_OTHER, 8.0 * (b + 1) * n, 0);
     SBR_CK(extract_band(n, b, A, lda, AB, ldab, kexp, flag, st), "extract_band");
+    h->launches += 1;
+  } else {   // each rank its own columns of the band, summed over the ranks; rank 0 returns it
+    Scope sc(h, SBR_K_OTHER, 8.0 * (b + 1) * n, 0);
+    SBR_CK(cudaMemsetAsync(h->ABd, 0, sizeof(float) * (b + 1) * n, st), "zero band");
+    SBR_CK(extract_band(n, b, A, lda, h->ABd, b + 1, n <= b + 1 ? nullptr : kexp, flag, st, ncols_loc, cm),
+           "extract_band");
+    SBR_CM(h->comm->all_reduce_sum_f32(h->ABd, (size_t)(b + 1) * n, st), "all-reduce band");
+    if (lead && AB)
+      SBR_CK(cudaMemcpy2DAsync(AB, ldab * sizeof(float), h->ABd, (b + 1) * sizeof(float), (b + 1) * sizeof(float), n,
+                               cudaMemcpyDeviceToDevice, st),
+             "band out");
     h->launches += 1;
   }
   return latch_status(h, st);   // errors found on the device are reported by sbr_sync / the next call
@@ -1006,7 +1068,7 @@ int sbr_destroy(sbr_handle_t h) {
   cudaSetDevice(h->device);
   cudaStreamSynchronize(h->stream);
   drain_stats(h);
-  if (h->comm) nccl::comm_destroy(h->comm);
+  delete h->comm;
   for (auto e : h->ev_pool) cudaEventDestroy(e);
   if (h->ws) cudaFree(h->ws);
   if (h->e2e) cudaFree(h->e2e);
@@ -1099,34 +1161,20 @@ int sbr_get_unique_id(void* id) {
   return SBR_OK;
 }
 
-int sbr_create_dist(sbr_handle_t* out, int device, void* stream, const void* unique_id, int rank, int nranks) {
-  if (!out) return -1;
-  if (!unique_id) return -4;
-  if (nranks < 1) return -6;
-  if (rank < 0 || rank >= nranks) return -5;
+static int create_dist_common(sbr_handle_t* out, int device, void* stream, int rank, int nranks,
+                              const std::function<sbr::Comm*(std::string*)>& make) {
   int rc = sbr_create(out, device, stream);
   if (rc != SBR_OK) return rc;
   sbr_ctx* h = *out;
   h->rank = rank;
   h->nranks = nranks;
-  const char* fc = getenv("SBR_DIST_COLLECTIVES");
-  h->force_coll = fc && strcmp(fc, "1") == 0;
-  if (const char* e = nccl::load()) {
-    std::lock_guard<std::mutex> lk(g_err_mu);
-    g_last_err = e;
-    sbr_destroy(h);
-    *out = nullptr;
-    return SBR_ERR_NCCL;
-  }
-  nccl::UniqueId u;
-  memcpy(&u, unique_id, sizeof(u));
-  const int r = nccl::comm_init_rank(&h->comm, nranks, u, rank);
-  if (r != 0) {
+  std::string msg;
+  h->comm = make(&msg);
+  if (!h->comm) {
     {
       std::lock_guard<std::mutex> lk(g_err_mu);
-      g_last_err = std::string("ncclCommInitRank: ") + nccl::error_string(r);
+      g_last_err = msg;
     }
-    h->comm = nullptr;
     sbr_destroy(h);
     *out = nullptr;
     return SBR_ERR_NCCL;
@@ -1134,15 +1182,49 @@ int sbr_create_dist(sbr_handle_t* out, int device, void* stream, const void* uni
   return SBR_OK;
 }
 
+int sbr_create_dist(sbr_handle_t* out, int device, void* stream, const void* unique_id, int rank, int nranks) {
+  if (!out) return -1;
+  if (!unique_id) return -4;
+  if (nranks < 1) return -6;
+  if (rank < 0 || rank >= nranks) return -5;
+  return create_dist_common(out, device, stream, rank, nranks, [&](std::string* msg) {
+    return sbr::make_nccl_comm(unique_id, rank, nranks, msg);
+  });
+}
+
+int sbr_create_dist_local(sbr_handle_t* out, int device, void* stream, int group, int rank, int nranks) {
+  if (!out) return -1;
+  if (nranks < 1 || nranks > 16) return -6;
+  if (rank < 0 || rank >= nranks) return -5;
+  SBR_CK(cudaSetDevice(device), "cudaSetDevice");
+  return create_dist_common(out, device, stream, rank, nranks, [&](std::string* msg) {
+    return sbr::make_local_comm(group, rank, nranks, msg);
+  });
+}
+
+int64_t sbr_local_cols(int64_t n, int nb, int rank, int nranks) {
+  if (n < 0 || nb < 1 || nranks < 1 || rank < 0 || rank >= nranks) return -1;
+  return local_cols(n, nb, nranks, rank);
+}
+
 int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, float* AB,
                     int64_t ldab, float* W, int64_t ldw) {
   if (!h) return -1;
   const bool lead = h->rank == 0;
-  // outputs are produced on rank 0 only; other ranks may pass AB = W = NULL
+  // outputs: the band on rank 0 (other ranks may pass AB = NULL); W_local on every rank (or NULL)
   int rc = validate(h, mode, n, b, nb, A, lda, lead ? AB : A, ldab < b + 1 && !lead ? b + 1 : ldab, W, ldw);
   if (rc != SBR_OK) return rc;
-  if (h->nranks > 1 && mode != SBR_FP16_FP32ACC) return SBR_ERR_UNSUPPORTED;
-  if (h->nranks > 1 && !h->comm) return SBR_ERR_NCCL;
+  if (h->nranks > 1) {
+    if (!h->comm) return SBR_ERR_NCCL;
+    // the tensor-core FP16 path with column blocks that align with the pass's tile groups and the
+    // SYR2K's tiles (configs 4/5: nb = 1024 / 2048)
+    if (mode != SBR_FP16_FP32ACC || b % 8 != 0 || nb % pass_dist_align(b) != 0 || nb % 256 != 0) {
+      std::lock_guard<std::mutex> lk(g_err_mu);
+      g_last_err = "sbr_reduce_dist with nranks > 1: FP16 mode, b % 8 == 0, nb a multiple of " +
+                   std::to_string(pass_dist_align(b));
+      return SBR_ERR_UNSUPPORTED;
+    }
+  }
   SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
   return reduce_device(h, mode, n, b, nb, A, lda, AB, ldab, W, ldw);
 }
@@ -1588,6 +1670,13 @@ extern "C" int sbr_test_pass_partition(int64_t M, int b, int rank, int nranks, i
   if (!t0 || !t1 || !total) return -5;
   pass_partition(M, b, rank, nranks, t0, t1, total);
   return SBR_OK;
+}
+
+// host-only: the pass tiles `rank` of `nranks` walks for block origin c0 in sbr_reduce_dist
+extern "C" int64_t sbr_test_pass_owned_tiles(int64_t n, int b, int nb, int64_t c0, int rank, int nranks, int* IJ,
+                                             int64_t cap) {
+  if (n < 1 || b < 1 || b > 64 || nb < b || nranks < 1 || rank < 0 || rank >= nranks || c0 < 0 || c0 + b >= n) return -1;
+  return pass_owned_tiles(n - c0 - b, b, c0, b, nb, nranks, rank, IJ, cap);
 }
 
 // host-only: (I, J) tile coordinates of tiles [t0, t1) in the pass's order, IJ[2k], IJ[2k+1]
