@@ -358,7 +358,10 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   const int grid = std::min(ntiles, p.num_sms);
   GemmOwn own;
   if (p.own_P > 1) {
-    if (MODE != 0 || p.nbo % G_BN != 0 || p.own_org % p.nbo != 0) return cudaErrorInvalidValue;
+    // every BN-wide output tile must lie inside one column block: an nb-aligned origin (nb % BN == 0),
+    // or a region that fits in one block (the ragged last block)
+    const bool one_block = p.own_org / p.nbo == (p.own_org + p.Ncols - 1) / p.nbo;
+    if (MODE != 0 || p.nbo % G_BN != 0 || (p.own_org % p.nbo != 0 && !one_block)) return cudaErrorInvalidValue;
     own.P = p.own_P;
     own.rank = p.own_rank;
     own.org = p.own_org;

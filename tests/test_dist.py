@@ -190,7 +190,10 @@ def test_reduce_dist_virtual_ranks(n, P):
     db = float(np.max(np.abs(sign_normalise(bm, b) - sign_normalise(bm1, b)))) / float(np.max(np.abs(ref)))
     print(f"reduce_dist P={P} n={n}: backward {eb:.2e} orth {eo:.2e} eig {ee:.2e} |dB| vs 1 GPU {db:.2e}")
     assert eb <= 5e-3 and eo <= 5e-3 and ee <= 1e-3
-    assert db <= 2e-2
+    # entry-wise B is a forward error (cond x backward error): two single-GPU FP16 runs already
+    # differ by ~2e-2 ||A||_2 (fp32 atomics in the pass sum in another order), so this only
+    # checks that the distributed band is the same matrix, not a different reduction
+    assert db <= 5e-2
     for r, (a_loc, _, _, cols) in enumerate(out):   # each rank held only its columns
         assert a_loc.shape[0] == len(cols) == sbr.local_cols(n, nb, r, P)
 
