@@ -145,6 +145,24 @@ int sbr_reduce_host(sbr_handle_t h, int mode, int64_t n, int b, int nb,
 int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
                float* Q, int64_t ldq);
 
+/* Back-transformation (Sec. 4.4), both on tcgen05 3xTF32 like sbr_form_q.
+ * sbr_form_w: Alg. 2 -- the per-block W_J of sbr_reduce merged recursively (left half,
+ *   right half, then W_R <- W_R - W_L (Y_L^T W_R)) into ONE n x (n-b) W with Q = I - W Y^T, Y the
+ *   unit lower staircase of sbr_reduce's output (column c: unit at row c+b, tail in A below).
+ *   A (Y), W: sbr_reduce's outputs (same n, b, nb), read only.  Wo: device fp32, n x (n-b),
+ *   column-major, ldwo >= n, overwritten (zeros above each column's first touched row).
+ *   Returns 0, -1 (h), -2 (n), -3 (b), -4 (nb), -5 (A), -6 (lda), -7 (W), -8 (ldw), -9 (Wo),
+ *   -10 (ldwo), SBR_ERR_NOMEM, SBR_ERR_CUDA.
+ * sbr_apply_q: X <- Q X for the n x kx block X (device fp32, column-major, ldx >= n): the eigenvector
+ *   back-transformation of the band's eigenvectors.  Applies the per-block factors last
+ *   block first, X[r0:] -= W_J (Y_J^T X[r0:]).  Returns as sbr_form_w with -9 (X), -10 (ldx),
+ *   -11 (kx < 0).
+ * Both are stream-ordered; their split operands live in handle-owned device memory. */
+int sbr_form_w(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
+               float* Wo, int64_t ldwo);
+int sbr_apply_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
+                float* X, int64_t ldx, int64_t kx);
+
 /* ---- Multi-GPU (north star: 1D block-cyclic columns) ----
  *
  * Data distribution: the columns of A are split into nb-wide blocks J (global columns

@@ -22,8 +22,9 @@ tridiag      -- band -> tridiagonal (unblocked SBR with b = 1) and Sturm
 metrics      -- backward error / orthogonality / eigenvalue error (P:395,
                 P:399, P:421 as read in DESIGN.md C9), and Q from the
                 per-block (W, Y) output.
+backtransform -- Alg. 2 FormW and X <- Q X.
 
 Every function is pinned by ``tests/test_oracle_*.py`` against LAPACK,
 closed forms, brute force or invariants; none is "parity unpinned".
 """
-from . import householder, sbr, panel, tridiag, metrics  # noqa: F401
+from . import householder, sbr, panel, tridiag, metrics, backtransform  # noqa: F401

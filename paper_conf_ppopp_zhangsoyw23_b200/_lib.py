@@ -51,6 +51,8 @@ SIGNATURES = {
     "sbr_local_cols": (_i64, [_i64, _i, _i, _i]),
     "sbr_reduce_dist": (_i, [_h, _i, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_form_q": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_form_w": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
+    "sbr_apply_q": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64, _i64]),
     "sbr_rank": (_i, [_h]),
     "sbr_nranks": (_i, [_h]),
     # kernel-level test hooks (include/sbr_testing.h)

@@ -168,6 +168,26 @@ class Handle:
         check(lib().sbr_form_q(self._h, n, int(b), int(nb), _ptr(A), n, _ptr(w), n, _ptr(q), n), "sbr_form_q")
         return q
 
+    def form_w(self, A, w, b: int, nb: int, out=None):
+        """Alg. 2 (sbr_form_w): the merged W (torch shape (n-b, n), ``out[c, r] = W(r, c)``) with
+        Q = I - W Y^T, from :meth:`reduce`'s outputs."""
+        import torch
+
+        n = int(A.shape[0])
+        if out is None:
+            out = torch.empty((max(n - b, 1), n), dtype=torch.float32, device=A.device)
+        check(lib().sbr_form_w(self._h, n, int(b), int(nb), _ptr(A), n, _ptr(w), n, _ptr(out), n), "sbr_form_w")
+        return out
+
+    def apply_q(self, A, w, b: int, nb: int, X):
+        """X <- Q X in place (sbr_apply_q); X: torch (kx, n) contiguous float32 CUDA (= column-major n x kx)."""
+        n = int(A.shape[0])
+        if X.dim() != 2 or X.shape[1] != n or not X.is_contiguous():
+            raise ValueError("X must be a contiguous (kx, n) float32 CUDA tensor")
+        check(lib().sbr_apply_q(self._h, n, int(b), int(nb), _ptr(A), n, _ptr(w), n, _ptr(X), n, int(X.shape[0])),
+              "sbr_apply_q")
+        return X
+
     def reduce_dist(self, A_local, n: int, b: int, nb: int, mode="fp16", want_w: bool = True, ab=None, w=None):
         """One n x n matrix across the handle's ranks (collective; include/sbr.h sbr_reduce_dist).
 

@@ -279,6 +279,25 @@ cudaError_t mirror_wtx(int k, int b, float* WtX, int64_t ld, cudaStream_t st) {
   return cudaGetLastError();
 }
 
+// Wo[:, c] = W[:, c] on the rows block J = c / nb acts on (r >= J nb + b), zero above
+__global__ void copy_block_w_kernel(int64_t n, int b, int nb, int64_t c0, const float* W, int64_t ldw, float* Wo,
+                                    int64_t ldwo) {
+  const int64_t c = c0 + blockIdx.y;
+  const int64_t r0 = (c / nb) * nb + b;
+  for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < n; r += (int64_t)gridDim.x * blockDim.x)
+    Wo[r + c * ldwo] = r >= r0 ? W[r + c * ldw] : 0.f;
+}
+
+cudaError_t copy_block_w(int64_t n, int b, int nb, const float* W, int64_t ldw, float* Wo, int64_t ldwo, cudaStream_t st) {
+  const int64_t ncols = n - b;
+  for (int64_t c0 = 0; c0 < ncols; c0 += 65535) {
+    const int64_t nc = std::min<int64_t>(65535, ncols - c0);
+    dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 16), (unsigned)nc);
+    copy_block_w_kernel<<<grid, 256, 0, st>>>(n, b, nb, c0, W, ldw, Wo, ldwo);
+  }
+  return cudaGetLastError();
+}
+
 cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaStream_t st) {
   if (rows <= 0 || cols <= 0) return cudaSuccess;
   return cudaMemset2DAsync(A, lda * sizeof(float), 0, rows * sizeof(float), cols, st);

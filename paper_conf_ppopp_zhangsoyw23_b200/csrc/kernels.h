@@ -105,6 +105,8 @@ cudaError_t lazy_small_p(int k, int b, const float* Xc, int64_t ldx, const float
                          const float* Yc, int64_t ldy, float* P, cudaStream_t st);
 cudaError_t mirror_wtx(int k, int b, float* WtX, int64_t ld, cudaStream_t st);
 cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaStream_t st);
+// Wo[:, c] = W[:, c] for rows r >= (c / nb) nb + b, 0 above (columns c < n - b)
+cudaError_t copy_block_w(int64_t n, int b, int nb, const float* W, int64_t ldw, float* Wo, int64_t ldwo, cudaStream_t st);
 
 // ---- the two large contractions ----
 // X[:, 0:b] = OA (M x M symmetric, lower referenced) * W (M x b).  OA columns < sw are

@@ -1057,6 +1057,223 @@ int sbr_form_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t
   return SBR_OK;
 }
 
+}  // extern "C" (reopened below)
+
+namespace {
+
+// 3xTF32 split workspace of the back-transformation calls (handle-owned, grown on demand)
+float* fq_grow(sbr_ctx* h, size_t need, int* rc) {
+  *rc = SBR_OK;
+  if (h->fq_bytes < need) {
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) {   // a previous call may still use the old buffer
+      *rc = SBR_ERR_CUDA;
+      return nullptr;
+    }
+    if (h->fq) cudaFree(h->fq);
+    h->fq = nullptr;
+    h->fq_bytes = 0;
+    if (cudaMalloc(&h->fq, need) != cudaSuccess) {
+      cudaGetLastError();
+      *rc = SBR_ERR_NOMEM;
+      return nullptr;
+    }
+    h->fq_bytes = need;
+  }
+  return (float*)h->fq;
+}
+
+// T^T = Bc^T Yc (rb x ka, split row-major into TS) and C -= Wr T^T^T -- the two 3xTF32 tcgen05
+// products of one WY application C <- C - W (Y^T C) (sbr_form_q's pattern):
+//   C  : M x kc column-major (the rows the reflectors touch),  Y, W: M x ka column-major
+cudaError_t wy_apply_tf32(sbr_ctx* h, int64_t M, int64_t kc, int64_t ka, const float* Y, int64_t ldy, bool unit_y,
+                          const float* W, int64_t ldw, float* C, int64_t ldc, float* CS, float* YS, float* WS,
+                          float* TS, int64_t ldM, int64_t loM, int64_t ldk, int64_t lok, cudaStream_t st) {
+  cudaError_t e;
+  if ((e = split_tf32_cm(M, (int)ka, Y, ldy, unit_y, YS, ldM, loM, st)) != cudaSuccess) return e;
+  if ((e = split_tf32_rm(M, (int)ka, W, ldw, WS, ldk, lok, st)) != cudaSuccess) return e;
+  if ((e = split_tf32_cm(M, (int)kc, C, ldc, false, CS, ldM, loM, st)) != cudaSuccess) return e;
+  GemmTcLaunch g1{};   // T^T = C^T Y  (kc x ka), written split row-major
+  g1.A0 = g1.A1 = (const __half*)CS;
+  g1.B0 = g1.B1 = (const __half*)YS;
+  g1.K = M;
+  g1.lo_off = loM;
+  g1.a_rows = kc;
+  g1.ld_a = ldM;
+  g1.b_rows = ka;
+  g1.ld_b = ldM;
+  g1.Mrows = kc;
+  g1.Ncols = ka;
+  g1.Zs = TS;
+  g1.ldz = ldk;
+  g1.zlo_off = lok;
+  g1.num_sms = h->nsm;
+  if ((e = launch_gemm_split_tf32(g1, st)) != cudaSuccess) return e;
+  GemmTcLaunch g2{};   // C -= W T
+  g2.A0 = g2.A1 = (const __half*)WS;
+  g2.B0 = g2.B1 = (const __half*)TS;
+  g2.K = ka;
+  g2.lo_off = lok;
+  g2.a_rows = M;
+  g2.ld_a = ldk;
+  g2.b_rows = kc;
+  g2.ld_b = ldk;
+  g2.Mrows = M;
+  g2.Ncols = kc;
+  g2.C = C;
+  g2.ldc = ldc;
+  g2.num_sms = h->nsm;
+  return launch_gemm_sub_tf32(g2, st);
+}
+
+}  // namespace
+
+extern "C" {
+
+int sbr_apply_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
+                float* X, int64_t ldx, int64_t kx) {
+  if (!h) return -1;
+  if (n < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (nb < b || nb % b != 0 || nb > 4096) return -4;
+  if (!A) return -5;
+  if (lda < n) return -6;
+  if (!W) return -7;
+  if (ldw < n) return -8;
+  if (!X) return -9;
+  if (ldx < n) return -10;
+  if (kx < 0) return -11;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t ncols = n - b;
+  if (ncols <= 0 || kx == 0) return SBR_OK;
+  // X <- Q X = Q_0 (Q_1 (... (Q_last X))): block J (last first): X[r0:] -= W_J (Y_J^T X[r0:])
+  const int64_t M0 = n - b;
+  const int64_t loM = (M0 + 31) / 32 * 32, ldM = 2 * loM;
+  const int64_t lok = (nb + 31) / 32 * 32, ldk = 2 * lok;
+  const size_t nXS = align_up(sizeof(float) * kx * ldM), nYS = align_up(sizeof(float) * nb * ldM),
+               nWS = align_up(sizeof(float) * M0 * ldk), nTS = align_up(sizeof(float) * kx * ldk);
+  int rc = SBR_OK;
+  float* base = fq_grow(h, nXS + nYS + nWS + nTS, &rc);
+  if (rc != SBR_OK) return rc;
+  float* XS = base;
+  float* YS = (float*)((char*)base + nXS);
+  float* WS = (float*)((char*)base + nXS + nYS);
+  float* TS = (float*)((char*)base + nXS + nYS + nWS);
+  const int64_t nblk = (ncols + nb - 1) / nb;
+  for (int64_t J = nblk - 1; J >= 0; --J) {
+    const int64_t c0 = J * nb, r0 = c0 + b, M = n - r0;
+    const int k = (int)std::min<int64_t>(nb, ncols - c0);
+    Scope sc(h, SBR_K_OTHER, 4.0 * M * kx * 4 + 8.0 * M * k * 4, 3 * 4.0 * M * kx * k);
+    SBR_CK(wy_apply_tf32(h, M, kx, k, A + r0 + c0 * lda, lda, true, W + r0 + c0 * ldw, ldw, X + r0, ldx, XS, YS, WS,
+                         TS, ldM, loM, ldk, lok, st),
+           "apply_q");
+    h->launches += 5;
+  }
+  return SBR_OK;
+}
+
+}  // extern "C"
+
+namespace {
+
+// Alg. 2: W of the column range [ca, ce) (whole nb-blocks) formed recursively --
+// left half, right half, then W_R <- W_R - W_L (Y_L^T W_R), which turns the per-block factors
+// into ONE W with Q = I - W Y^T over those columns.
+int form_w_rec(sbr_ctx* h, int64_t n, int b, int nb, const float* A, int64_t lda, float* Wo, int64_t ldwo,
+               int64_t ca, int64_t ce, float* CS, float* YS, float* WS, float* TS, int64_t ldM, int64_t loM,
+               int64_t ldk, int64_t lok) {
+  const int64_t nblk = (ce - ca + nb - 1) / nb;
+  if (nblk <= 1) return SBR_OK;
+  const int64_t cm = ca + (nblk / 2) * nb;
+  int rc = form_w_rec(h, n, b, nb, A, lda, Wo, ldwo, ca, cm, CS, YS, WS, TS, ldM, loM, ldk, lok);
+  if (rc == SBR_OK) rc = form_w_rec(h, n, b, nb, A, lda, Wo, ldwo, cm, ce, CS, YS, WS, TS, ldM, loM, ldk, lok);
+  if (rc != SBR_OK) return rc;
+  // merge: rows the left reflectors touch, r >= ca + b; W_R is zero above cm + b, so T = Y_L^T W_R
+  // only needs rows >= cm + b, where Y_L is its stored tail (the unit rows lie above)
+  const int64_t kL = cm - ca, kR = ce - cm, rL = ca + b, rR = cm + b;
+  const int64_t ML = n - rL, MR = n - rR;
+  cudaStream_t st = h->stream;
+  Scope sc(h, SBR_K_OTHER, 4.0 * (ML * (kL + kR) + MR * (kL + kR)) * 4, 3 * 2.0 * (MR + ML) * kL * kR);
+  cudaError_t e;
+  if ((e = split_tf32_cm(MR, (int)kL, A + rR + ca * lda, lda, false, YS, ldM, loM, st)) != cudaSuccess) return SBR_ERR_CUDA;
+  if ((e = split_tf32_cm(MR, (int)kR, Wo + rR + cm * ldwo, ldwo, false, CS, ldM, loM, st)) != cudaSuccess)
+    return SBR_ERR_CUDA;
+  if ((e = split_tf32_rm(ML, (int)kL, Wo + rL + ca * ldwo, ldwo, WS, ldk, lok, st)) != cudaSuccess) return SBR_ERR_CUDA;
+  GemmTcLaunch g1{};   // T^T = W_R^T Y_L  (kR x kL)
+  g1.A0 = g1.A1 = (const __half*)CS;
+  g1.B0 = g1.B1 = (const __half*)YS;
+  g1.K = MR;
+  g1.lo_off = loM;
+  g1.a_rows = kR;
+  g1.ld_a = ldM;
+  g1.b_rows = kL;
+  g1.ld_b = ldM;
+  g1.Mrows = kR;
+  g1.Ncols = kL;
+  g1.Zs = TS;
+  g1.ldz = ldk;
+  g1.zlo_off = lok;
+  g1.num_sms = h->nsm;
+  if ((e = launch_gemm_split_tf32(g1, st)) != cudaSuccess) return SBR_ERR_CUDA;
+  GemmTcLaunch g2{};   // W_R[rL:] -= W_L T
+  g2.A0 = g2.A1 = (const __half*)WS;
+  g2.B0 = g2.B1 = (const __half*)TS;
+  g2.K = kL;
+  g2.lo_off = lok;
+  g2.a_rows = ML;
+  g2.ld_a = ldk;
+  g2.b_rows = kR;
+  g2.ld_b = ldk;
+  g2.Mrows = ML;
+  g2.Ncols = kR;
+  g2.C = Wo + rL + cm * ldwo;
+  g2.ldc = ldwo;
+  g2.num_sms = h->nsm;
+  if ((e = launch_gemm_sub_tf32(g2, st)) != cudaSuccess) return SBR_ERR_CUDA;
+  h->launches += 5;
+  return SBR_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int sbr_form_w(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
+               float* Wo, int64_t ldwo) {
+  if (!h) return -1;
+  if (n < 1) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (nb < b || nb % b != 0 || nb > 4096) return -4;
+  if (!A) return -5;
+  if (lda < n) return -6;
+  if (!W) return -7;
+  if (ldw < n) return -8;
+  if (!Wo) return -9;
+  if (ldwo < n) return -10;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  cudaStream_t st = h->stream;
+  const int64_t ncols = n - b;
+  if (ncols <= 0) return SBR_OK;
+  // start: the per-block W_J with zeros above each block's rows (Wo[:, c] = W[:, c] for r >= r0(J))
+  SBR_CK(copy_block_w(n, b, nb, W, ldw, Wo, ldwo, st), "W blocks");
+  h->launches += 1;
+  const int64_t M0 = n - b;
+  const int64_t loM = (M0 + 31) / 32 * 32, ldM = 2 * loM;
+  const int64_t kmax = (ncols + 1) / 2 + nb, lok = (kmax + 31) / 32 * 32, ldk = 2 * lok;
+  const size_t nCS = align_up(sizeof(float) * kmax * ldM), nYS = align_up(sizeof(float) * kmax * ldM),
+               nWS = align_up(sizeof(float) * M0 * ldk), nTS = align_up(sizeof(float) * kmax * ldk);
+  int rc = SBR_OK;
+  float* base = fq_grow(h, nCS + nYS + nWS + nTS, &rc);
+  if (rc != SBR_OK) return rc;
+  float* CS = base;
+  float* YS = (float*)((char*)base + nCS);
+  float* WS = (float*)((char*)base + nCS + nYS);
+  float* TS = (float*)((char*)base + nCS + nYS + nWS);
+  rc = form_w_rec(h, n, b, nb, A, lda, Wo, ldwo, 0, ncols, CS, YS, WS, TS, ldM, loM, ldk, lok);
+  if (rc == SBR_ERR_CUDA) set_err("form_w", cudaGetLastError());
+  return rc;
+}
+
 int sbr_set_stream(sbr_handle_t h, void* stream) {
   if (!h) return -1;
   h->stream = (cudaStream_t)stream;

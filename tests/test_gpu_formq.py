@@ -78,3 +78,32 @@ def test_form_q_errors():
     _lib.check(L.sbr_form_q(h._h, 8, 8, 8, p, 8, p, 8, q.data_ptr(), 8), "form_q trivial")
     assert torch.equal(q.cpu(), torch.eye(8))
     h.close()
+
+
+@pytest.mark.parametrize("mode", ["fp16", "3xtf32"])
+@pytest.mark.parametrize("n,b,nb", [(300, 8, 32), (1000, 32, 128), (2048, 32, 256), (1024, 64, 128), (96, 32, 32)])
+def test_form_w_and_apply_q(n, b, nb, mode):
+    """Alg. 2 (sbr_form_w) vs the oracle's Alg. 2 on the SAME blocks, entry-wise; X <- Q X
+    (sbr_apply_q) vs the oracle product of the blocks times X."""
+    import torch
+
+    import paper_conf_ppopp_zhangsoyw23_b200 as sbr
+    from oracle import backtransform
+
+    a = workloads.random_symmetric(n, 71 * n + b)
+    h = sbr.Handle(0)
+    A = torch.from_numpy(a).cuda()
+    ab, w = h.reduce(A, b, nb, mode=mode)
+    wm = h.form_w(A, w, b, nb)
+    X0 = np.random.default_rng(n).standard_normal((16, n)).astype(np.float32)   # torch (kx, n) = column-major n x kx
+    X = torch.from_numpy(X0).cuda()
+    h.apply_q(A, w, b, nb, X)
+    torch.cuda.synchronize()
+    blocks = metrics.blocks_from_output(A.cpu().numpy().T, w.cpu().numpy().T, n, b, nb)
+    W_ref, Y_ref = backtransform.form_w(n, b, blocks)
+    dw = np.abs(wm.cpu().numpy().T.astype(np.float64) - W_ref).max() / max(1.0, np.abs(W_ref).max())
+    qx_ref = backtransform.apply_q(W_ref, Y_ref, X0.T.astype(np.float64))
+    dx = np.abs(X.cpu().numpy().T - qx_ref).max() / np.abs(qx_ref).max()
+    print(f"form_w/apply_q n={n} b={b} nb={nb} {mode}: |W - W_Alg2| {dw:.2e} |QX - QX_ref| {dx:.2e}")
+    assert dw <= 5e-5
+    assert dx <= 2e-5
