@@ -163,6 +163,38 @@ int sbr_form_w(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t
 int sbr_apply_q(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t lda, const float* W, int64_t ldw,
                 float* X, int64_t ldx, int64_t kx);
 
+/* ---- Stage two: band -> tridiagonal -> eigenvalues on the GPU ----
+ * The paper's two-stage EVD (Fig. 1) runs stage two on the CPU (MAGMA, after a
+ * device->host copy of the band) and names a GPU stage two as future work.
+ * These calls run it on the device, in fp64, stream-ordered (return after enqueue):
+ *
+ * sbr_band_to_tridiag: T = Q2^T B Q2 tridiagonal, by Householder bulge chasing (SBR with target
+ *   bandwidth 1, Fig. 2; sweep s annihilates column s and chases the bulge in b-row
+ *   steps; sweeps run pipelined, one warp each).  Q2 is not formed.
+ *   AB : device fp32 band in LAPACK lower band storage, AB[d + j ldab] = B[j+d, j], 0 <= d <= b
+ *        (sbr_reduce's AB output), ldab >= b+1; read only.  Entries with j+d >= n are ignored.
+ *   d  : device fp64, n entries: diag(T).  e: device fp64, n-1 entries: subdiag(T) (signs are
+ *        not normalised: T is unique up to D T D, D = diag(+-1)).
+ *   Returns 0, -1 (h), -2 (n < 0), -3 (b not in 1..64), -4 (AB), -5 (ldab), -6 (d), -7 (e),
+ *   SBR_ERR_NOMEM, SBR_ERR_CUDA.
+ * sbr_tridiag_eigenvalues: all eigenvalues of tridiag(d, e), ascending, into lam (device fp64,
+ *   n), by bisection on Sturm counts: eigenvalue k is the smallest x with more than k
+ *   negative pivots in the LDL^T factorisation of T - x I, each interval halved from the
+ *   Gershgorin bounds until its width is <= 2 eps max(|lo|, |hi|) (pivots below
+ *   DBL_MIN max(1, max(|d|,|e|)^2) in magnitude replaced by -that).  One thread per eigenvalue.
+ *   Returns 0, -1 (h), -2 (n), -3 (d), -4 (e), -5 (lam), SBR_ERR_NOMEM, SBR_ERR_CUDA.
+ * sbr_band_eigenvalues: both steps (d, e in handle-owned memory).  Arguments as
+ *   sbr_band_to_tridiag, lam = argument 6.
+ * sbr_eigenvalues: the whole two-stage pipeline on one GPU -- sbr_reduce (W not kept; A is
+ *   overwritten as by sbr_reduce) then sbr_band_eigenvalues into lam (device fp64, n).  Argument
+ *   errors 1-7 as sbr_reduce, -8 (lam NULL); latched reduction errors as sbr_reduce.
+ * Workspace: about (16 b + 28) n bytes (plus the band for sbr_eigenvalues), handle-owned, grown
+ * on demand and freed by sbr_destroy. */
+int sbr_band_to_tridiag(sbr_handle_t h, int64_t n, int b, const float* AB, int64_t ldab, double* d, double* e);
+int sbr_tridiag_eigenvalues(sbr_handle_t h, int64_t n, const double* d, const double* e, double* lam);
+int sbr_band_eigenvalues(sbr_handle_t h, int64_t n, int b, const float* AB, int64_t ldab, double* lam);
+int sbr_eigenvalues(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, double* lam);
+
 /* ---- Multi-GPU (north star: 1D block-cyclic columns) ----
  *
  * Data distribution: the columns of A are split into nb-wide blocks J (global columns
@@ -235,7 +267,8 @@ int sbr_generate_symmetric(sbr_handle_t h, uint64_t seed, int64_t n, float* A, i
 #define SBR_K_PASS 3    /* X_t = OA W_t (a4)                       */
 #define SBR_K_SYR2K 4   /* trailing update (a6, with Z formation)  */
 #define SBR_K_OTHER 5   /* setup, band extraction                  */
-#define SBR_K_COUNT 6
+#define SBR_K_STAGE2 6  /* stage two: bulge chase, bisection (f2)  */
+#define SBR_K_COUNT 7
 int sbr_set_kernel_timing(sbr_handle_t h, int enable);
 int sbr_reset_kernel_stats(sbr_handle_t h);
 int sbr_kernel_stats(sbr_handle_t h, int kid, int64_t* launches, double* ms,

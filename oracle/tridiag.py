@@ -44,9 +44,10 @@ def sturm_count(d: np.ndarray, e: np.ndarray, x: np.ndarray) -> np.ndarray:
 def bisection_eigenvalues(d: np.ndarray, e: np.ndarray, tol: float | None = None) -> np.ndarray:
     """All eigenvalues of tridiag(d, e), ascending, by bisection on Gershgorin bounds.
 
-    Eigenvalue k (0-based) is the smallest x with ``sturm_count(x) > k``; every
-    interval is halved until its width is below ``tol`` (default
-    ``2 eps max|lambda|``).
+    Eigenvalue k (0-based) is the smallest x with ``sturm_count(x) > k``; each
+    interval is halved until ITS width is at most ``tol`` (default
+    ``2 eps max(|lo|, |hi|)`` of the Gershgorin bounds) -- per-interval
+    convergence, as LAPACK dstebz tests each interval on its own.
     """
     d = np.asarray(d, dtype=np.float64)
     e = np.asarray(e, dtype=np.float64)
@@ -66,12 +67,13 @@ def bisection_eigenvalues(d: np.ndarray, e: np.ndarray, tol: float | None = None
     hi = np.full(n, hi_b + tol)
     k = np.arange(n)
     for _ in range(200):                    # ~ log2(span / tol) halvings suffice
-        if np.max(hi - lo) <= tol:
+        active = (hi - lo) > tol
+        if not np.any(active):
             break
         mid = 0.5 * (lo + hi)
         below = sturm_count(d, e, mid) > k
-        hi = np.where(below, mid, hi)
-        lo = np.where(below, lo, mid)
+        hi = np.where(active & below, mid, hi)
+        lo = np.where(active & ~below, mid, lo)
     return 0.5 * (lo + hi)
 
 

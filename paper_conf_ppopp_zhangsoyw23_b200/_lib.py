@@ -22,7 +22,7 @@ SBR_ERR_UNSUPPORTED = 5
 SBR_FP16_FP32ACC = 0
 SBR_3XTF32 = 1
 SBR_OUT_BAND, SBR_OUT_Y, SBR_OUT_W = 1, 2, 4
-KERNEL_CLASSES = {"panel": 0, "lazy": 1, "wmerge": 2, "pass": 3, "syr2k": 4, "other": 5}
+KERNEL_CLASSES = {"panel": 0, "lazy": 1, "wmerge": 2, "pass": 3, "syr2k": 4, "other": 5, "stage2": 6}
 
 # symbol -> (restype, argtypes): the complete exported surface of include/sbr.h
 _h = ctypes.c_void_p
@@ -53,6 +53,10 @@ SIGNATURES = {
     "sbr_form_q": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_form_w": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64]),
     "sbr_apply_q": (_i, [_h, _i64, _i, _i, _p, _i64, _p, _i64, _p, _i64, _i64]),
+    "sbr_band_to_tridiag": (_i, [_h, _i64, _i, _p, _i64, _p, _p]),
+    "sbr_tridiag_eigenvalues": (_i, [_h, _i64, _p, _p, _p]),
+    "sbr_band_eigenvalues": (_i, [_h, _i64, _i, _p, _i64, _p]),
+    "sbr_eigenvalues": (_i, [_h, _i, _i64, _i, _i, _p, _i64, _p]),
     "sbr_rank": (_i, [_h]),
     "sbr_nranks": (_i, [_h]),
     # kernel-level test hooks (include/sbr_testing.h)

@@ -188,6 +188,55 @@ class Handle:
               "sbr_apply_q")
         return X
 
+    # ---- stage two (include/sbr.h sbr_band_to_tridiag ...)
+    def band_to_tridiag(self, ab, d=None, e=None):
+        """Band (torch (n, b+1) float32 CUDA, ``ab[j, k] = B[j+k, j]``, :meth:`reduce`'s output) ->
+        tridiagonal ``(d, e)`` (float64, n and n-1 entries) by bulge chasing on the GPU."""
+        import torch
+
+        n, bp1 = int(ab.shape[0]), int(ab.shape[1])
+        if ab.dtype != torch.float32 or not ab.is_cuda or not ab.is_contiguous():
+            raise ValueError("ab must be a contiguous (n, b+1) float32 CUDA tensor")
+        d = torch.empty(n, dtype=torch.float64, device=ab.device) if d is None else d
+        e = torch.empty(max(n - 1, 0), dtype=torch.float64, device=ab.device) if e is None else e
+        check(lib().sbr_band_to_tridiag(self._h, n, bp1 - 1, _ptr(ab), bp1, _ptr(d), _ptr(e)), "sbr_band_to_tridiag")
+        return d, e
+
+    def tridiag_eigenvalues(self, d, e, lam=None):
+        """Eigenvalues (ascending, float64 CUDA) of tridiag(d, e) by Sturm bisection on the GPU."""
+        import torch
+
+        n = int(d.shape[0])
+        if d.dtype != torch.float64 or e.dtype != torch.float64 or not d.is_cuda or not e.is_cuda:
+            raise ValueError("d, e must be float64 CUDA tensors")
+        lam = torch.empty(n, dtype=torch.float64, device=d.device) if lam is None else lam
+        check(lib().sbr_tridiag_eigenvalues(self._h, n, _ptr(d.contiguous()), _ptr(e.contiguous()), _ptr(lam)),
+              "sbr_tridiag_eigenvalues")
+        return lam
+
+    def band_eigenvalues(self, ab, lam=None):
+        """All eigenvalues of the band ``ab`` (stage two on the GPU: bulge chase + bisection)."""
+        import torch
+
+        n, bp1 = int(ab.shape[0]), int(ab.shape[1])
+        if ab.dtype != torch.float32 or not ab.is_cuda or not ab.is_contiguous():
+            raise ValueError("ab must be a contiguous (n, b+1) float32 CUDA tensor")
+        lam = torch.empty(n, dtype=torch.float64, device=ab.device) if lam is None else lam
+        check(lib().sbr_band_eigenvalues(self._h, n, bp1 - 1, _ptr(ab), bp1, _ptr(lam)), "sbr_band_eigenvalues")
+        return lam
+
+    def eigenvalues(self, A, b: int, nb: int, mode="fp16", lam=None):
+        """Two-stage EVD, eigenvalues only (sbr_eigenvalues): A (overwritten) -> band -> lam (float64)."""
+        import torch
+
+        n = int(A.shape[0])
+        if A.dim() != 2 or A.shape[1] != n or A.dtype != torch.float32 or not A.is_cuda or not A.is_contiguous():
+            raise ValueError("A must be a contiguous square float32 CUDA tensor")
+        lam = torch.empty(n, dtype=torch.float64, device=A.device) if lam is None else lam
+        check(lib().sbr_eigenvalues(self._h, _mode(mode), n, int(b), int(nb), _ptr(A), n, _ptr(lam)),
+              "sbr_eigenvalues")
+        return lam
+
     def reduce_dist(self, A_local, n: int, b: int, nb: int, mode="fp16", want_w: bool = True, ab=None, w=None):
         """One n x n matrix across the handle's ranks (collective; include/sbr.h sbr_reduce_dist).
 

@@ -303,4 +303,12 @@ cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ld
 cudaError_t to_half_cm(int64_t rows, int cols, int cols_pad, const float* src, int64_t lds, __half* dst,
                        int64_t ldd, cudaStream_t st);
 
+// stage two (k_stage2.cu): band (fp32, LAPACK lower band storage) -> tridiagonal
+// (d, e fp64) by Householder bulge chasing; eigenvalues of tridiag(d, e) by Sturm bisection
+size_t stage2_ws_bytes(int64_t n, int b);
+cudaError_t band_to_tridiag(int64_t n, int b, const float* AB, int64_t ldab, void* ws, double* d, double* e,
+                            cudaStream_t st);
+size_t tridiag_eig_ws_bytes(int64_t n);
+cudaError_t tridiag_eigenvalues(int64_t n, const double* d, const double* e, void* ws, double* lam, cudaStream_t st);
+
 }  // namespace sbr

@@ -88,6 +88,9 @@ struct sbr_ctx {
   // sbr_form_q split operands (grown on demand, kept for the next call)
   void* fq = nullptr;
   size_t fq_bytes = 0;
+  // stage two (k_stage2.cu): working band, progress counters, d/e/e^2, band of sbr_eigenvalues
+  void* s2 = nullptr;
+  size_t s2_bytes = 0;
   // stats
   bool timing = false;
   std::vector<cudaEvent_t> ev_pool;
@@ -1274,6 +1277,121 @@ int sbr_form_w(sbr_handle_t h, int64_t n, int b, int nb, const float* A, int64_t
   return rc;
 }
 
+// ---------------------------------------------------------------- stage two
+static char* s2_grow(sbr_ctx* h, size_t need, int* rc) {
+  *rc = SBR_OK;
+  if (h->s2_bytes < need) {
+    if (cudaStreamSynchronize(h->stream) != cudaSuccess) {
+      *rc = SBR_ERR_CUDA;
+      return nullptr;
+    }
+    if (h->s2) cudaFree(h->s2);
+    h->s2 = nullptr;
+    h->s2_bytes = 0;
+    if (cudaMalloc(&h->s2, need) != cudaSuccess) {
+      cudaGetLastError();
+      *rc = SBR_ERR_NOMEM;
+      return nullptr;
+    }
+    h->s2_bytes = need;
+  }
+  return (char*)h->s2;
+}
+
+static int stage2_run(sbr_ctx* h, int64_t n, int b, const float* AB, int64_t ldab, double* d, double* e, double* lam,
+                      char* ws) {
+  cudaStream_t st = h->stream;
+  if (AB) {
+    // bulge chase: per step ~ 3 b x b fp64 blocks read + written
+    const int64_t steps = n > 2 && b > 1 ? (n - 2) * ((n + b - 1) / b) / 2 : 0;
+    Scope sc(h, SBR_K_STAGE2, 48.0 * b * b * (double)steps, 8.0 * b * b * (double)steps);
+    SBR_CK(band_to_tridiag(n, b, AB, ldab, ws, d, e, st), "band_to_tridiag");
+    h->launches += (n > 2 && b > 1) ? 3 : 2;
+  }
+  if (lam) {
+    Scope sc(h, SBR_K_STAGE2, 16.0 * n, 4.0 * 53.0 * (double)n * n);
+    SBR_CK(tridiag_eigenvalues(n, d, e, ws, lam, st), "tridiag_eigenvalues");
+    h->launches += 2;
+  }
+  return SBR_OK;
+}
+
+static size_t s2_align(size_t x) { return (x + 255) & ~size_t(255); }
+
+int sbr_band_to_tridiag(sbr_handle_t h, int64_t n, int b, const float* AB, int64_t ldab, double* d, double* e) {
+  if (!h) return -1;
+  if (n < 0) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (!AB && n > 0) return -4;
+  if (ldab < b + 1) return -5;
+  if (!d && n > 0) return -6;
+  if (!e && n > 1) return -7;
+  if (n == 0) return SBR_OK;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  int rc = SBR_OK;
+  char* ws = s2_grow(h, stage2_ws_bytes(n, b), &rc);
+  if (rc != SBR_OK) return rc;
+  return stage2_run(h, n, b, AB, ldab, d, e, nullptr, ws);
+}
+
+int sbr_tridiag_eigenvalues(sbr_handle_t h, int64_t n, const double* d, const double* e, double* lam) {
+  if (!h) return -1;
+  if (n < 0) return -2;
+  if (!d && n > 0) return -3;
+  if (!e && n > 1) return -4;
+  if (!lam && n > 0) return -5;
+  if (n == 0) return SBR_OK;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  int rc = SBR_OK;
+  char* ws = s2_grow(h, tridiag_eig_ws_bytes(n), &rc);
+  if (rc != SBR_OK) return rc;
+  return stage2_run(h, n, 1, nullptr, 0, const_cast<double*>(d), const_cast<double*>(e), lam, ws);
+}
+
+int sbr_band_eigenvalues(sbr_handle_t h, int64_t n, int b, const float* AB, int64_t ldab, double* lam) {
+  if (!h) return -1;
+  if (n < 0) return -2;
+  if (b < 1 || b > 64) return -3;
+  if (!AB && n > 0) return -4;
+  if (ldab < b + 1) return -5;
+  if (!lam && n > 0) return -6;
+  if (n == 0) return SBR_OK;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  const size_t sde = s2_align(sizeof(double) * 2 * n);
+  const size_t sw = std::max(stage2_ws_bytes(n, b), tridiag_eig_ws_bytes(n));
+  int rc = SBR_OK;
+  char* base = s2_grow(h, sde + sw, &rc);
+  if (rc != SBR_OK) return rc;
+  double* d = (double*)base;
+  double* e = d + n;
+  char* ws = base + sde;
+  if ((rc = stage2_run(h, n, b, AB, ldab, d, e, nullptr, ws)) != SBR_OK) return rc;
+  return stage2_run(h, n, b, nullptr, 0, d, e, lam, ws);
+}
+
+int sbr_eigenvalues(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, double* lam) {
+  if (!h) return -1;
+  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32) return -2;
+  if (n < 1) return -3;
+  if (b < 1 || b > 64) return -4;
+  if (!lam) return -8;
+  SBR_CK(cudaSetDevice(h->device), "cudaSetDevice");
+  const size_t sab = s2_align(sizeof(float) * (size_t)(b + 1) * n);
+  const size_t sde = s2_align(sizeof(double) * 2 * n);
+  const size_t sw = std::max(stage2_ws_bytes(n, b), tridiag_eig_ws_bytes(n));
+  int rc = SBR_OK;
+  char* base = s2_grow(h, sab + sde + sw, &rc);
+  if (rc != SBR_OK) return rc;
+  float* AB = (float*)base;
+  double* d = (double*)(base + sab);
+  double* e = d + n;
+  char* ws = base + sab + sde;
+  rc = sbr_reduce(h, mode, n, b, nb, A, lda, AB, b + 1, nullptr, 0);
+  if (rc != SBR_OK) return rc;   // argument positions 1-7 coincide with sbr_reduce's
+  if ((rc = stage2_run(h, n, b, AB, b + 1, d, e, nullptr, ws)) != SBR_OK) return rc;
+  return stage2_run(h, n, b, nullptr, 0, d, e, lam, ws);
+}
+
 int sbr_set_stream(sbr_handle_t h, void* stream) {
   if (!h) return -1;
   h->stream = (cudaStream_t)stream;
@@ -1290,6 +1408,7 @@ int sbr_destroy(sbr_handle_t h) {
   if (h->ws) cudaFree(h->ws);
   if (h->e2e) cudaFree(h->e2e);
   if (h->fq) cudaFree(h->fq);
+  if (h->s2) cudaFree(h->s2);
   if (h->ptrace) cudaFree(h->ptrace);
   if (h->pinned) cudaFreeHost(h->pinned);
   for (auto e : h->slot_ev)
