@@ -2,8 +2,8 @@
 sbr_band_eigenvalues, sbr_eigenvalues), against the oracle (oracle.tridiag, pinned to LAPACK
 dstebz / dense eigvalsh in tests/test_oracle_sbr.py) and the mathematics:
 
-  * bisection: the GPU follows the oracle's algorithm (same bounds, tolerance, pivmin,
-    recurrence and operation order, IEEE fp64) -> the eigenvalues agree to the bit;
+  * bisection: the GPU multisection keeps the oracle bisection's invariant (same bounds,
+    tolerance, pivmin, recurrence and operation order, IEEE fp64) -> within tol of it;
   * bulge chase: T = Q2^T B Q2 is tridiagonal with the spectrum of B (fp64, backward stable:
     |lam(T) - lam(B)| <= 1e-11 ||B||), ||T||_F = ||B||_F, and (Q2 e_0 = e_0, implicit-Q theorem)
     T equals the oracle's b = 1 reduction up to the signs of e on small cases;
@@ -40,8 +40,11 @@ def _band_dense(ab):
     return m
 
 
-@pytest.mark.parametrize("n", [1, 2, 3, 17, 257, 1000])
-def test_bisection_bitwise_equals_oracle(n):
+@pytest.mark.parametrize("n", [1, 2, 3, 17, 257, 1000, 5000])
+def test_multisection_matches_oracle_bisection(n):
+    """Both keep count(lo) <= k < count(hi) and stop at width <= tol = 2 eps max|Gershgorin|; the
+    GPU's Sturm recurrence divides with a refined reciprocal (a few ulps), which can move a count
+    transition by a few ulps of the spectrum: the midpoints agree within 4 tol."""
     import torch
 
     from oracle.tridiag import bisection_eigenvalues
@@ -55,8 +58,14 @@ def test_bisection_bitwise_equals_oracle(n):
     h = _handle()
     lam = h.tridiag_eigenvalues(torch.from_numpy(d).cuda(), torch.from_numpy(e).cuda()).cpu().numpy()
     ref = bisection_eigenvalues(d, e)
-    print(f"bisection n={n}: max|gpu - oracle| {np.max(np.abs(lam - ref)) if n else 0:.1e}")
-    assert np.array_equal(lam, ref)
+    rad = np.zeros(n)
+    rad[:-1] += np.abs(e)
+    rad[1:] += np.abs(e)
+    tol = 2 * np.finfo(np.float64).eps * max(abs(np.min(d - rad)), abs(np.max(d + rad)))
+    err = float(np.max(np.abs(lam - ref)))
+    print(f"multisection n={n}: max|gpu - oracle| {err:.1e} (tol {tol:.1e})")
+    assert err <= 4 * tol
+    assert np.all(np.diff(lam) >= 0)
     h.close()
 
 
