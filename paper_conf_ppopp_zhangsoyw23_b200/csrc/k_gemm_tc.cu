@@ -45,21 +45,47 @@ template <bool TF> struct GCfg {
 };
 }  // namespace
 
-// tile index -> (I, Jc); SYR2K: the lower tiles, row I holding floor(I*BM/BN)+1 tiles of BN columns
+// tile index -> (I, Jc).  ZFORM / GEMM modes: the full grid, row-major.  SYR2K: the lower tiles
+// (Jc * BN <= I * BM + BM - 1, i.e. I >= r Jc with r = BN / BM) in an L2-friendly raster: bands of
+// H tile rows, inside a band column-major (all rows I of column Jc, then Jc + 1).  The ~148 tiles
+// in flight then share one or two B panels (rows Jc of [Z | Y]) and sweep the band's A panels
+// (H x 128 rows of [Y | Z], which stay L2-resident), so B is read from DRAM once per band
+// instead of once per tile row (the operands of a large block, 2 x M x 2nb, exceed L2).
 template <int MODE, int BN>
-SBR_DEV void gemm_tile(int t, int ntn, int& I, int& Jc) {
-  if (MODE != 0) {  // ZFORM / GEMM modes: full grid, row-major
+SBR_DEV void gemm_tile(int t, int ntn, int ntm, int& I, int& Jc) {
+  if (MODE != 0) {
     I = t / ntn;
     Jc = t % ntn;
-  } else {
-    int i = 0;
-    while (true) {
-      const int cnt = i * G_BM / BN + 1;
-      if (t < cnt) { I = i; Jc = t; return; }
-      t -= cnt;
-      ++i;
-    }
+    return;
   }
+  constexpr int r = BN / G_BM;                       // 1 or 2
+  constexpr int H = BN == 256 ? 64 : 32;             // band height in tile rows (A band <= ~64 MB)
+  for (int I0 = 0; I0 < ntm; I0 += H) {
+    const int I1 = min(I0 + H, ntm), Hs = I1 - I0;
+    const int F = I0 / r + 1;                        // columns with every band row valid
+    const int D = I1 - r * F;                        // rows of column F (then D - r, D - 2r, ...)
+    const int jmax = D > 0 ? (D + r - 1) / r : 0;
+    const int full = F * Hs, tri = jmax * D - r * jmax * (jmax - 1) / 2;
+    if (t < full) {
+      Jc = t / Hs;
+      I = I0 + t % Hs;
+      return;
+    }
+    t -= full;
+    if (t < tri) {   // C(j) = j D - r j (j - 1) / 2 tiles before triangular column j
+      const double a = D + 0.5 * r;
+      int j = (int)((a - sqrt(fmax(a * a - 2.0 * r * t, 0.0))) / r);
+      j = max(0, min(j, jmax - 1));
+      while (j + 1 < jmax && (j + 1) * D - r * (j + 1) * j / 2 <= t) ++j;
+      while (j > 0 && j * D - r * j * (j - 1) / 2 > t) --j;
+      const int u = t - (j * D - r * j * (j - 1) / 2);
+      Jc = F + j;
+      I = r * Jc + u;
+      return;
+    }
+    t -= tri;
+  }
+  I = Jc = 0;   // not reached for t < ntiles
 }
 
 // Multi-GPU column ownership of the SYR2K output (sbr_reduce_dist): output column rel (relative to
@@ -122,13 +148,14 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   const uint32_t tmem = *tmem_slot;
   pdl_wait();
   const int nk = segs.n * kpb;
+  const int ntm = (int)((Mrows + G_BM - 1) / G_BM);
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
       int st = 0; uint32_t ph = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
         int I, Jc;
-        gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+        gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
         if (!own.owned((int64_t)Jc * G_BN)) continue;
         for (int kc = 0; kc < nk; ++kc) {
           const int sg = kc / kpb, kin = (kc % kpb) * BK;
@@ -153,7 +180,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
         if (own.P > 1) {
           int I, Jc;
-          gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+          gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
           if (!own.owned((int64_t)Jc * G_BN)) continue;
         }
         for (int kc = 0; kc < nk; ++kc) {
@@ -193,7 +220,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
-      gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
       if (!own.owned((int64_t)Jc * G_BN)) continue;
       float acc[64];
 #pragma unroll
@@ -246,7 +273,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
-      gemm_tile<MODE, G_BN>(t, ntn, I, Jc);
+      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
       if (!own.owned((int64_t)Jc * G_BN)) continue;
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();

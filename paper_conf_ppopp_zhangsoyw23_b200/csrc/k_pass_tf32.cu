@@ -50,24 +50,52 @@ constexpr int P3_SMEM = P3_OFF_BAR + P3_NBAR * 8 + 16 + 1024;
 constexpr int P3_THREADS = 512;   // + converter warps 12-15 (two converter groups of 4 warps)
 static_assert(P3_SMEM <= 232448, "3xTF32 pass smem");
 
-struct Walk1 {   // C = 1 tile walk: column J, rows I = J .. NT-1
+// Tile ownership (sbr_reduce_dist, 1D block-cyclic): the tile grid starts at global column gr0
+// (the block start, nb-aligned; OA begins `off` rows/columns into it), tile column J lies in the
+// nb-block blk0 + J / gpb, owned by rank (block % P); P = 1: every tile.
+struct PassOwnTf {
+  int P = 1, rank = 0, gpb = 1;
+  int64_t blk0 = 0, nbo = 1, gr0 = 0;
+  SBR_DEV bool owned(int J) const { return P <= 1 || (int)((blk0 + J / gpb) % P) == rank; }
+  SBR_DEV int64_t lcol(int64_t g) const {   // local column of global column g
+    if (P <= 1) return g;
+    const int64_t Jb = g / nbo;
+    return (Jb / P) * nbo + (g - Jb * nbo);
+  }
+};
+
+struct Walk1 {   // C = 1 tile walk: owned tile columns J in order, rows I = J .. NT-1
   int NT, I, J;
   int64_t left;
   bool first;   // first tile of a group (column) in this CTA's range
-  SBR_DEV void start(int NT_, int64_t t0, int64_t count) {
+  PassOwnTf own;
+  SBR_DEV void start(int NT_, int64_t t0, int64_t count, const PassOwnTf& o) {
     NT = NT_;
+    own = o;
     left = count;
-    J = 0;
-    while (t0 >= NT - J) { t0 -= NT - J; ++J; }
-    I = J + (int)t0;
     first = true;
+    I = J = 0;
+    if (count <= 0) return;
+    J = 0;
+    for (;;) {
+      if (own.owned(J)) {
+        if (t0 < NT - J) break;
+        t0 -= NT - J;
+      }
+      ++J;
+    }
+    I = J + (int)t0;
   }
   SBR_DEV bool valid() const { return left > 0; }
   SBR_DEV bool glast() const { return left == 1 || I + 1 == NT; }
   SBR_DEV void next() {
     --left;
     first = false;
-    if (++I == NT) { ++J; I = J; first = true; }
+    if (++I == NT) {
+      do { ++J; } while (J < NT && !own.owned(J));
+      I = J;
+      first = true;
+    }
   }
 };
 }  // namespace
@@ -76,8 +104,8 @@ SBR_DEV void fence_proxy_async_smem() { asm volatile("fence.proxy.async.shared::
 
 __global__ void __launch_bounds__(P3_THREADS, 1)
     pass_tf32_kernel(const __grid_constant__ CUtensorMap mapA, const __grid_constant__ CUtensorMap mapS,
-                     const __grid_constant__ CUtensorMap mapW, int r0, int M, int NT, int jstrip, int64_t T0,
-                     int64_t T, int b, float* X, int64_t ldx, int l2normal) {
+                     const __grid_constant__ CUtensorMap mapW, int M, int off, int NT, int jstrip, int64_t T,
+                     int b, float* X, int64_t ldx, int l2normal, PassOwnTf own) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint64_t* bars = (uint64_t*)(smem + P3_OFF_BAR);
@@ -97,8 +125,8 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
   uint32_t* tmem_slot = (uint32_t*)(bars + P3_NBAR);
   const int warp = warp_id(), lane = lane_id();
   pdl_trigger();
-  const int64_t t_beg = T0 + (int64_t)blockIdx.x * T / gridDim.x;
-  const int64_t t_end = T0 + (int64_t)(blockIdx.x + 1) * T / gridDim.x;
+  const int64_t t_beg = (int64_t)blockIdx.x * T / gridDim.x;
+  const int64_t t_end = (int64_t)(blockIdx.x + 1) * T / gridDim.x;
   if (threadIdx.x == 0) {
     for (int i = 0; i < P3_NS; ++i) {
       mbar_init(&l_full[i], 1); mbar_init(&l_empty[i], 1); mbar_init(&hi_done[i], 1);
@@ -128,26 +156,29 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
       const uint64_t lpol = l2normal ? l2_policy_evict_normal() : l2_policy_evict_first();
       int st = 0; uint32_t ph = 0;
       uint32_t jph = 0;
-      for (w.start(NT, t_beg, t_end - t_beg); w.valid(); w.next()) {
+      for (w.start(NT, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
         if (w.first) {
           mbar_wait(wj_empty, jph ^ 1);
           jph ^= 1;
           mbar_expect_tx(wj_full, P3_WT);
           for (int rc = 0; rc < 4; ++rc)
-            tma_load_2d(smem + P3_OFF_WJ + rc * 8192, &mapW, wj_full, w.J * 128 + rc * 32, 0);
+            tma_load_2d(smem + P3_OFF_WJ + rc * 8192, &mapW, wj_full, w.J * 128 + rc * 32 - off, 0);
         }
         mbar_wait(&l_empty[st], ph ^ 1);
         mbar_expect_tx(&l_full[st], P3_STAGE);
         uint8_t* dst = smem + st * P3_STAGE;
         const bool strip = w.J < jstrip;
+        // grid rows / columns from gr0; the strip and W are indexed from OA's origin (gr0 + off):
+        // coordinates below 0 (the `off` rows / columns in front of OA) read as zeros (TMA OOB fill)
+        const int lc = (int)own.lcol(own.gr0 + (int64_t)w.J * 128);
         for (int rc = 0; rc < 4; ++rc) {
           if (strip)
-            tma_load_2d_hint(dst + rc * 16384, &mapS, &l_full[st], w.I * 128 + rc * 32, w.J * 128, lpol);
+            tma_load_2d_hint(dst + rc * 16384, &mapS, &l_full[st], w.I * 128 + rc * 32 - off, w.J * 128 - off, lpol);
           else
-            tma_load_2d_hint(dst + rc * 16384, &mapA, &l_full[st], r0 + w.I * 128 + rc * 32, r0 + w.J * 128, lpol);
+            tma_load_2d_hint(dst + rc * 16384, &mapA, &l_full[st], (int)own.gr0 + w.I * 128 + rc * 32, lc, lpol);
         }
         for (int rc = 0; rc < 4; ++rc)
-          tma_load_2d(dst + P3_LT + rc * 8192, &mapW, &l_full[st], w.I * 128 + rc * 32, 0);
+          tma_load_2d(dst + P3_LT + rc * 8192, &mapW, &l_full[st], w.I * 128 + rc * 32 - off, 0);
         if (++st == P3_NS) { st = 0; ph ^= 1; }
       }
     }
@@ -160,7 +191,7 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
       int rb = 0; uint32_t rph = 0;
       int cb = 0; uint32_t cph = 0;
       uint32_t jph = 0, taph = 0, dph = 0;
-      for (w.start(NT, t_beg, t_end - t_beg); w.valid(); w.next()) {
+      for (w.start(NT, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
         if (w.first) {
           mbar_wait(wj_full, jph);
           jph ^= 1;
@@ -222,7 +253,7 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     int st = 0; uint32_t ph = 0;
     uint32_t tph = 0;
-    for (w.start(NT, t_beg, t_end - t_beg); w.valid(); w.next()) {
+    for (w.start(NT, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
       uint8_t* lt = smem + st * P3_STAGE;
       mbar_wait(&l_full[st], ph);
       if (w.I == w.J) {   // stale upper triangle -> 0, diagonal halved
@@ -284,7 +315,7 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
     float creg[32];   // X_J of the current group, summed over its tiles in fp32 (round to nearest)
 #pragma unroll
     for (int c = 0; c < 32; ++c) creg[c] = 0.f;
-    for (w.start(NT, t_beg, t_end - t_beg); w.valid(); w.next()) {
+    for (w.start(NT, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
       mbar_wait(&racc_full[rb], rph);
       tc_fence_after();
       {
@@ -293,8 +324,8 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
         tmem_ld32(tmem + P3_RACC + rb * 64 + 32 + lane_off, u);
         tc_fence_before();
         mbar_arrive(&racc_empty[rb]);
-        const int64_t row = (int64_t)w.I * 128 + row_in_tile;
-        if (row < M) {
+        const int64_t row = (int64_t)w.I * 128 + row_in_tile - off;
+        if (row >= 0 && row < M) {
 #pragma unroll
           for (int c = 0; c < 32; ++c)
             if (c < b) atomicAdd(&X[row + (int64_t)c * ldx], v[c] + u[c]);
@@ -314,8 +345,8 @@ __global__ void __launch_bounds__(P3_THREADS, 1)
         if (++cb == 2) { cb = 0; cph ^= 1; }
       }
       if (w.glast()) {
-        const int64_t row = (int64_t)w.J * 128 + row_in_tile;
-        if (row < M) {
+        const int64_t row = (int64_t)w.J * 128 + row_in_tile - off;
+        if (row >= 0 && row < M) {
 #pragma unroll
           for (int c = 0; c < 32; ++c)
             if (c < b) atomicAdd(&X[row + (int64_t)c * ldx], creg[c]);
@@ -346,28 +377,39 @@ cudaError_t launch_pass_tf32(const PassTf32Launch& p, cudaStream_t st) {
     cudaError_t e = func_attr((const void*)kern, cudaFuncAttributeMaxDynamicSharedMemorySize, P3_SMEM);
     if (e != cudaSuccess) return e;
   }
-  const int NT = (int)((p.M + 127) / 128);
-  const int jstrip = p.S ? (int)std::min<int64_t>((p.sw + 127) / 128, NT) : 0;
+  const int off = p.off;
+  const int NT = (int)((p.M + off + 127) / 128);
+  // tile columns J < jstrip read the frozen strip, which holds OA columns [0, 128 jstrip - off)
+  const int jstrip = p.S ? (int)std::min<int64_t>((p.sw + off + 127) / 128, NT) : 0;
+  PassOwnTf own;
+  own.gr0 = p.r0 - off;
+  if (p.own_P > 1) {
+    if (p.nbo % 128 != 0 || own.gr0 % p.nbo != 0) return cudaErrorInvalidValue;
+    own.P = p.own_P;
+    own.rank = p.own_rank;
+    own.nbo = p.nbo;
+    own.gpb = (int)(p.nbo / 128);
+    own.blk0 = own.gr0 / p.nbo;
+  }
   CUtensorMap mapA, mapS, mapW;
-  cudaError_t e = make_tmap_2d(&mapA, p.A, false, p.n, p.n, p.lda, 32, 128);
+  cudaError_t e = make_tmap_2d(&mapA, p.A, false, p.n, p.ncols > 0 ? p.ncols : p.n, p.lda, 32, 128);
   if (e != cudaSuccess) return e;
   if (jstrip > 0) {
-    e = make_tmap_2d(&mapS, p.S, false, p.M, (uint64_t)jstrip * 128 < (uint64_t)p.M ? jstrip * 128 : p.M, p.lds,
-                     32, 128);
+    e = make_tmap_2d(&mapS, p.S, false, p.M, std::min<int64_t>((int64_t)jstrip * 128 - off, p.M), p.lds, 32, 128);
     if (e != cudaSuccess) return e;
   } else {
     mapS = mapA;
   }
   e = make_tmap_2d(&mapW, p.WS, false, p.M, 64, p.ldws, 32, 64);
   if (e != cudaSuccess) return e;
-  const int64_t Tall = pass_tf32_tiles(p.M);
-  const int64_t T0 = Tall * p.rank / p.nranks, T1 = Tall * (p.rank + 1) / p.nranks;
-  const int64_t T = T1 - T0;
+  int64_t T = 0;
+  for (int J = 0; J < NT; ++J)
+    if (own.P <= 1 || (int)((own.blk0 + J / own.gpb) % own.P) == own.rank) T += NT - J;
   if (T <= 0) return cudaSuccess;
   const int grid = (int)std::min<int64_t>(T, p.num_sms);
   static const int l2normal = (getenv("SBR_TF32_L2") && !strcmp(getenv("SBR_TF32_L2"), "normal")) ? 1 : 0;
-  return launch_pdl(kern, dim3(grid), dim3(P3_THREADS), P3_SMEM, st, mapA, mapS, mapW, (int)p.r0, (int)p.M, NT,
-                    jstrip, T0, T, p.b, p.X, p.ldx, l2normal);
+  return launch_pdl(kern, dim3(grid), dim3(P3_THREADS), P3_SMEM, st, mapA, mapS, mapW, (int)p.M, off, NT, jstrip, T,
+                    p.b, p.X, p.ldx, l2normal, own);
 }
 
 // ---------------------------------------------------------------- operand splits (3xTF32)

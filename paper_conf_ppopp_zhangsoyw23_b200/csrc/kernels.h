@@ -154,14 +154,19 @@ int64_t pass_owned_tiles(int64_t M, int b, int64_t r0g, int off, int64_t nbo, in
 // columns J < ceil(sw/128), read from the strip S (M x >= min(128 ceil(sw/128), M), ld lds).
 // WS: M x 64 column-major [W_hi (32 cols) | W_lo (32 cols)] from split_tf32_w (bn = 32).
 struct PassTf32Launch {
-  const float* A; int64_t n, lda, r0;
+  const float* A; int64_t n, lda, r0;   // OA = A[r0:, r0:] (global rows / columns)
   const float* S; int64_t lds; int64_t sw;
   const float* WS; int64_t ldws;
   int64_t M;
   int b;
   float* X; int64_t ldx;
   int num_sms;
-  int rank = 0, nranks = 1;
+  // sbr_reduce_dist: the 128-aligned tile grid starts `off` rows / columns before OA (at the
+  // block start); only tile columns of this rank's nb-blocks are visited; A holds `ncols` local
+  // columns (1D block-cyclic, nb = nbo)
+  int off = 0;
+  int own_P = 1, own_rank = 0;
+  int64_t nbo = 0, ncols = 0;
 };
 cudaError_t launch_pass_tf32(const PassTf32Launch& p, cudaStream_t st);
 int64_t pass_tf32_tiles(int64_t M);

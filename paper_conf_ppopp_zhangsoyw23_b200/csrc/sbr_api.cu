@@ -443,9 +443,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   // TMA cannot address (lda % 4 != 0) and for the SBR_TF32_TC=0 ablation
   const bool tc32 = mode == SBR_3XTF32 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0 && b % 4 == 0 &&
                     nb % 4 == 0;
-  if (dist && !tc16) {   // checked by sbr_reduce_dist
+  if (dist && !tc16 && !tc32) {   // checked by sbr_reduce_dist (the SIMT fp32 path is single-GPU)
     std::lock_guard<std::mutex> lk(g_err_mu);
-    g_last_err = "sbr_reduce_dist: FP16 mode with b, nb multiples of 8 only";
+    g_last_err = "sbr_reduce_dist: the tensor-core paths only (b, nb multiples of 8 / 4, A 16-byte aligned)";
     return SBR_ERR_UNSUPPORTED;
   }
   if (tc16) {  // a0: fp16 shadow of OA_0 (strict lower, half diagonal, zero upper) -- this rank's columns
@@ -476,8 +476,8 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int64_t ldwb = W ? ldw : ldn;
     float* OA = AJ + r0 + r0 * lda;
     const int sw = std::min<int64_t>((int64_t)(p - 1) * b, M);  // OA columns rewritten during the block
-    if (sw > 0 && !tc16) {  // tc32: whole 128-column tiles of the strip
-      const int64_t swc = tc32 ? std::min<int64_t>((sw + 127) / 128 * 128, M) : sw;
+    if (sw > 0 && !tc16 && leadJ) {  // tc32: whole 128-column tiles of the (offset) pass grid
+      const int64_t swc = tc32 ? std::min<int64_t>((sw + off + 127) / 128 * 128 - off, M) : sw;
       Scope sc(h, SBR_K_OTHER, 8.0 * M * swc, 0);
       SBR_CK(cudaMemcpy2DAsync(h->Strip, ldn * sizeof(float), OA, lda * sizeof(float), M * sizeof(float), swc,
                                cudaMemcpyDeviceToDevice, st),
@@ -591,7 +591,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         const int64_t c = tb - b;  // OA column of the panel's first column
         const int64_t rows = M - c;
         float* Ablk = AJ + g + g * lda;
-        if (tc16 && !leadJ) {
+        if (!leadJ) {
           // not this rank's step
         } else if (tc16) {  // P = W^T R (SIMT), then GA = OA(:,c) - [X | Y] [Y_c | P^T]^T on tcgen05 (fp16 operands)
           Scope sc(h, SBR_K_LAZY, 2.0 * rows * 2.0 * k + 8.0 * rows * b, 4.0 * rows * k * b);
@@ -773,7 +773,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         }
         continue;
       }
-      if (t >= 1) {  // ---- a3 (SIMT fp32): W merge
+      if (t >= 1 && leadJ) {  // ---- a3 (SIMT fp32): W merge
         Scope sc(h, SBR_K_WMERGE, 4.0 * (M - tb) * (k + b) + 4.0 * M * (k + 2 * b), 2.0 * (2.0 * M - tb) * k * b);
         SBR_CK(zero_matrix(k, b, h->Gb, k, st), "zero G");
         SBR_CK(gemm_tn(M - tb, k, b, 1.f, h->Yb + tb, ldn, Wb + tb + tb * ldwb, ldwb, h->Gb, k, st), "Y^T W0");
@@ -783,12 +783,21 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         h->launches += 2;
       }
       if (tc32) {  // ---- a4 (3xTF32 on tcgen05): OA frozen = A + strip copy, 32 W columns per launch
-        Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 12.0 * M * b, 3 * 2.0 * M * M * b);
-        SBR_CK(zero_matrix(M, b, h->Xb + tb * ldn, ldn, st), "zero X_t");
+        Scope sc(h, SBR_K_PASS, (4.0 * M * M / 2 + 12.0 * M * b) / P, 3 * 2.0 * M * M * b / P);
+        // distributed: the padding rows between X_t's columns are zeroed too (the all-reduce spans them)
+        SBR_CK(zero_matrix(dist ? ldn : M, b, h->Xb + tb * ldn, ldn, st), "zero X_t");
         for (int c = 0; c < b; c += 32) {
           const int bh = std::min(32, b - c);
-          SBR_CK(split_tf32_w(M, bh, 32, Wb + (tb + c) * ldwb, ldwb, h->WS, h->ldws, st), "split W_t");
+          if (leadJ) SBR_CK(split_tf32_w(M, bh, 32, Wb + (tb + c) * ldwb, ldwb, h->WS, h->ldws, st), "split W_t");
+          if (dist) SBR_CM(h->comm->broadcast(h->WS, (size_t)h->ldws * 64 * sizeof(float), own, st), "broadcast W_t");
           PassTf32Launch pl{};
+          if (dist) {   // this rank's tile columns of the 128-aligned grid from the block start
+            pl.off = off;
+            pl.own_P = P;
+            pl.own_rank = rank;
+            pl.nbo = nb;
+            pl.ncols = ncols_loc;
+          }
           pl.A = A;
           pl.n = n;
           pl.lda = lda;
@@ -807,13 +816,15 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           h->launches += 2;
         }
         h->launches += 1;
+        if (dist)
+          SBR_CM(h->comm->all_reduce_sum_f32(h->Xb + tb * ldn, (size_t)(b - 1) * ldn + M, st), "all-reduce X_t");
       } else {  // ---- a4 (3xTF32 mode, SIMT fp32): OA frozen = A + strip copy
         Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 8.0 * M * b, 2.0 * M * M * b);
         SBR_CK(sym_pass(M, b, OA, lda, h->Strip, ldn, sw, Wb + tb * ldwb, ldwb, h->Xb + tb * ldn, ldn, st),
                "pass");
         h->launches += 1;
       }
-      {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
+      if (leadJ) {  // W^T X column block (P:223 l.9 needs W^T OA W) -> WtX[:, tb:tb+b] and mirror
         Scope sc(h, SBR_K_WMERGE, 4.0 * M * (k + 2 * b), 2.0 * M * (k + b) * b);
         SBR_CK(zero_matrix(k + b, b, h->WtX + tb * nb, nb, st), "zero wtx");
         SBR_CK(gemm_tn(M, k + b, b, 1.f, Wb, ldwb, h->Xb + tb * ldn, ldn, h->WtX + tb * nb, nb, st), "W^T X");
@@ -827,6 +838,10 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
     const int kk = p * b;
     if (Mt > 0 && tc16 && dist) {   // the owner's Y (fp16) and W^T X for every rank's trailing update
       SBR_CM(h->comm->broadcast(h->Yh, (size_t)M * h->ldk * sizeof(__half), own, st), "broadcast Y");
+      SBR_CM(h->comm->broadcast(h->WtX, (size_t)nb * nb * sizeof(float), own, st), "broadcast W^T X");
+    }
+    if (Mt > 0 && tc32 && dist) {   // 3xTF32: Y in fp32 (split on every rank)
+      SBR_CM(h->comm->broadcast(h->Yb, (size_t)ldn * kk * sizeof(float), own, st), "broadcast Y");
       SBR_CM(h->comm->broadcast(h->WtX, (size_t)nb * nb * sizeof(float), own, st), "broadcast W^T X");
     }
     if (Mt > 0 && tc16) {
@@ -909,9 +924,15 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       gs.ld_a = gs.ld_b = h->ldts;
       gs.arow0 = gs.brow0 = s;
       gs.Mrows = gs.Ncols = Mt;
-      gs.C = A + (r0 + s) + (r0 + s) * lda;
+      gs.C = A + (r0 + s) + (dist ? 0 : (r0 + s) * lda);   // distributed: local columns via the ownership map
       gs.ldc = lda;
       gs.num_sms = h->nsm;
+      if (dist) {   // this rank's columns of the trailing region only
+        gs.own_P = P;
+        gs.own_rank = rank;
+        gs.own_org = r0 + s;
+        gs.nbo = nb;
+      }
       SBR_CK(launch_syr2k_tf32(gs, st), "syr2k_tf32");
       h->launches += 4;
     } else if (Mt > 0) {
@@ -1554,10 +1575,15 @@ int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A
     if (!h->comm) return SBR_ERR_NCCL;
     // the tensor-core FP16 path with column blocks that align with the pass's tile groups and the
     // SYR2K's tiles (configs 4/5: nb = 1024 / 2048)
-    if (mode != SBR_FP16_FP32ACC || b % 8 != 0 || nb % pass_dist_align(b) != 0 || nb % 256 != 0) {
+    // FP16: the pass's 128-row tile groups (pass_dist_align); 3xTF32: 128-column tiles, b % 4 == 0 and
+    // a 16-byte aligned A; both: the SYR2K's 256-column tiles
+    const bool ok16 = mode == SBR_FP16_FP32ACC && b % 8 == 0 && nb % pass_dist_align(b) == 0 && nb % 256 == 0;
+    const bool ok32 = mode == SBR_3XTF32 && h->tf32_tc && b % 4 == 0 && nb % 256 == 0 && lda % 4 == 0 &&
+                      ((uintptr_t)A & 15) == 0;
+    if (!ok16 && !ok32) {
       std::lock_guard<std::mutex> lk(g_err_mu);
-      g_last_err = "sbr_reduce_dist with nranks > 1: FP16 mode, b % 8 == 0, nb a multiple of " +
-                   std::to_string(pass_dist_align(b));
+      g_last_err = "sbr_reduce_dist with nranks > 1: FP16 mode with b % 8 == 0 and nb a multiple of " +
+                   std::to_string(pass_dist_align(b)) + ", or 3xTF32 with b % 4 == 0 and nb a multiple of 256";
       return SBR_ERR_UNSUPPORTED;
     }
   }

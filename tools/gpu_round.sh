@@ -36,9 +36,11 @@ for s in $STEPS; do
       python tools/launch_summary.py $O/launches_$TAG.csv > $O/launches_$TAG.txt 2>&1;;
     ncu)
       for k in ${NCU_KERNELS:-pass_tc_kernel}; do
-        timeout 900 ncu --set full --clock-control none --import-source on -k regex:$k -s ${NCU_SKIP:-300} -c 1 \
-          -o $O/full_${k}_$TAG -f python tools/prof_run.py $PROF_ARGS > $O/ncu_full_${k}_$TAG.log 2>&1
-        python tools/ncu_summary.py $O/full_${k}_$TAG.ncu-rep > $O/ncu_full_${k}_$TAG.txt 2>&1
+        kn=$(echo "$k" | tr -c 'A-Za-z0-9_\n' '_')
+        sk=${NCU_SKIP:-300}; case $k in *gemm_tc*|*chain*|*s2_*) sk=${NCU_SKIP_GEMM:-0};; esac
+        timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base ${NCU_BASE:-function} \
+          -k "regex:$k" -s $sk -c 1 -o $O/full_${kn}_$TAG -f python tools/prof_run.py $PROF_ARGS > $O/ncu_full_${kn}_$TAG.log 2>&1
+        python tools/ncu_summary.py $O/full_${kn}_$TAG.ncu-rep > $O/ncu_full_${kn}_$TAG.txt 2>&1
       done;;
     sanitize)
       for tool in racecheck synccheck memcheck; do
