@@ -419,7 +419,7 @@ def main():
     # capture (profiles/traffic.json), times this run's algorithmic bytes per launch
     try:
         with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
-            tr = json.load(f).get(dom)
+            tr = json.load(f).get(f"{dom}:{mode}")   # captures are per kernel AND mode (fp16 / 3xtf32 kernels differ)
         if tr:
             roof["traffic"] = tr["dram_per_algorithmic_byte"] * st["bytes"] / max(1, st["launches"])
             roof["traffic_source"] = tr["source"]

@@ -227,8 +227,10 @@ int sbr_eigenvalues(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A
  *   On return: A_local holds the owned columns in sbr_reduce's output layout (band + Y below
  *   it), W_local (may be NULL, ldw >= n) the owned blocks' W columns (same local columns), and
  *   AB (rank 0; may be NULL elsewhere) the whole band, assembled over the ranks.  With
- *   nranks > 1: FP16 mode, b % 8 == 0 and nb a multiple of 128 x the pass's tile columns per
- *   group (1024 for b <= 32, 512 for b = 64), else SBR_ERR_UNSUPPORTED.  Same argument
+ *   nranks > 1: FP16 mode with b % 8 == 0 and nb a multiple of 128 x the pass's tile columns
+ *   per group (1024 for b <= 32, 512 for b = 64), or 3xTF32 mode with b % 4 == 0, nb a
+ *   multiple of 256 and A_local 16-byte aligned with lda % 4 == 0 (3xTF32 broadcasts W_t and Y
+ *   in fp32 and every rank splits them); else SBR_ERR_UNSUPPORTED.  Same argument
  *   errors as sbr_reduce; SBR_ERR_NCCL on a communication error (a failing rank can leave
  *   the others blocked in a collective: treat it as fatal for the group).
  * With nranks == 1, sbr_reduce_dist is sbr_reduce. */
