@@ -93,7 +93,8 @@ int64_t sbr_test_pass_owned_tiles(int64_t n, int b, int nb, int64_t c0, int rank
 int sbr_test_panel_declines(sbr_handle_t h, int reset, int64_t* count);
 
 /* Experiment knobs (timing experiments only; process-wide, 0 = production behaviour):
- *   knob 0 (pass experiment bits): 1 = skip the pass's L W MMAs, 2 = skip its L^T W MMAs
+ *   knob 0 (pass experiment bits): 1 = skip the pass's L W MMAs, 2 = skip its L^T W MMAs,
+ *     8 = skip its X reductions (row and column accumulators), 16 = skip the column ones only
  *   (results are WRONG: for timing the stream alone), 4 = normal L2 policy for the OA stream.
  * Returns 0, or -1 for an unknown knob. */
 int sbr_test_set_knob(int knob, int value);

@@ -145,10 +145,62 @@ __global__ void choose_scale_kernel(const double* scan, unsigned* flag, int* kex
   *kexp = k;
 }
 
+// The same scan with 16-byte loads (A 16-byte aligned, lda % 4 == 0): CTAs stride over whole
+// columns, the rows of a column as float4 (scalar head / tail), one atomic per CTA at the end
+// (the one-CTA-per-column-segment version above issues an fp64 atomic per segment).
+__global__ void __launch_bounds__(256) prep_scan_vec_kernel(int64_t n, int64_t ncols, const float* __restrict__ A,
+                                                            int64_t lda, ColMap cm, double* scan) {
+  double s = 0.0;
+  bool bad = false;
+  for (int64_t j = blockIdx.x; j < ncols; j += gridDim.x) {
+    const int64_t g = cm.g(j);
+    const float* col = A + j * lda;
+    const int64_t h0 = min(n, (g + 3) & ~(int64_t)3), t0 = max(h0, n & ~(int64_t)3);
+    for (int64_t i = g + threadIdx.x; i < h0; i += blockDim.x) {   // head (< 4 rows), incl. the diagonal
+      const float v = col[i];
+      if (!isfinite(v)) bad = true;
+      else s += (i == g ? 1.0 : 2.0) * (double)v * (double)v;
+    }
+    for (int64_t i = h0 + 4 * (int64_t)threadIdx.x; i < t0; i += 4 * (int64_t)blockDim.x) {
+      const float4 v = __ldcs(reinterpret_cast<const float4*>(col + i));
+      bad |= !(isfinite(v.x) && isfinite(v.y) && isfinite(v.z) && isfinite(v.w));
+      const double a = v.x, b = v.y, c = v.z, d = v.w;
+      const double q = (a * a + b * b) + (c * c + d * d);
+      s += 2.0 * q - (i == g ? a * a : 0.0);   // the diagonal (i == g: first lane entry) once
+    }
+    for (int64_t i = t0 + threadIdx.x; i < n; i += blockDim.x) {   // tail
+      const float v = col[i];
+      if (!isfinite(v)) bad = true;
+      else s += (i == g ? 1.0 : 2.0) * (double)v * (double)v;
+    }
+  }
+  if (bad) s = 0.0;
+  const int anybad = __syncthreads_or(bad);
+  __shared__ double red[32];
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+  if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = s;
+  __syncthreads();
+  if (threadIdx.x < 32) {
+    s = threadIdx.x < (blockDim.x >> 5) ? red[threadIdx.x] : 0.0;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (threadIdx.x == 0) {
+      if (s != 0.0) atomicAdd(scan, s);
+      if (anybad) atomicAdd(scan + 1, 1.0);
+    }
+  }
+}
+
 cudaError_t prep_scan(int64_t n, int64_t ncols, const float* A, int64_t lda, ColMap cm, double* scan,
                       cudaStream_t st) {
   cudaError_t e = cudaMemsetAsync(scan, 0, 2 * sizeof(double), st);
   if (e != cudaSuccess) return e;
+  if (lda % 4 == 0 && ((uintptr_t)A & 15) == 0) {
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ncols, (int64_t)current_device_sms() * 8));
+    prep_scan_vec_kernel<<<grid, 256, 0, st>>>(n, ncols, A, lda, cm, scan);
+    return cudaGetLastError();
+  }
   for (int64_t j0 = 0; j0 < ncols; j0 += 65535) {
     const int64_t nc = std::min<int64_t>(65535, ncols - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 16), (unsigned)nc);
@@ -325,9 +377,69 @@ __global__ void shadow_init_kernel(int64_t n, int64_t j0, float* A, int64_t lda,
   }
 }
 
+// 16-byte version (A 16-byte aligned with lda % 4 == 0, shadow 8-byte aligned with ldsh % 4 == 0):
+// CTAs stride over columns, 4 rows per thread step (float4 in/out, 4 halves out).
+__global__ void __launch_bounds__(256) shadow_init_vec_kernel(int64_t n, int64_t ncols, float* __restrict__ A,
+                                                              int64_t lda, __half* __restrict__ Sh, int64_t ldsh,
+                                                              const int* kexp, ColMap cm) {
+  const int k = kexp ? *kexp : 0;
+  const int64_t n4 = n & ~(int64_t)3;
+  for (int64_t j = blockIdx.x; j < ncols; j += gridDim.x) {
+    const int64_t g = cm.g(j);
+    float* col = A + j * lda;
+    __half* sc = Sh + j * ldsh;
+    for (int64_t i = 4 * (int64_t)threadIdx.x; i < n4; i += 4 * (int64_t)blockDim.x) {
+      float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+      if (i + 3 >= g) {
+        v = *reinterpret_cast<const float4*>(col + i);
+        float* e = &v.x;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          if (i + u < g) e[u] = 0.f;
+          else if (k != 0) e[u] = k == kScaleZero ? 0.f : scale_pow2(e[u], k);
+        }
+        if (k != 0) {   // the scaled master (rows above the diagonal keep their values)
+          if (i >= g) {
+            *reinterpret_cast<float4*>(col + i) = v;
+          } else {
+#pragma unroll
+            for (int u = 0; u < 4; ++u)
+              if (i + u >= g) col[i + u] = e[u];
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u)
+          if (i + u == g) e[u] *= 0.5f;
+      }
+      __half2 h01 = __floats2half2_rn(v.x, v.y), h23 = __floats2half2_rn(v.z, v.w);
+      uint2 pk;
+      pk.x = *reinterpret_cast<uint32_t*>(&h01);
+      pk.y = *reinterpret_cast<uint32_t*>(&h23);
+      *reinterpret_cast<uint2*>(sc + i) = pk;
+    }
+    for (int64_t i = n4 + threadIdx.x; i < n; i += blockDim.x) {   // tail rows
+      float v = 0.f;
+      if (i >= g) {
+        v = col[i];
+        if (k != 0) {
+          v = k == kScaleZero ? 0.f : scale_pow2(v, k);
+          col[i] = v;
+        }
+        if (i == g) v *= 0.5f;
+      }
+      sc[i] = __float2half_rn(v);
+    }
+  }
+}
+
 cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ldsh, const int* kexp,
                         cudaStream_t st, int64_t ncols, ColMap cm) {
   if (ncols < 0) ncols = n;
+  if (lda % 4 == 0 && ((uintptr_t)A & 15) == 0 && ldsh % 4 == 0 && ((uintptr_t)Sh & 7) == 0) {
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ncols, (int64_t)current_device_sms() * 8));
+    shadow_init_vec_kernel<<<grid, 256, 0, st>>>(n, ncols, A, lda, Sh, ldsh, kexp, cm);
+    return cudaGetLastError();
+  }
   for (int64_t j0 = 0; j0 < ncols; j0 += 65535) {
     const int64_t nc = std::min<int64_t>(65535, ncols - j0);
     dim3 grid((unsigned)std::min<int64_t>((n + 255) / 256, 32), (unsigned)nc);

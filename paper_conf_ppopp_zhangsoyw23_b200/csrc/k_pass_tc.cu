@@ -26,7 +26,12 @@ struct PassCfg {
   static constexpr int OFF_L = (C + 2) * WT;
   static constexpr int OFF_BAR = OFF_L + NS * LT;
   static constexpr int NBAR = 2 * NS + 4 + 4 + 4;
-  static constexpr int SMEM = OFF_BAR + NBAR * 8 + 16 + 1024;  // + alignment slack
+  // epilogue transpose buffers (one 32 x 33 fp32 block per epilogue warp) for 16-byte reductions
+  // into X, when they fit next to the pipeline
+  static constexpr int OFF_T = OFF_BAR + NBAR * 8 + 16;
+  static constexpr int TBYTES = 4 * 32 * 33 * 4;
+  static constexpr bool VT = OFF_T + TBYTES + 1024 <= 232448;
+  static constexpr int SMEM = OFF_T + (VT ? TBYTES : 0) + 1024;  // + alignment slack
   static constexpr int TMEM_USED = (C + 2) * BN;
   static constexpr int TMEM_COLS = TMEM_USED <= 32 ? 32 : TMEM_USED <= 64 ? 64 : TMEM_USED <= 128 ? 128
                                    : TMEM_USED <= 256 ? 256 : 512;
@@ -113,6 +118,11 @@ struct PassWalk {
     I = J = J0;
   }
 };
+
+SBR_DEV void red_add_v4(float* addr, float a, float b, float c, float d) {
+  asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(addr), "f"(a), "f"(b), "f"(c), "f"(d)
+               : "memory");
+}
 
 template <int BN, int C, int NS>
 __global__ void __launch_bounds__(256, 1)
@@ -280,22 +290,48 @@ __global__ void __launch_bounds__(256, 1)
     int rb = 0; uint32_t rph = 0;
     uint32_t cph = 0;
     uint32_t touched = 0;
+    // X += this warp's 32 rows (rows rbase + lane) x columns c0 .. c0 + 31.  Column-major X: with
+    // 16-byte alignment, the block goes through shared memory so that each lane issues 8 reductions
+    // of 4 consecutive rows of one column (red.global.add.v4.f32: a quarter of the L2 atomic
+    // operations of per-element reductions, which cost ~8 ms per config-4 step at the launch
+    // tails); otherwise per element.
+    float* tb = (float*)(smem + Cfg::OFF_T) + q * (32 * 33);
+    const bool vec = Cfg::VT && M % 4 == 0 && off % 4 == 0 && ldx % 4 == 0 && ((uintptr_t)X & 15) == 0;
+    auto flush32 = [&](const float (&v)[32], int64_t rbase, int c0) {
+      if (vec) {
+#pragma unroll
+        for (int c = 0; c < 32; ++c) tb[c * 33 + lane] = v[c];
+        __syncwarp();
+        const int r4 = 4 * (lane & 7);
+        const int64_t r = rbase + r4;
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const int c = (lane >> 3) + 4 * k;
+          const float* src = tb + c * 33 + r4;
+          if (c0 + c < b && r >= 0 && r < M) red_add_v4(&X[r + (int64_t)(c0 + c) * ldx], src[0], src[1], src[2], src[3]);
+        }
+        __syncwarp();
+      } else {
+        const int64_t row = rbase + lane;
+        if (row >= 0 && row < M) {
+#pragma unroll
+          for (int c = 0; c < 32; ++c)
+            if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
+        }
+      }
+    };
     for (w.start(NT, C, t_beg, t_end - t_beg, own); w.valid(); w.next()) {
       if (w.gfirst) touched = 0;
       touched |= 1u << (w.J - w.J0);
       if (w.rlast()) {
         mbar_wait(&racc_full[rb], rph);
         tc_fence_after();
-        const int64_t row = (int64_t)w.I * 128 + row_in_tile - off;
+        const int64_t rbase = (int64_t)w.I * 128 + q * 32 - off;
 #pragma unroll
         for (int c0 = 0; c0 < BN; c0 += 32) {
           float v[32];
           tmem_ld32(t_row + rb * BN + c0 + lane_off, v);
-          if (row >= 0 && row < M) {
-#pragma unroll
-            for (int c = 0; c < 32; ++c)
-              if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
-          }
+          if (!(exper & 8)) flush32(v, rbase, c0);
         }
         tc_fence_before();
         mbar_arrive(&racc_empty[rb]);
@@ -307,16 +343,12 @@ __global__ void __launch_bounds__(256, 1)
         tc_fence_after();
         for (int jj = 0; jj < w.ceff; ++jj) {
           if (!((touched >> jj) & 1u)) continue;
-          const int64_t row = (int64_t)(w.J0 + jj) * 128 + row_in_tile - off;
+          const int64_t rbase = (int64_t)(w.J0 + jj) * 128 + q * 32 - off;
 #pragma unroll
           for (int c0 = 0; c0 < BN; c0 += 32) {
             float v[32];
             tmem_ld32(t_col + jj * BN + c0 + lane_off, v);
-            if (row >= 0 && row < M) {
-#pragma unroll
-              for (int c = 0; c < 32; ++c)
-                if (c0 + c < b) atomicAdd(&X[row + (int64_t)(c0 + c) * ldx], v[c]);
-            }
+            if (!(exper & 24)) flush32(v, rbase, c0);
           }
         }
         tc_fence_before();
