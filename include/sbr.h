@@ -106,10 +106,10 @@ int sbr_workspace_query(sbr_handle_t h, int64_t n, int b, int nb, int mode, size
  * Returns (argument checks, enqueue failures) 0, -i, SBR_ERR_CUDA, SBR_ERR_NOMEM, or an error
  * LATCHED by an earlier call on this handle.  The call never synchronises the host: errors
  * detected on the device -- SBR_ERR_NONFINITE (Inf/NaN in the referenced input, or a
- * non-finite band entry, i.e. fp16 range exceeded after scaling) and SBR_ERR_UNSUPPORTED (a
- * panel taller than the TSQR fallback's capacity, 148 x 256 rows at b <= 32, n >~ 37900, was
- * numerically rank deficient for CholeskyQR) -- are latched and returned by sbr_sync or by
- * the next call on the handle; the outputs of that reduction are then invalid. */
+ * non-finite band entry, i.e. fp16 range exceeded after scaling) -- are latched and returned
+ * by sbr_sync or by the next call on the handle; the outputs of that reduction are then
+ * invalid.  A panel that CholeskyQR declines (numerically rank deficient) is factored by
+ * Householder QR inside the same kernel, at any height: rank deficiency is not an error. */
 int sbr_reduce(sbr_handle_t h, int mode, int64_t n, int b, int nb,
                float* A, int64_t lda, float* AB, int64_t ldab, float* W, int64_t ldw);
 

@@ -34,7 +34,8 @@ int sbr_test_syr2k_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int sbr_test_zform_fp16(sbr_handle_t h, int64_t M, int K, const float* Y, int64_t ldy, const float* G, int64_t ldg,
                         const float* X, int64_t ldx, float* Z, int64_t ldz);
 
-/* One panel factorisation (TSQR + reconstruction, steps a1-a2) of the m x b panel P
+/* One panel factorisation (steps a1-a2: CholeskyQR + reconstruction with the in-kernel
+ * Householder fallback for m > 512, the paper's TSQR for m <= 512 or SBR_PANEL=tsqr) of the m x b panel P
  * (overwritten with the compact form); explicit Y and W = Y T (m x b, ld ldyw).  If
  * trace != NULL it receives 16 int64 globaltimer stamps (ns) of the kernel's phases. */
 int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_t ldp, float* Y, float* W, int64_t ldyw,
@@ -88,7 +89,7 @@ int sbr_test_zform_tf32(sbr_handle_t h, int64_t M, int K, const float* Y, int64_
 int64_t sbr_test_pass_owned_tiles(int64_t n, int b, int nb, int64_t c0, int rank, int nranks, int* IJ, int64_t cap);
 
 /* Number of CholeskyQR panels that declined (rank deficient / not orthonormal after three
- * rounds, so the paper's TSQR factored them) since the handle's workspace was allocated or
+ * rounds, so the kernel's Householder QR fallback factored them) since the handle's workspace was allocated or
  * the last call with reset != 0.  Synchronises.  Returns 0, -1 (h), -3 (count NULL). */
 int sbr_test_panel_declines(sbr_handle_t h, int reset, int64_t* count);
 

@@ -48,7 +48,9 @@ template <int B> constexpr int pc_ngrp() { return PC_THREADS / pc_nt<B>() > 0 ? 
 constexpr size_t PCW_SETS = 0;
 constexpr size_t PCW_CTL = PCW_SETS + sizeof(double) * 2 * PC_NSET * PC_NCOPY * PC_SETSTRIDE;
 constexpr size_t PCW_LU = PCW_CTL + 256;
-constexpr size_t PCW_BYTES = PCW_LU + sizeof(float) * (2 * 64 * 64 + 2 * 64);
+constexpr size_t PCW_FB = PCW_LU + sizeof(float) * (2 * 64 * 64 + 2 * 64);   // Householder fallback:
+// [64 x 64 doubles: per-column sums x_2^T p_c][64 x 64 doubles: V^T V][64 x 64 floats: R rows]
+constexpr size_t PCW_BYTES = PCW_FB + sizeof(double) * 2 * 64 * 64 + sizeof(float) * 64 * 64;
 
 size_t panel_chol_ws_bytes() { return PCW_BYTES; }
 int* panel_chol_fail(void* ws) { return reinterpret_cast<int*>((char*)ws + PCW_CTL) + 3; }
@@ -532,6 +534,158 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     }
   };
 
+  // rows of the block above the panel: Y = W = 0
+  auto zero_above = [&]() {
+    const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t nth = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = tid; i < a.row0; i += nth) {
+#pragma unroll
+      for (int c = 0; c < B; ++c) {
+        a.Y[i + c * a.ldy] = 0.f;
+        a.W[i + c * a.ldw] = 0.f;
+        if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
+        if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
+      }
+      if (a.Yh) {
+#pragma unroll
+        for (int c = 0; c < B; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
+      }
+    }
+  };
+
+  // ---- Householder QR fallback (CholeskyQR declined: numerically rank deficient, or not
+  //      orthonormal after three rounds).  dgeqr2 on the fp32 panel in global memory, fp64
+  //      sums: per column j ONE grid reduction of t_c = x_2^T p_c (c >= j; x_2 = rows > j of
+  //      column j), then every CTA forms dlarfg's (beta, tau) and w_c = tau (p_jc + t_c / (alpha -
+  //      beta)) and updates its own rows; row j (R) goes to a side buffer so no CTA reads a row
+  //      another one is writing.  Then T (dlarft) from V^T V (one more reduction) and the same
+  //      outputs as the CholeskyQR path: Y = V, W^0 = V T, compact panel [R; V].
+  auto hh_fallback = [&](unsigned& nb_) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+      *fail = 0;
+      atomicAdd(ctl + 4, 1u);   // declines since the workspace was zeroed (sbr_test_panel_declines)
+    }
+    double* fsum = reinterpret_cast<double*>(ws + PCW_FB);
+    double* fvv = fsum + 64 * 64;
+    float* fR = reinterpret_cast<float*>(fvv + 64 * 64);
+    float* P = a.P;
+    const int64_t ldp = a.ldp;
+    for (int e = blockIdx.x * blockDim.x + threadIdx.x; e < 2 * 64 * 64; e += G * blockDim.x) fsum[e] = 0.0;
+    __syncthreads();   // Gpart (smem scratch below) is free: all Gram traffic is complete
+    bar_arrive(ctr);
+    bar_wait(ctr, (unsigned)G * ++nb_);
+    double* wsm = Gpart;           // smem: w_c [B]
+    double* taus = Gpart + 64;     // tau [B]
+    double* Tm = Gpart + 128;      // T [B x B] row-major (fp64)
+    float* Tf = reinterpret_cast<float*>(Tm + B * B);   // T as fp32
+    const int64_t rb = r_beg, re = r_end;
+    for (int j = 0; j < B; ++j) {
+      const int64_t i0 = std::max<int64_t>(rb, j + 1);
+      for (int c = j + warp; c < B; c += PC_THREADS / 32) {
+        double sacc = 0.0;
+        for (int64_t il = i0 + lane; il < re; il += 32)
+          sacc = fma((double)__ldcg(P + il + (int64_t)j * ldp), (double)__ldcg(P + il + (int64_t)c * ldp), sacc);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) sacc += __shfl_xor_sync(0xffffffffu, sacc, o);
+        if (lane == 0 && sacc != 0.0) atomicAdd(fsum + j * 64 + c, sacc);
+      }
+      bar_arrive(ctr);
+      bar_wait(ctr, (unsigned)G * ++nb_);
+      const double sig2 = __ldcg(fsum + j * 64 + j);
+      const double alpha = (double)__ldcg(P + j + (int64_t)j * ldp);
+      double tj, bj, scal;
+      if (!(sig2 > 0.0)) {   // x_2 = 0: H = I (dlarfg: tau = 0, beta = alpha)
+        tj = 0.0;
+        bj = alpha;
+        scal = 0.0;
+      } else {
+        const double nrm = sqrt(fma(alpha, alpha, sig2));
+        bj = alpha >= 0.0 ? -nrm : nrm;
+        tj = (bj - alpha) / bj;
+        scal = 1.0 / (alpha - bj);
+      }
+      const bool own_j = (j >= rb && j < re);
+      if (threadIdx.x < B) {
+        const int c = threadIdx.x;
+        if (c > j) {
+          const double pj = (double)__ldcg(P + j + (int64_t)c * ldp);
+          const double wc = tj * (pj + scal * __ldcg(fsum + j * 64 + c));
+          wsm[c] = wc;
+          if (own_j) fR[j * 64 + c] = (float)(pj - wc);
+        } else if (c == j) {
+          taus[j] = tj;
+          if (own_j) fR[j * 64 + j] = (float)bj;
+        }
+      }
+      __syncthreads();
+      for (int64_t il = i0 + threadIdx.x; il < re; il += blockDim.x) {
+        const double v = (double)P[il + (int64_t)j * ldp] * scal;
+        P[il + (int64_t)j * ldp] = (float)v;
+        for (int c = j + 1; c < B; ++c) {
+          float* pc = P + il + (int64_t)c * ldp;
+          *pc = (float)fma(-v, wsm[c], (double)*pc);
+        }
+      }
+      __syncthreads();
+    }
+    // V^T V (strict upper; v_i = 1 at row i, 0 above): one warp per pair, lanes over rows >= j2
+    for (int e = warp; e < B * B; e += PC_THREADS / 32) {
+      const int i = e / B, j2 = e % B;
+      if (j2 <= i) continue;
+      double sv = 0.0;
+      for (int64_t il = std::max<int64_t>(rb, j2) + lane; il < re; il += 32) {
+        const double vj = (il == j2) ? 1.0 : (double)P[il + (int64_t)j2 * ldp];
+        sv = fma((double)P[il + (int64_t)i * ldp], vj, sv);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) sv += __shfl_xor_sync(0xffffffffu, sv, o);
+      if (lane == 0 && sv != 0.0) atomicAdd(fvv + i * 64 + j2, sv);
+    }
+    bar_arrive(ctr);
+    bar_wait(ctr, (unsigned)G * ++nb_);
+    // T (dlarft forward columnwise): T_jj = tau_j, T[0:j, j] = -tau_j T[0:j, 0:j] (V^T v_j)
+    for (int e = threadIdx.x; e < B * B; e += blockDim.x) Tm[e] = 0.0;
+    __syncthreads();
+    if (warp == 0) {
+      for (int j = 0; j < B; ++j) {
+        for (int i = lane; i < j; i += 32) {
+          double sacc = 0.0;
+          for (int l = i; l < j; ++l) sacc = fma(Tm[i * B + l], __ldcg(fvv + l * 64 + j), sacc);
+          Tm[i * B + j] = -taus[j] * sacc;
+        }
+        if (lane == 0) Tm[j * B + j] = taus[j];
+        __syncwarp();
+      }
+    }
+    __syncthreads();
+    for (int e = threadIdx.x; e < B * B; e += blockDim.x) Tf[e] = (float)Tm[e];
+    __syncthreads();
+    // outputs per row: y = v, w = v T, compact panel
+    for (int64_t il = rb + threadIdx.x; il < re; il += blockDim.x) {
+      const int64_t gr = a.row0 + il;
+      float v[B];
+#pragma unroll
+      for (int c = 0; c < B; ++c) v[c] = (il > c) ? P[il + (int64_t)c * ldp] : (il == c ? 1.f : 0.f);
+      __align__(16) __half yh[B];
+#pragma unroll
+      for (int c = 0; c < B; ++c) {
+        float w = 0.f;
+#pragma unroll
+        for (int k = 0; k <= c; ++k) w = fmaf(v[k], Tf[k * B + c], w);
+        a.W[gr + (int64_t)c * a.ldw] = w;
+        if (a.Wh) a.Wh[gr + (int64_t)c * a.ldwh] = __float2half_rn(w);
+        if (a.Wrh) a.Wrh[gr * a.ldwrh + c] = __float2half_rn(w);
+        a.Y[gr + (int64_t)c * a.ldy] = v[c];
+        yh[c] = __float2half_rn(v[c]);
+        if (il <= c) P[il + (int64_t)c * ldp] = __ldcg(fR + il * 64 + c);   // R (il < B here)
+      }
+      if (a.Yh) {
+#pragma unroll
+        for (int c = 0; c < B; ++c) a.Yh[gr * a.ldyh + c] = yh[c];
+      }
+    }
+  };
+
   // ---- round 0: G = P^T P, R_0 = chol(G), Q = P R_0^-1
   gram_zero();
   gram_acc(crows(0));
@@ -544,13 +698,12 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   gram_arrive(0);
   stamp(2);
   bar_wait(ctr, (unsigned)G);
+  unsigned nbar = 1;   // grid barriers passed (the counter target of the next is G * (nbar + 1))
   stamp(3);
   gram_read(0);
-  if (!chol(0.0)) {                    // not numerically SPD: leave the panel to TSQR
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-      *fail = 1;
-      atomicAdd(ctl + 4, 1u);   // declines since the workspace was zeroed (sbr_test_panel_declines)
-    }
+  if (!chol(0.0)) {                    // not numerically SPD: Householder QR in this launch
+    hh_fallback(nbar);
+    zero_above();
     return;
   }
   stamp(4);
@@ -579,6 +732,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     }
     if (k == 1) stamp(7);
     bar_wait(ctr, (unsigned)G * (k + 1));
+    nbar = k + 1;
     if (k == 1) stamp(8);
     gram_read(k);
     double dev = 0.0;
@@ -594,11 +748,9 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     if (!stream) solve(Rrm, rd, rows);
     if (blockIdx.x == 0 || stream) racc_update(false);
   }
-  if (!done) {
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-      *fail = 1;
-      atomicAdd(ctl + 4, 1u);   // declines since the workspace was zeroed (sbr_test_panel_declines)
-    }
+  if (!done) {   // still not orthonormal after three rounds: Householder QR in this launch
+    hh_fallback(nbar);
+    zero_above();
     return;
   }
   stamp(9);
@@ -708,22 +860,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     }
   }
   }   // chunks
-  // rows of the block above the panel: Y = W = 0
-  const int64_t tid = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  const int64_t nth = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t i = tid; i < row0; i += nth) {
-#pragma unroll
-    for (int c = 0; c < B; ++c) {
-      a.Y[i + c * a.ldy] = 0.f;
-      a.W[i + c * a.ldw] = 0.f;
-      if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
-      if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
-    }
-    if (a.Yh) {
-#pragma unroll
-      for (int c = 0; c < B; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
-    }
-  }
+  zero_above();
   stamp(11);
 }
 

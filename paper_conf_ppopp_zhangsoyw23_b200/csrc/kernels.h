@@ -48,11 +48,11 @@ struct PanelWs {
 PanelWs panel_ws_sizes(int64_t m_max, int b);
 cudaError_t launch_panel(PanelArgs& a, int max_ctas, cudaStream_t st);
 int panel_max_ctas(int b);
-// shifted CholeskyQR3 (fp64) + reconstruction; *fail = 1 (panel untouched) if rank deficient
 // CholeskyQR panel (k_panel_chol.cu): b in {8,16,32,64}; returns cudaErrorNotSupported when it
-// does not apply (then run TSQR unconditionally).  ws: panel_chol_ws_bytes() bytes, zeroed once
-// at allocation; launch: per-handle launch counter (buffers are double-buffered by its parity).
-// On return the TSQR fallback must be launched with run_if = panel_chol_fail(ws).
+// does not apply (then run TSQR).  A declined panel (rank deficient / not orthonormal after
+// three rounds) is factored by Householder QR in the same launch.  ws: panel_chol_ws_bytes()
+// bytes, zeroed once at allocation; launch: per-handle launch counter (buffers are
+// double-buffered by its parity).
 size_t panel_chol_ws_bytes();
 int* panel_chol_fail(void* ws);
 unsigned* panel_chol_declines(void* ws);   // count of declined CholeskyQR panels (device)

@@ -674,30 +674,26 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         pa.orth_tol = tc16 ? 1e-6 : 1e-8;
         if (h->ptrace && h->ptrace_used < h->ptrace_cap) pa.trace = h->ptrace + 32 * (int64_t)h->ptrace_used++;
         bool chol = false;
-        if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu); TSQR only if it declines
+        if (h->panel_mode == 0 && m > 512) {   // CholeskyQR (k_panel_chol.cu), in-kernel Householder QR if it declines
           const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches, st);
           if (ce == cudaSuccess) {
             h->chol_launches++;   // the Gram-set / barrier parity advances only with a launched kernel
-            pa.run_if = h->pfail;
             h->launches += 1;
             chol = true;
           } else if (ce != cudaErrorNotSupported) {
             SBR_CK(ce, "panel_chol");
           }
         }
-        pa.trace = nullptr;   // the phase trace is CholeskyQR's (the TSQR fallback has its own stamps)
-        const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
-        SBR_CK(te, "panel");
-        if (pa.over_capacity && chol) {
-          // panel taller than the TSQR tree can hold (one co-resident CTA per 256-row leaf): no
-          // fallback; a declined CholeskyQR is recorded and reported after the reduction
-          SBR_CK(note_unhandled(h->pfail, h->flag + 1, st), "note_unhandled");
-        } else if (pa.over_capacity) {
-          std::lock_guard<std::mutex> lk(g_err_mu);
-          g_last_err = "panel of " + std::to_string(m) + " x " + std::to_string(b) +
-                       " exceeds the panel kernels' capacity (CholeskyQR: 148 CTAs x rows in smem)";
-          return SBR_ERR_UNSUPPORTED;
-        } else {
+        pa.trace = nullptr;   // the phase trace is CholeskyQR's (TSQR has its own stamps)
+        if (!chol) {          // the paper's TSQR: panels of <= 512 rows, or SBR_PANEL=tsqr
+          const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
+          SBR_CK(te, "panel");
+          if (pa.over_capacity) {
+            std::lock_guard<std::mutex> lk(g_err_mu);
+            g_last_err = "panel of " + std::to_string(m) + " x " + std::to_string(b) +
+                         " exceeds the TSQR tree's capacity (one co-resident CTA per 256-row leaf)";
+            return SBR_ERR_UNSUPPORTED;
+          }
           h->launches += 1;
         }
       }
@@ -1953,20 +1949,15 @@ extern "C" int sbr_test_panel(sbr_handle_t h, int64_t m, int b, float* P, int64_
     const cudaError_t ce = launch_panel_chol(pa, h->chol_ws, h->chol_launches, st);
     if (ce == cudaSuccess) {
       h->chol_launches++;
-      pa.run_if = h->pfail;
       chol = true;
     } else if (ce != cudaErrorNotSupported) {
       SBR_CK(ce, "panel_chol");
     }
   }
-  const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
-  SBR_CK(te, "panel");
-  if (pa.over_capacity && !chol) return SBR_ERR_UNSUPPORTED;
-  if (pa.over_capacity && chol) {   // taller than the TSQR tree: CholeskyQR only (as sbr_reduce)
-    int failed = 0;
-    SBR_CK(cudaMemcpyAsync(&failed, h->pfail, sizeof(int), cudaMemcpyDeviceToHost, st), "fail D2H");
-    SBR_CK(cudaStreamSynchronize(st), "sync");
-    if (failed) return SBR_ERR_UNSUPPORTED;
+  if (!chol) {
+    const cudaError_t te = launch_panel(pa, h->panel_ctas, st);
+    SBR_CK(te, "panel");
+    if (pa.over_capacity) return SBR_ERR_UNSUPPORTED;
   }
   if (trace_host) {
     SBR_CK(cudaMemcpyAsync(trace_host, tr.p, sizeof(int64_t) * 16, cudaMemcpyDeviceToHost, st), "trace D2H");
