@@ -67,12 +67,12 @@ struct CholSmem {
   static constexpr size_t OFF_RRM = OFF_G + sizeof(double) * B * LDG;            // double B x B, R row-major
   static constexpr size_t OFF_RACC = OFF_RRM + sizeof(double) * B * B;           // double B x B (CTA 0: R product)
   static constexpr size_t OFF_RD = OFF_RACC + sizeof(double) * B * B;            // double B (1 / r_jj)
-  static constexpr size_t OFF_RROW = OFF_RD + sizeof(double) * B;                // double B (row broadcast)
+  static constexpr size_t OFF_RROW = OFF_RD + sizeof(double) * B;                // double 2B (row broadcast, padded)
   // L, U alias the Gram partials (Gpart is dead once a round's bulk reduction completed;
   // the LU of a round is recomputed after any later Gram)
   static constexpr size_t OFF_LC = OFF_GP;                                       // float B x B: Lcol[k*B + c] = L[c][k]
   static constexpr size_t OFF_UR = OFF_LC + sizeof(float) * B * B;               // float B x B: Urow[k*B + c] = U[k][c]
-  static constexpr size_t OFF_S = OFF_RROW + sizeof(double) * B;                 // float B signs
+  static constexpr size_t OFF_S = OFF_RROW + sizeof(double) * 2 * B;             // float B signs
   static constexpr size_t OFF_DI = OFF_S + sizeof(float) * B;                    // float B 1/U[k][k]
   static constexpr size_t OFF_LR = OFF_DI + sizeof(float) * B;
   static constexpr size_t OFF_RDA = (OFF_LR + sizeof(float) * B + 15) / 16 * 16;   // double B: 1 / Racc_jj
@@ -102,13 +102,14 @@ SBR_DEV void bar_wait(const unsigned* ctr, unsigned target) {
   __syncthreads();
 }
 
-// Cholesky G = R^T R of a B x B (B <= 32) fp64 matrix by ONE warp: lane c holds column c
-// in registers; R row j is broadcast through shared memory (rrow); the next pivot is
-// computed first so the chain per column is shfl -> rsqrt -> mul -> fma.  (Measured on
-// B200, tools/ubench/ubench_fact.cu: ~9.1k cycles for b = 32, vs 9.8k with all-shuffle
-// broadcasts and 14-20k for rolled variants.)  Writes R (upper, row-major) to Rrm,
-// R (upper, ld LDG) to G and 1/r_jj to rd.  Returns false on breakdown
-// (pivot <= floor_rel * max diag).
+// Cholesky G = R^T R of a B x B (B <= 32, power of two) fp64 matrix by ONE warp: lane c holds
+// column c in registers, SHIFTED so that row j sits in slot 0 at step j; R row j is broadcast
+// through shared memory, stored shifted too (rrow[i] = r_{j,j+i}, zero past B) so that every
+// lane reads it with aligned 16-byte loads;
+// the next pivot is computed first so the chain per column is shfl -> rsqrt -> mul -> fma.
+// The step loop is unrolled (measured in the reduction: 5.6 us vs 6.9 us rolled -- one warp
+// streams its straight-line code without the fetch stalls the CTA-wide phases show).  Writes R (upper, row-major) to Rrm, R (upper, ld LDG)
+// to G and 1/r_jj to rd.  Returns false on breakdown (pivot <= floor_rel * max diag).
 template <int B, int LDG>
 SBR_DEV bool warp_chol(double* G, double* Rrm, double* rd, double* rrow, double floor_rel) {
   const int lane = lane_id();
@@ -124,25 +125,26 @@ SBR_DEV bool warp_chol(double* G, double* Rrm, double* rd, double* rrow, double 
   for (int j = 0; j < B; ++j) {
     ok = ok && (piv > floor_rel * dmax);
     const double r = rsqrt(fmax(piv, 1e-300));   // 1 / r_jj
-    const double rjc = g[j] * r;                  // r_jc (lane j: r_jj)
-    g[j] = rjc;
-    if (j + 1 < B) piv = __shfl_sync(0xffffffffu, fma(-rjc, rjc, g[j + 1]), j + 1);
+    const double rjc = (lane >= j) ? g[0] * r : 0.0;   // r_jc (lane j: r_jj)
+    const double pn = __shfl_sync(0xffffffffu, fma(-rjc, rjc, g[1]), (j + 1) & 31);
     if (lane == j) rd[j] = r;
-    if (lane < B) rrow[lane] = rjc;
-    __syncwarp();
-#pragma unroll
-    for (int i = j + 1; i < B; ++i) g[i] = fma(-rrow[i], rjc, g[i]);
-    __syncwarp();
-  }
-  if (lane < B) {
-#pragma unroll
-    for (int i = 0; i < B; ++i) {
-      const double v = (i <= lane) ? g[i] : 0.0;
-      G[i + lane * LDG] = v;
-      Rrm[i * B + lane] = v;
+    if (lane < B) {
+      rrow[(lane - j) & (B - 1)] = rjc;   // shifted: rrow[i] = r_{j, j+i} (zero past B: lanes < j)
+      Rrm[j * B + lane] = rjc;
+      G[j + lane * LDG] = rjc;
     }
+    __syncwarp();
+    const double2* rr2 = reinterpret_cast<const double2*>(rrow);
+#pragma unroll
+    for (int h = 0; h < B / 2; ++h) {
+      const double2 rr = rr2[h];
+      if (h > 0) g[2 * h - 1] = fma(-rr.x, rjc, g[2 * h]);
+      g[2 * h] = fma(-rr.y, rjc, g[2 * h + 1]);
+    }
+    g[B - 1] = 0.0;
+    piv = pn;
+    __syncwarp();
   }
-  __syncwarp();
   return __all_sync(0xffffffffu, ok);
 }
 
@@ -175,43 +177,50 @@ SBR_DEV bool cta_chol(double* G, double* Rrm, double* rd, double floor_rel) {
   return ok;
 }
 
-// Modified LU of Q_1 - S (s_j = -sign(d_j)) of a B x B (B <= 32) matrix by ONE
-// warp (fp32).  Lane c holds column c, shifted so col[k] is row j+k at step j (rolled step
-// loop, static register indices -- see warp_chol); L column j is broadcast from lane j by
-// shuffles.  Writes Lcol[k*B + c] = L[c][k] (unit lower), Urow[k*B + c] = U[k][c], S and
-// dinv = 1/U[k][k].
+// Modified LU of Q_1 - S (s_j = -sign(d_j)) of a B x B (B <= 32) matrix by ONE warp
+// (fp32).  Lane i holds ROW i in registers, shifted so that column j sits in slot 0 at step j;
+// the pivot row is broadcast through a ping-pong shared buffer with 16-byte stores / loads
+// (stage, 2 x B floats), so a step is 2B/4 vector memory ops + B FMAs instead of B shuffles.
+// Writes Lcol[k*B + c] = L[c][k] (unit lower), Urow[k*B + c] = U[k][c], S and dinv = 1/U[k][k].
 template <int B, int LDQ>
-SBR_DEV void warp_lu(const double* Q1, float* Lcol, float* Urow, float* Ss, float* dinv) {
+SBR_DEV void warp_lu(const double* Q1, float* Lcol, float* Urow, float* Ss, float* dinv, float* stage) {
   const int lane = lane_id();
-  float col[B];
+  float x[B];
 #pragma unroll
-  for (int i = 0; i < B; ++i) col[i] = (lane < B) ? (float)Q1[i * LDQ + lane] : 0.f;
+  for (int c = 0; c < B; ++c) x[c] = (lane < B) ? (float)Q1[lane * LDQ + c] : 0.f;
 #pragma unroll 1
   for (int j = 0; j < B; ++j) {
-    const float d = __shfl_sync(0xffffffffu, col[0], j);   // A[j][j]
+    float* st = stage + (j & 1) * B;
+    if (lane == j) {
+#pragma unroll
+      for (int c = 0; c < B; c += 4) *reinterpret_cast<float4*>(st + c) = make_float4(x[c], x[c + 1], x[c + 2], x[c + 3]);
+    }
+    __syncwarp();
+    float u[B];
+#pragma unroll
+    for (int c = 0; c < B; c += 4) {
+      const float4 t = *reinterpret_cast<const float4*>(st + c);
+      u[c] = t.x;
+      u[c + 1] = t.y;
+      u[c + 2] = t.z;
+      u[c + 3] = t.w;
+    }
+    const float d = u[0];                      // A[j][j]
     const float sj = (d >= 0.f) ? -1.f : 1.f;
     const float piv = d - sj;
     const float inv = __fdividef(1.f, piv);
-    const float ujc = (lane == j) ? piv : col[0];   // lane c >= j: U[j][c]
     if (lane < B) {
-      Urow[j * B + lane] = (lane >= j) ? ujc : 0.f;
-      Lcol[lane * B + j] = (lane < j) ? col[0] : (lane == j ? 1.f : 0.f);   // L[j][lane]
+      Urow[j * B + lane] = (lane > j) ? st[(lane - j) & (B - 1)] : (lane == j ? piv : 0.f);
+      const float l = (lane > j) ? x[0] * inv : (lane == j ? 1.f : 0.f);
+      Lcol[j * B + lane] = l;
+#pragma unroll
+      for (int c = 1; c < B; ++c) x[c - 1] = fmaf(-l, u[c], x[c]);
+      x[B - 1] = 0.f;
     }
     if (lane == j) {
       Ss[j] = sj;
       dinv[j] = inv;
     }
-#pragma unroll
-    for (int k0 = 1; k0 < B; k0 += 8) {
-      if (j + k0 < B) {
-#pragma unroll
-        for (int k = k0; k < k0 + 8 && k < B; ++k) {
-          const float lk = __shfl_sync(0xffffffffu, col[k], j) * inv;   // L[j+k][j]
-          col[k - 1] = (lane > j) ? fmaf(-lk, ujc, col[k]) : ((lane == j) ? lk : col[k]);
-        }
-      }
-    }
-    col[B - 1] = 0.f;
   }
   __syncwarp();
 }
@@ -435,43 +444,61 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       return cta_chol<B, LDG>(Gk, Rrm, rd, floor_rel);
     }
   };
-  // Q <- Q R^-1 on Qd rows [0, n): forward substitution, 2 rows per thread (R row-major, rdg = 1/R_jj)
+  // Q <- Q R^-1 on Qd rows [0, n), 2 rows per thread: column-oriented forward substitution over
+  // a SHIFTED copy of R (Rsh[k][i] = R[k][k+i], zero beyond B; in the Gram slot Gk, dead between
+  // a round's Cholesky and the next Gram).  The k loop is rolled and the register row shifts
+  // down one slot per step, so the code is a few hundred instructions: this phase runs once
+  // per panel per SM, and inside the reduction (the pass's stream between panels evicts it)
+  // fetching a fully unrolled triangle's code cost more than its arithmetic.
   auto solve = [&](const double* Rm, const double* rdg, int n) {
+    double* Rsh = Gk;
+    for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+      const int k = e / B, i = e % B;
+      Rsh[e] = (k + i < B) ? Rm[k * B + k + i] : 0.0;
+    }
+    __syncthreads();
     const int half = (n + 1) >> 1;
     for (int r = threadIdx.x; r < half; r += blockDim.x) {
       const int r2 = r + half;
       const bool two = r2 < n;
-      const double2* R2 = reinterpret_cast<const double2*>(Rm);
-      asm volatile("" : "+l"(R2));   // opaque: no hoisting of the b^2 loads out of the row loop
+      double* qrow = Qd + r * LDQ;
+      double* prow = Qd + (two ? r2 : r) * LDQ;
       double q[B], p[B];
 #pragma unroll
       for (int c = 0; c < B; c += 2) {
-        const double2 t = *reinterpret_cast<const double2*>(Qd + r * LDQ + c);
+        const double2 t = *reinterpret_cast<const double2*>(qrow + c);
         q[c] = t.x;
         q[c + 1] = t.y;
-        const double2 u = two ? *reinterpret_cast<const double2*>(Qd + r2 * LDQ + c) : make_double2(0.0, 0.0);
+        const double2 u = *reinterpret_cast<const double2*>(prow + c);
         p[c] = u.x;
         p[c + 1] = u.y;
       }
+#pragma unroll 1
+      for (int k0 = 0; k0 < B; k0 += 2) {
+        double qo[2], po[2];
 #pragma unroll
-      for (int c = 0; c < B; ++c) {
-        q[c] *= rdg[c];
-        p[c] *= rdg[c];
+        for (int s2 = 0; s2 < 2; ++s2) {
+          const int k = k0 + s2;
+          const double rk = rdg[k];
+          const double qk = q[0] * rk, pk = p[0] * rk;
+          qo[s2] = qk;
+          po[s2] = pk;
+          const double2* R2 = reinterpret_cast<const double2*>(Rsh + k * B);
 #pragma unroll
-        for (int h = (c + 1) / 2; h < B / 2; ++h) {
-          const double2 rr = R2[c * (B / 2) + h];
-          if (2 * h > c) {
-            q[2 * h] = fma(-q[c], rr.x, q[2 * h]);
-            p[2 * h] = fma(-p[c], rr.x, p[2 * h]);
+          for (int h = 0; h < B / 2; ++h) {
+            const double2 rr = R2[h];
+            if (h > 0) {
+              q[2 * h - 1] = fma(-qk, rr.x, q[2 * h]);
+              p[2 * h - 1] = fma(-pk, rr.x, p[2 * h]);
+            }
+            q[2 * h] = fma(-qk, rr.y, q[2 * h + 1]);
+            p[2 * h] = fma(-pk, rr.y, p[2 * h + 1]);
           }
-          q[2 * h + 1] = fma(-q[c], rr.y, q[2 * h + 1]);
-          p[2 * h + 1] = fma(-p[c], rr.y, p[2 * h + 1]);
+          q[B - 1] = 0.0;
+          p[B - 1] = 0.0;
         }
-      }
-#pragma unroll
-      for (int c = 0; c < B; c += 2) {
-        *reinterpret_cast<double2*>(Qd + r * LDQ + c) = make_double2(q[c], q[c + 1]);
-        if (two) *reinterpret_cast<double2*>(Qd + r2 * LDQ + c) = make_double2(p[c], p[c + 1]);
+        *reinterpret_cast<double2*>(qrow + k0) = make_double2(qo[0], qo[1]);
+        if (two) *reinterpret_cast<double2*>(prow + k0) = make_double2(po[0], po[1]);
       }
     }
     __syncthreads();
@@ -514,7 +541,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
   };
   auto lu_publish = [&](unsigned gen) {   // CTA 0: LU of Q_1 - S, to smem and to global
     if constexpr (B <= 32) {
-      if (warp == 0) warp_lu<B, LDQ>(Qd, Lc, Ur, Ss, Di);
+      if (warp == 0) warp_lu<B, LDQ>(Qd, Lc, Ur, Ss, Di, reinterpret_cast<float*>(rrow));
       __syncthreads();
     } else {
       cta_lu<B, LDQ>(Qd, Lc, Ur, Ss, Di);
@@ -546,9 +573,10 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
         if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
         if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
       }
-      if (a.Yh) {
+      if (a.Yh) {   // 16-byte row stores
+        const uint4 z = make_uint4(0u, 0u, 0u, 0u);
 #pragma unroll
-        for (int c = 0; c < B; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
+        for (int c = 0; c < B; c += 8) *reinterpret_cast<uint4*>(a.Yh + i * a.ldyh + c) = z;
       }
     }
   };
@@ -774,92 +802,113 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
     *fail = 0;
   }
   stamp(10);
-  // ---- rows: w L_1^T = e_il - q S ;  y = L_1 row (il < B) or y U = q ;  compact panel
+  // ---- rows: w L_1^T = e_il - q S ;  y = L_1 row (il < B) or y U = q ;  compact panel.
+  //      Both triangular solves are column-oriented over SHIFTED fp32 factors (in the dead Rrm
+  //      slot: Lsh[k][i] = L[k+i][k], Ush[k][i] = U[k][k+i], zero beyond B) with the k loop
+  //      rolled in groups of 8 columns; each group's 8 outputs leave as coalesced fp32 / fp16
+  //      column stores and one 16-byte fp16 row store (per-column 2-byte row stores measured
+  //      slower inside the reduction: this phase is bound by its stores, not its arithmetic).
   const int64_t row0 = a.row0;
+  float* Lsh = reinterpret_cast<float*>(Rrm);
+  float* Ush = Lsh + B * B;
+  for (int e = threadIdx.x; e < B * B; e += blockDim.x) {
+    const int k = e / B, c = k + e % B;
+    Lsh[e] = (c < B) ? Lc[k * B + c] : 0.f;
+    Ush[e] = (c < B) ? Ur[k * B + c] : 0.f;
+  }
+  __syncthreads();
+  stamp(12);
   for (int ch = 0; ch < nch; ++ch) {
   const int c0 = ch * CH, nr = crows(ch);
   if (stream) stream_q(ch);   // Q rows of this chunk (resident otherwise)
   for (int r = threadIdx.x; r < nr; r += blockDim.x) {
     const int64_t il = r_beg + c0 + r;
     const int64_t gr = row0 + il;
-    // opaque per-iteration copies of the smem factors: keeps the compiler from hoisting
-    // all b^2 loads out of the row loop (which spills)
-    const float* Lc_ = Lc;
-    const float* Ur_ = Ur;
-    asm volatile("" : "+l"(Lc_), "+l"(Ur_));
-    const float4* Lc4 = reinterpret_cast<const float4*>(Lc_);
-    const float4* Ur4 = reinterpret_cast<const float4*>(Ur_);
-    float qf[B], v_[B];
+    const double* qrow = Qd + r * LDQ;
+    float v[B];
 #pragma unroll
     for (int c = 0; c < B; c += 2) {
-      const double2 t = *reinterpret_cast<const double2*>(Qd + r * LDQ + c);
-      qf[c] = (float)t.x;
-      qf[c + 1] = (float)t.y;
+      const double2 t = *reinterpret_cast<const double2*>(qrow + c);
+      v[c] = ((il == c) ? 1.f : 0.f) - (float)t.x * Ss[c];
+      v[c + 1] = ((il == c + 1) ? 1.f : 0.f) - (float)t.y * Ss[c + 1];
     }
+#pragma unroll 1
+    for (int k0 = 0; k0 < B; k0 += 8) {
+      float wo[8];
 #pragma unroll
-    for (int c = 0; c < B; ++c) v_[c] = ((il == c) ? 1.f : 0.f) - qf[c] * Ss[c];
+      for (int s8 = 0; s8 < 8; ++s8) {
+        const float wk = v[0];
+        wo[s8] = wk;
+        const float4* L4 = reinterpret_cast<const float4*>(Lsh + (k0 + s8) * B);
 #pragma unroll
-    for (int k = 0; k < B; ++k)
-#pragma unroll
-      for (int h = (k + 1) / 4; h < B / 4; ++h) {
-        const float4 l4 = Lc4[k * (B / 4) + h];
-        const float lv[4] = {l4.x, l4.y, l4.z, l4.w};
-#pragma unroll
-        for (int u = 0; u < 4; ++u)
-          if (4 * h + u > k) v_[4 * h + u] = fmaf(-v_[k], lv[u], v_[4 * h + u]);
+        for (int h = 0; h < B / 4; ++h) {
+          const float4 l = L4[h];
+          if (h > 0) v[4 * h - 1] = fmaf(-wk, l.x, v[4 * h]);
+          v[4 * h] = fmaf(-wk, l.y, v[4 * h + 1]);
+          v[4 * h + 1] = fmaf(-wk, l.z, v[4 * h + 2]);
+          v[4 * h + 2] = fmaf(-wk, l.w, v[4 * h + 3]);
+        }
+        v[B - 1] = 0.f;
       }
+      __align__(16) __half wh[8];
 #pragma unroll
-    for (int c = 0; c < B; ++c) a.W[gr + c * a.ldw] = v_[c];
-    if (a.Wh) {
-#pragma unroll
-      for (int c = 0; c < B; ++c) a.Wh[gr + c * a.ldwh] = __float2half_rn(v_[c]);
+      for (int s8 = 0; s8 < 8; ++s8) {
+        const int64_t c = k0 + s8;
+        a.W[gr + c * a.ldw] = wo[s8];
+        wh[s8] = __float2half_rn(wo[s8]);
+        if (a.Wh) a.Wh[gr + c * a.ldwh] = wh[s8];
+      }
+      if (a.Wrh) *reinterpret_cast<uint4*>(a.Wrh + gr * a.ldwrh + k0) = *reinterpret_cast<const uint4*>(wh);
     }
-    if (a.Wrh) {
+    if (r == 0 && ch == 0) stamp(13);
+    float q[B];
 #pragma unroll
-      for (int c = 0; c < B; ++c) a.Wrh[gr * a.ldwrh + c] = __float2half_rn(v_[c]);
+    for (int c = 0; c < B; c += 2) {
+      const double2 t = *reinterpret_cast<const double2*>(qrow + c);
+      q[c] = (float)t.x;
+      q[c + 1] = (float)t.y;
     }
-    if (il < B) {
+#pragma unroll 1
+    for (int k0 = 0; k0 < B; k0 += 8) {
+      float yo[8];
+      if (il >= B) {
 #pragma unroll
-      for (int c = 0; c < B; ++c) v_[c] = Lc_[c * B + il];   // L[il][c]
-    } else {
+        for (int s8 = 0; s8 < 8; ++s8) {
+          const float yk = q[0] * Di[k0 + s8];
+          yo[s8] = yk;
+          const float4* U4 = reinterpret_cast<const float4*>(Ush + (k0 + s8) * B);
 #pragma unroll
-      for (int k = 0; k < B; ++k) {
-        qf[k] *= Di[k];
+          for (int h = 0; h < B / 4; ++h) {
+            const float4 u = U4[h];
+            if (h > 0) q[4 * h - 1] = fmaf(-yk, u.x, q[4 * h]);
+            q[4 * h] = fmaf(-yk, u.y, q[4 * h + 1]);
+            q[4 * h + 1] = fmaf(-yk, u.z, q[4 * h + 2]);
+            q[4 * h + 2] = fmaf(-yk, u.w, q[4 * h + 3]);
+          }
+          q[B - 1] = 0.f;
+        }
+      } else {   // top rows (CTA 0): y = row il of the unit lower L (Lsh[k][il-k] = L[il][k])
 #pragma unroll
-        for (int h = (k + 1) / 4; h < B / 4; ++h) {
-          const float4 u4 = Ur4[k * (B / 4) + h];
-          const float uv[4] = {u4.x, u4.y, u4.z, u4.w};
-#pragma unroll
-          for (int u = 0; u < 4; ++u)
-            if (4 * h + u > k) qf[4 * h + u] = fmaf(-qf[k], uv[u], qf[4 * h + u]);
+        for (int s8 = 0; s8 < 8; ++s8) {
+          const int c = k0 + s8;
+          yo[s8] = (c < il) ? Lsh[c * B + ((int)il - c)] : (c == il ? 1.f : 0.f);
         }
       }
+      __align__(16) __half yh[8];
 #pragma unroll
-      for (int c = 0; c < B; ++c) v_[c] = qf[c];
-    }
-#pragma unroll
-    for (int c = 0; c < B; ++c) {
-      a.Y[gr + c * a.ldy] = v_[c];
-      // compact panel: Y tail strictly below, R_h = S R on and above the diagonal (CTA 0)
-      a.P[il + (int64_t)c * a.ldp] = (il > c) ? v_[c] : (il < B ? (float)((double)Ss[il] * Racc[il * B + c]) : 0.f);
-    }
-    if (a.Yh) {
-      __half* yh = a.Yh + gr * a.ldyh;
-      if constexpr (B % 8 == 0) {
-#pragma unroll
-        for (int c = 0; c < B; c += 8) {
-          __align__(16) __half hv[8];
-#pragma unroll
-          for (int u = 0; u < 8; ++u) hv[u] = __float2half_rn(v_[c + u]);
-          *reinterpret_cast<uint4*>(yh + c) = *reinterpret_cast<const uint4*>(hv);
-        }
-      } else {
-#pragma unroll
-        for (int c = 0; c < B; ++c) yh[c] = __float2half_rn(v_[c]);
+      for (int s8 = 0; s8 < 8; ++s8) {
+        const int c = k0 + s8;
+        a.Y[gr + (int64_t)c * a.ldy] = yo[s8];
+        // compact panel: Y tail strictly below, R_h = S R on and above the diagonal (il < B)
+        a.P[il + (int64_t)c * a.ldp] = (il > c) ? yo[s8] : (float)((double)Ss[il] * Racc[il * B + c]);
+        yh[s8] = __float2half_rn(yo[s8]);
       }
+      if (a.Yh) *reinterpret_cast<uint4*>(a.Yh + gr * a.ldyh + k0) = *reinterpret_cast<const uint4*>(yh);
     }
+    if (r == 0 && ch == 0) stamp(14);
   }
   }   // chunks
+  stamp(15);
   zero_above();
   stamp(11);
 }

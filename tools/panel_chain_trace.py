@@ -35,6 +35,17 @@ for lo, hi in ((0, 32), (480, 512), (960, 992)):
         md = np.nanmedian(d[lo:hi], axis=0)
         print(f"panels {lo}-{hi}: total {np.nanmedian(rel[lo:hi, 11]):.1f} us; " +
               " ".join(f"{names[i]}->{names[i+1]}={md[i]:.1f}" for i in range(11)))
+# output phase detail (stamps 12-15): factor tables, thread 0's first row W / Y, all rows, rows above
+T2 = np.frombuffer(buf, dtype=np.int64)[: 32 * cnt.value].reshape(cnt.value, 32)[:, :16].astype(np.float64)
+o = T2[:, [10, 12, 13, 14, 15, 11]]
+o[o <= 0] = np.nan
+if True:
+    do = np.diff(o, axis=1) / 1e3
+    for lo, hi in ((0, 32), (480, 512), (960, 992)):
+        if hi <= cnt.value:
+            md = np.nanmedian(do[lo:hi], axis=0)
+            print(f"  output phase {lo}-{hi}: tables {md[0]:.1f} row0-W {md[1]:.1f} row0-Y {md[2]:.1f} "
+                  f"other rows {md[3]:.1f} rows-above {md[4]:.1f} us")
 gap = (T[1:, 0] - T[:-1, 11]) / 1e3
 print(f"end(panel t) -> start(panel t+1): median {np.median(gap):.1f} us (the rest of the chain)")
 for m in (32000, 16000, 4000):
