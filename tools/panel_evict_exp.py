@@ -19,6 +19,8 @@ P0 = torch.randn(b, n, device="cuda")
 Y = torch.zeros(b, m, device="cuda"); W = torch.zeros(b, m, device="cuda")
 big = torch.empty(1 << 28, device="cuda")          # 1 GiB, 512 pages of 2 MiB
 small = torch.empty(1 << 22, device="cuda")        # 16 MiB: 8 pages
+mid = torch.empty(40 << 20, device="cuda")         # 160 MiB: 80 pages, more than the 126 MB L2
+tlb_idx = torch.arange(0, 1 << 28, 1 << 19, device="cuda")   # one float per 2 MiB page of big
 sink = torch.empty(1, device="cuda")
 
 def run(pre):
@@ -32,6 +34,10 @@ def run(pre):
                 small.sum()
         elif pre == "write":
             big.fill_(1.0)
+        elif pre == "l2sweep":   # evicts the L2 through 80 pages only
+            mid.sum()
+        elif pre == "tlbsweep":  # touches 512 pages, one 4-byte load each: TLB churn, L2 intact
+            big.index_select(0, tlb_idx).sum()
         tr = (ctypes.c_int64 * 16)()
         _lib.check(lib.sbr_test_panel(h._h, m, b, P.data_ptr(), n, Y.data_ptr(), W.data_ptr(), m, tr), "panel")
         t = np.array([tr[i] for i in range(16)], dtype=np.float64)
@@ -40,6 +46,6 @@ def run(pre):
     r = (t[:12] - t[0]) / 1e3
     print(f"{pre:8s}: " + " ".join(f"{names[i]}->{names[i+1]}={r[i+1]-r[i]:.1f}" for i in range(11)) + f" total {r[11]:.1f}")
 
-for pre in ("warm", "sweep", "write", "l2only", "warm"):
+for pre in ("warm", "sweep", "l2sweep", "tlbsweep", "write", "warm"):
     run(pre)
 h.close()
