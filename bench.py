@@ -526,10 +526,10 @@ def main():
             "seconds_per_step": ms_per_step / 1e3,
             "higher_is_better": True,
             "vs_baseline": None,
-            "dtype": "f32" if mode == "3xtf32" else "f16",
+            "dtype": {"3xtf32": "f32", "bf16": "bf16"}.get(mode, "f16"),
             "data": "synthetic",
             "config": {"workload": f"{cfg_name}: n={n} {input_desc}, b={b}, nb={nb}, "
-                                   f"{'FP16-in/FP32-acc' if mode == 'fp16' else '3xTF32'}",
+                                   f"{ {'fp16': 'FP16-in/FP32-acc', 'bf16': 'BF16-in/FP32-acc (ablation)'}.get(mode, '3xTF32')}",
                        "n": n, "b": b, "nb": nb, "mode": mode,
                        "parallelism": f"sbr_reduce_dist over {world} GPUs: 1D block-cyclic nb-column blocks "
                                       f"(owner factors its panels; pass and SYR2K on own columns; NCCL "

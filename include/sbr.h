@@ -57,8 +57,15 @@ typedef struct sbr_ctx* sbr_handle_t;
  *                      (kind::f16) -- the paper's Tensor Core mode.
  *   SBR_3XTF32       : FP32-accurate "EC-TCGEMM" mode (reading C11):
  *                      a = hi + lo with hi = rna_tf32(a), lo = rna_tf32(a - hi);
- *                      C = hi*hi' + (hi*lo' + lo*hi'). */
-typedef enum { SBR_FP16_FP32ACC = 0, SBR_3XTF32 = 1 } sbr_precision_t;
+ *                      C = hi*hi' + (hi*lo' + lo*hi').
+ *   SBR_BF16_FP32ACC : the FP16 path with bfloat16 operands (RN) instead of fp16 -- an ablation
+ *                      (SURVEY 8(f) f4): same kernels and speed, 8 bits less mantissa (2^-9 vs
+ *                      2^-12 unit roundoff), so its errors are ~8x the FP16 mode's and exceed
+ *                      the 5e-3 FP16 gates; its wider range needs no scaling (a0 still applies).
+ *                      The operand format is a per-device setting written in stream order at the
+ *                      start of each reduction: do not run FP16 and BF16 reductions concurrently
+ *                      on one device.  Not supported by the opt-in fused chain (SBR_FUSED=1). */
+typedef enum { SBR_FP16_FP32ACC = 0, SBR_3XTF32 = 1, SBR_BF16_FP32ACC = 2 } sbr_precision_t;
 
 /* Create a handle on CUDA device `device`, bound to `stream` (a cudaStream_t;
  * NULL = the legacy default stream).  Allocates nothing large.

@@ -21,6 +21,7 @@ SBR_ERR_NOMEM = 4
 SBR_ERR_UNSUPPORTED = 5
 SBR_FP16_FP32ACC = 0
 SBR_3XTF32 = 1
+SBR_BF16_FP32ACC = 2   # ablation: the FP16 path with bfloat16 operands (sbr.h)
 SBR_OUT_BAND, SBR_OUT_Y, SBR_OUT_W = 1, 2, 4
 KERNEL_CLASSES = {"panel": 0, "lazy": 1, "wmerge": 2, "pass": 3, "syr2k": 4, "other": 5, "stage2": 6}
 

@@ -6,7 +6,7 @@ import ctypes
 from . import _lib
 from ._lib import check, lib
 
-MODES = {"fp16": _lib.SBR_FP16_FP32ACC, "3xtf32": _lib.SBR_3XTF32}
+MODES = {"fp16": _lib.SBR_FP16_FP32ACC, "3xtf32": _lib.SBR_3XTF32, "bf16": _lib.SBR_BF16_FP32ACC}
 
 
 def _mode(mode) -> int:

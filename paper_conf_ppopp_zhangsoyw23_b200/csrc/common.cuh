@@ -2,6 +2,7 @@
 #pragma once
 #include <cuda_runtime.h>
 #include <cuda_fp16.h>
+#include <cuda_bf16.h>
 #include <stdint.h>
 #include <algorithm>
 #include <cstdlib>
@@ -35,6 +36,26 @@ SBR_DEV float tf32_rna(float x) {
   asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
   return __uint_as_float(r & 0xffffe000u);
 }
+
+// 16-bit tensor-core operand format of the reduction: IEEE fp16 (SBR_FP16_FP32ACC, the paper's
+// P:348) or bfloat16 (SBR_BF16_FP32ACC, the ablation of SURVEY 8(f) f4) in the same 2-byte
+// storage.  One __constant__ flag per translation unit, set from the host in stream order before
+// a reduction's first kernel (set_op16_all, sbr_api.cu); read by every float -> 16-bit operand
+// conversion and by the kind::f16 instruction descriptors (a/b format bits: 0 f16, 1 bf16).
+static __constant__ int g_op16_bf16;
+SBR_DEV __half cvt16(float x) {
+  if (g_op16_bf16) return __ushort_as_half(__bfloat16_as_ushort(__float2bfloat16_rn(x)));
+  return __float2half_rn(x);
+}
+SBR_DEV float from16(__half h) {
+  if (g_op16_bf16) return __bfloat162float(__ushort_as_bfloat16(__half_as_ushort(h)));
+  return __half2float(h);
+}
+SBR_DEV uint32_t op16_fmt() { return g_op16_bf16 ? ((1u << 7) | (1u << 10)) : 0u; }
+#define SBR_OP16_SETTER(name)                                                                   \
+  cudaError_t set_op16_##name(int bf16, cudaStream_t st) {                                        \
+    return cudaMemcpyToSymbolAsync(g_op16_bf16, &bf16, sizeof(int), 0, cudaMemcpyHostToDevice, st); \
+  }
 
 SBR_DEV int lane_id() { return threadIdx.x & 31; }
 SBR_DEV int warp_id() { return threadIdx.x >> 5; }

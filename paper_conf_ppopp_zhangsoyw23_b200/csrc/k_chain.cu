@@ -126,7 +126,7 @@ __global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
     if (q < k) {
       if (lazy) {
         const float d = __ldcg(a.X + (a.c + p) + (int64_t)q * a.ldx) - s;
-        a.Ph[(int64_t)p * a.ldph + q] = __float2half_rn(d);
+        a.Ph[(int64_t)p * a.ldph + q] = cvt16(d);
       } else {
         const float d = __ldcg(a.H + q + (int64_t)p * a.ldg) - s;
         WtX[q + (int64_t)(k + p) * ldwx] = d;
@@ -146,7 +146,7 @@ __global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
     const int64_t tid = ((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * blockDim.x + threadIdx.x;
     for (int64_t e = tid; e < (int64_t)k * b; e += nth) {
       const int r = (int)(e % k), p = (int)(e / k);
-      a.Gh[r + (int64_t)p * a.ldgh] = __float2half_rn(__ldcg(a.G + r + (int64_t)p * a.ldg));
+      a.Gh[r + (int64_t)p * a.ldgh] = cvt16(__ldcg(a.G + r + (int64_t)p * a.ldg));
     }
   }
   cluster.sync();   // keep this CTA's partials alive until every reader is done
@@ -242,10 +242,10 @@ __global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
     if (vec) {
       __align__(16) __half hv[8];
 #pragma unroll
-      for (int u = 0; u < 8; ++u) hv[u] = __float2half_rn(Xs[r][g * 8 + u]);
+      for (int u = 0; u < 8; ++u) hv[u] = cvt16(Xs[r][g * 8 + u]);
       *reinterpret_cast<uint4*>(dst) = *reinterpret_cast<const uint4*>(hv);
     } else {
-      for (int u = 0; u < 8 && g * 8 + u < b; ++u) dst[u] = __float2half_rn(Xs[r][g * 8 + u]);
+      for (int u = 0; u < 8 && g * 8 + u < b; ++u) dst[u] = cvt16(Xs[r][g * 8 + u]);
     }
   }
   // partial W_t^T X_t over this CTA's rows: thread (ti, tj) owns rows i = ti*BI+u, cols j = tj*BI+v
@@ -304,5 +304,7 @@ cudaError_t launch_postpass(int64_t M, int b, const float* X, int64_t ldx, const
   return launch_pdl(postpass_kernel<64>, dim3(grid(pp_rows<64>())), dim3(256), 0, st, M, b, X, ldx, W, ldw, Xh,
                     ldxh, WtXtt, ldwtx);
 }
+
+SBR_OP16_SETTER(chain)
 
 }  // namespace sbr

@@ -171,7 +171,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     }
   } else if (warp == 1) {
     if (lane == 0) {  // ---------------- MMA issuer
-      constexpr uint32_t idesc = idesc_make(G_BM, G_BN, TF ? 2 : 0, 0, 0);
+      const uint32_t idesc = idesc_make(G_BM, G_BN, TF ? 2 : 0, 0, 0) | (TF ? 0u : op16_fmt());
       int st = 0; uint32_t ph = 0;
       int ab = 0; uint32_t aph = 0;
       const uint32_t s0 = smem_u32(smem);
@@ -300,7 +300,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
             if (col <= row) {
               const float nv = old[c] - v[c];
               __stcs(cp + c * ldc, nv);
-              sp[c * ldsh] = __float2half_rn(col == row ? 0.5f * nv : nv);
+              sp[c * ldsh] = cvt16(col == row ? 0.5f * nv : nv);
             }
           }
         } else {
@@ -310,7 +310,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
           __half* Zh = (__half*)Zout;
           __align__(16) __half z[32];
 #pragma unroll
-          for (int c = 0; c < 32; ++c) z[c] = __float2half_rn(fmaf(-0.5f, v[c], xv[c]));
+          for (int c = 0; c < 32; ++c) z[c] = cvt16(fmaf(-0.5f, v[c], xv[c]));
           __half* zp = Zh + row * ldz + col0;
           if (col0 + 32 <= Ncols) {
 #pragma unroll
@@ -405,5 +405,7 @@ cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) { return l
 cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, true>(p, st); }
 cudaError_t launch_gemm_split_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<2, true>(p, st); }
 cudaError_t launch_gemm_sub_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<3, true>(p, st); }
+
+SBR_OP16_SETTER(gemm)
 
 }  // namespace sbr

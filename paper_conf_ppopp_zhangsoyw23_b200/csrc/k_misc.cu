@@ -373,7 +373,7 @@ __global__ void shadow_init_kernel(int64_t n, int64_t j0, float* A, int64_t lda,
       }
       if (i == g) v *= 0.5f;
     }
-    Sh[i + j * ldsh] = __float2half_rn(v);
+    Sh[i + j * ldsh] = cvt16(v);
   }
 }
 
@@ -411,7 +411,7 @@ __global__ void __launch_bounds__(256) shadow_init_vec_kernel(int64_t n, int64_t
         for (int u = 0; u < 4; ++u)
           if (i + u == g) e[u] *= 0.5f;
       }
-      __half2 h01 = __floats2half2_rn(v.x, v.y), h23 = __floats2half2_rn(v.z, v.w);
+      __half2 h01 = __halves2half2(cvt16(v.x), cvt16(v.y)), h23 = __halves2half2(cvt16(v.z), cvt16(v.w));
       uint2 pk;
       pk.x = *reinterpret_cast<uint32_t*>(&h01);
       pk.y = *reinterpret_cast<uint32_t*>(&h23);
@@ -427,7 +427,7 @@ __global__ void __launch_bounds__(256) shadow_init_vec_kernel(int64_t n, int64_t
         }
         if (i == g) v *= 0.5f;
       }
-      sc[i] = __float2half_rn(v);
+      sc[i] = cvt16(v);
     }
   }
 }
@@ -451,7 +451,7 @@ cudaError_t shadow_init(int64_t n, float* A, int64_t lda, __half* Sh, int64_t ld
 __global__ void to_half_cm_kernel(int64_t rows, int cols, const float* src, int64_t lds, __half* dst, int64_t ldd) {
   const int c = blockIdx.y;
   for (int64_t r = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; r < rows; r += (int64_t)gridDim.x * blockDim.x)
-    dst[r + c * ldd] = __float2half_rn(c < cols ? src[r + c * lds] : 0.f);
+    dst[r + c * ldd] = cvt16(c < cols ? src[r + c * lds] : 0.f);
 }
 
 // dst[r + c*ldd] = fp16(src[r + c*lds]) for c < cols, 0 for cols <= c < cols_pad
@@ -475,7 +475,7 @@ __global__ void f32cm_to_f16rm_kernel2(int64_t rows, int cols, const float* src,
 #pragma unroll
     for (int i = 0; i < 8; ++i) {
       const int c = g * 8 + i;
-      v[i] = __float2half_rn(c < cols ? src[r + (int64_t)c * lds] : 0.f);
+      v[i] = cvt16(c < cols ? src[r + (int64_t)c * lds] : 0.f);
     }
     if (g * 8 + 8 <= cols && ((r * ldd + g * 8) & 7) == 0) {
       *reinterpret_cast<uint4*>(dst + r * ldd + g * 8) = *reinterpret_cast<const uint4*>(v);
@@ -503,8 +503,8 @@ __global__ void build_lazy_b_kernel(int k, int b, const __half* Yh, int64_t ldyh
   for (int j = blockIdx.x * blockDim.x + threadIdx.x; j < kp + k; j += gridDim.x * blockDim.x) {
     __half v;
     if (j < k) v = Yh[(c + n) * ldyh + j];
-    else if (j < kp) v = __float2half_rn(0.f);
-    else v = __float2half_rn(P[(j - kp) + (int64_t)n * k]);
+    else if (j < kp) v = cvt16(0.f);
+    else v = cvt16(P[(j - kp) + (int64_t)n * k]);
     Bl[n * ldbl + j] = v;
   }
 }
@@ -515,5 +515,7 @@ cudaError_t build_lazy_b(int k, int b, const __half* Yh, int64_t ldyh, int64_t c
   build_lazy_b_kernel<<<dim3((kp + k + 255) / 256, b), 256, 0, st>>>(k, b, Yh, ldyh, c, P, Bl, ldbl);
   return cudaGetLastError();
 }
+
+SBR_OP16_SETTER(misc)
 
 }  // namespace sbr

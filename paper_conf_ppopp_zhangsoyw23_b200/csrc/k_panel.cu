@@ -432,22 +432,22 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
     for (int64_t i = threadIdx.x; i < M; i += blockDim.x) {
       if (i < row0) {
         for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
-        if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
-        if (a.Wh) for (int c = 0; c < b; ++c) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
-        if (a.Wrh) for (int c = 0; c < b; ++c) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
+        if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = cvt16(0.f);
+        if (a.Wh) for (int c = 0; c < b; ++c) a.Wh[i + c * a.ldwh] = cvt16(0.f);
+        if (a.Wrh) for (int c = 0; c < b; ++c) a.Wrh[i * a.ldwrh + c] = cvt16(0.f);
         continue;
       }
       const int64_t il = i - row0;
       for (int c = 0; c < b; ++c) {
         const float y = Vs[il + c * RSN];
         a.Y[i + c * a.ldy] = y;
-        if (a.Yh) a.Yh[i * a.ldyh + c] = __float2half_rn(y);
+        if (a.Yh) a.Yh[i * a.ldyh + c] = cvt16(y);
         a.P[il + c * a.ldp] = (il > c) ? y : (il < b ? Rs[il + c * b] : 0.f);
         float w = 0.f;
         for (int k = 0; k <= c; ++k) w = fmaf(Vs[il + k * RSN], T[k + c * LDU], w);
         a.W[i + c * a.ldw] = w;
-        if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(w);
-        if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(w);
+        if (a.Wh) a.Wh[i + c * a.ldwh] = cvt16(w);
+        if (a.Wrh) a.Wrh[i * a.ldwrh + c] = cvt16(w);
       }
     }
     return;
@@ -584,8 +584,8 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
     for (int c = 0; c < B; ++c)
       if (c < b) {
         a.W[gr + c * a.ldw] = v_[c];
-        if (a.Wh) a.Wh[gr + c * a.ldwh] = __float2half_rn(v_[c]);
-        if (a.Wrh) a.Wrh[gr * a.ldwrh + c] = __float2half_rn(v_[c]);
+        if (a.Wh) a.Wh[gr + c * a.ldwh] = cvt16(v_[c]);
+        if (a.Wrh) a.Wrh[gr * a.ldwrh + c] = cvt16(v_[c]);
       }
     // y = L_1 row (il < b)  or  y U = q
 #pragma unroll
@@ -608,7 +608,7 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
       if (c < b) {
         a.Y[gr + c * a.ldy] = v_[c];
         a.P[il + (int64_t)c * a.ldp] = (il > c) ? v_[c] : (Ss[il] * rroot[il + c * b]);   // il < b here
-        if (a.Yh) a.Yh[gr * a.ldyh + c] = __float2half_rn(v_[c]);
+        if (a.Yh) a.Yh[gr * a.ldyh + c] = cvt16(v_[c]);
       }
     }
   }
@@ -617,9 +617,9 @@ __global__ void __launch_bounds__(P_NW * 32, 1) panel_tsqr_kernel(PanelArgs a) {
   const int64_t nth = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = tid; i < row0; i += nth) {
     for (int c = 0; c < b; ++c) { a.Y[i + c * a.ldy] = 0.f; a.W[i + c * a.ldw] = 0.f; }
-    if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = __float2half_rn(0.f);
-    if (a.Wh) for (int c = 0; c < b; ++c) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
-    if (a.Wrh) for (int c = 0; c < b; ++c) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
+    if (a.Yh) for (int c = 0; c < b; ++c) a.Yh[i * a.ldyh + c] = cvt16(0.f);
+    if (a.Wh) for (int c = 0; c < b; ++c) a.Wh[i + c * a.ldwh] = cvt16(0.f);
+    if (a.Wrh) for (int c = 0; c < b; ++c) a.Wrh[i * a.ldwrh + c] = cvt16(0.f);
   }
   PTRACE(9);
 }
@@ -708,5 +708,7 @@ int panel_max_ctas(int b) {
   const int per = func_blocks_per_sm(k, P_NW * 32, smem);
   return std::max(1, per) * nsm;
 }
+
+SBR_OP16_SETTER(panel)
 
 }  // namespace sbr

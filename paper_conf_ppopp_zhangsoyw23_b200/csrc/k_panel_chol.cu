@@ -570,8 +570,8 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       for (int c = 0; c < B; ++c) {
         a.Y[i + c * a.ldy] = 0.f;
         a.W[i + c * a.ldw] = 0.f;
-        if (a.Wh) a.Wh[i + c * a.ldwh] = __float2half_rn(0.f);
-        if (a.Wrh) a.Wrh[i * a.ldwrh + c] = __float2half_rn(0.f);
+        if (a.Wh) a.Wh[i + c * a.ldwh] = cvt16(0.f);
+        if (a.Wrh) a.Wrh[i * a.ldwrh + c] = cvt16(0.f);
       }
       if (a.Yh) {   // 16-byte row stores
         const uint4 z = make_uint4(0u, 0u, 0u, 0u);
@@ -701,10 +701,10 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
 #pragma unroll
         for (int k = 0; k <= c; ++k) w = fmaf(v[k], Tf[k * B + c], w);
         a.W[gr + (int64_t)c * a.ldw] = w;
-        if (a.Wh) a.Wh[gr + (int64_t)c * a.ldwh] = __float2half_rn(w);
-        if (a.Wrh) a.Wrh[gr * a.ldwrh + c] = __float2half_rn(w);
+        if (a.Wh) a.Wh[gr + (int64_t)c * a.ldwh] = cvt16(w);
+        if (a.Wrh) a.Wrh[gr * a.ldwrh + c] = cvt16(w);
         a.Y[gr + (int64_t)c * a.ldy] = v[c];
-        yh[c] = __float2half_rn(v[c]);
+        yh[c] = cvt16(v[c]);
         if (il <= c) P[il + (int64_t)c * ldp] = __ldcg(fR + il * 64 + c);   // R (il < B here)
       }
       if (a.Yh) {
@@ -855,7 +855,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
       for (int s8 = 0; s8 < 8; ++s8) {
         const int64_t c = k0 + s8;
         a.W[gr + c * a.ldw] = wo[s8];
-        wh[s8] = __float2half_rn(wo[s8]);
+        wh[s8] = cvt16(wo[s8]);
         if (a.Wh) a.Wh[gr + c * a.ldwh] = wh[s8];
       }
       if (a.Wrh) *reinterpret_cast<uint4*>(a.Wrh + gr * a.ldwrh + k0) = *reinterpret_cast<const uint4*>(wh);
@@ -901,7 +901,7 @@ __global__ void __launch_bounds__(PC_THREADS, 1) panel_chol_kernel(PanelArgs a, 
         a.Y[gr + (int64_t)c * a.ldy] = yo[s8];
         // compact panel: Y tail strictly below, R_h = S R on and above the diagonal (il < B)
         a.P[il + (int64_t)c * a.ldp] = (il > c) ? yo[s8] : (float)((double)Ss[il] * Racc[il * B + c]);
-        yh[s8] = __float2half_rn(yo[s8]);
+        yh[s8] = cvt16(yo[s8]);
       }
       if (a.Yh) *reinterpret_cast<uint4*>(a.Yh + gr * a.ldyh + k0) = *reinterpret_cast<const uint4*>(yh);
     }
@@ -959,5 +959,7 @@ cudaError_t launch_panel_chol(PanelArgs& a, void* ws, unsigned launch, cudaStrea
     default: return cudaErrorNotSupported;
   }
 }
+
+SBR_OP16_SETTER(chol)
 
 }  // namespace sbr

@@ -221,8 +221,8 @@ __global__ void __launch_bounds__(256, 1)
   } else if (warp == 1) {
     // ------------------------------------------------ MMA issuer (one thread)
     if (lane == 0) {
-      constexpr uint32_t idesc_dir = idesc_make(128, BN, 0, /*a MN-major*/ 1, 0);
-      constexpr uint32_t idesc_tr = idesc_make(128, BN, 0, 0, 0);
+      const uint32_t idesc_dir = idesc_make(128, BN, 0, /*a MN-major*/ 1, 0) | op16_fmt();
+      const uint32_t idesc_tr = idesc_make(128, BN, 0, 0, 0) | op16_fmt();
       int st = 0; uint32_t ph = 0;
       int ws = 0; uint32_t wph = 0;
       int rb = 0; uint32_t rph = 0;
@@ -477,5 +477,7 @@ cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st) {
 int pass_bn(int b) { return b <= 16 ? 16 : b <= 32 ? 32 : 64; }
 
 int pass_dist_align(int b) { return 128 * pass_group_cols(b); }
+
+SBR_OP16_SETTER(pass)
 
 }  // namespace sbr

@@ -75,7 +75,7 @@ __global__ void __launch_bounds__(256, 1)
       if (++st == Cfg::NS) { st = 0; ph ^= 1; }
     }
   } else if (warp == 1 && lane == 0) {
-    constexpr uint32_t idesc = idesc_make(128, BN, 0, 0, 0);
+    const uint32_t idesc = idesc_make(128, BN, 0, 0, 0) | op16_fmt();
     int st = 0; uint32_t ph = 0;
     const uint32_t s0 = smem_u32(smem);
     for (int kc = kb; kc < ke; ++kc) {
@@ -125,7 +125,7 @@ __global__ void __launch_bounds__(256, 1)
         for (int c = 0; c < 32; ++c) {
           const int n = c0 + c;
           const float d = o[n] - v[c];
-          hv[c] = __float2half_rn(d);
+          hv[c] = cvt16(d);
           if (n < b) {
             Dout[r + (int64_t)n * ldd] = d;
             if (Hcm) Hcm[r + (int64_t)n * ldhc] = hv[c];
@@ -254,7 +254,7 @@ __global__ void __launch_bounds__(256, 1)
     }
   } else if (warp == 1 && lane == 0) {
     // A^T is MN-major: 64-wide K1 atoms 8 KB apart (LBO), 8-row K groups 1 KB apart (SBO)
-    constexpr uint32_t idesc = idesc_make(128, BN, 0, 1, 0);
+    const uint32_t idesc = idesc_make(128, BN, 0, 1, 0) | op16_fmt();
     int st = 0; uint32_t ph = 0;
     const uint32_t s0 = smem_u32(smem);
     for (int ks = 0; ks < nks; ++ks) {
@@ -331,5 +331,7 @@ cudaError_t launch_skinny_tn(const SkinnyTN& p, cudaStream_t st) {
   if (bn == 32) return launch_tn_t<32>(p, st);
   return launch_tn_t<64>(p, st);
 }
+
+SBR_OP16_SETTER(skinny)
 
 }  // namespace sbr

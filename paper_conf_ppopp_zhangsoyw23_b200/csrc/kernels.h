@@ -316,4 +316,16 @@ cudaError_t band_to_tridiag(int64_t n, int b, const float* AB, int64_t ldab, voi
 size_t tridiag_eig_ws_bytes(int64_t n);
 cudaError_t tridiag_eigenvalues(int64_t n, const double* d, const double* e, void* ws, double* lam, cudaStream_t st);
 
+// 16-bit operand format (fp16 / bf16) of each translation unit's conversions and kind::f16
+// descriptors (common.cuh g_op16_bf16); set_op16_all (sbr_api.cu) calls them all in stream order.
+cudaError_t set_op16_chain(int bf16, cudaStream_t st);
+cudaError_t set_op16_gemm(int bf16, cudaStream_t st);
+cudaError_t set_op16_misc(int bf16, cudaStream_t st);
+cudaError_t set_op16_panel(int bf16, cudaStream_t st);
+cudaError_t set_op16_chol(int bf16, cudaStream_t st);
+cudaError_t set_op16_skinny(int bf16, cudaStream_t st);
+cudaError_t set_op16_pass(int bf16, cudaStream_t st);
+cudaError_t set_op16_api(int bf16, cudaStream_t st);
+cudaError_t set_op16_all(int bf16, cudaStream_t st);
+
 }  // namespace sbr

@@ -21,6 +21,7 @@
 
 #include "../../include/sbr.h"
 #include "common.cuh"
+#include "common.cuh"
 #include "kernels.h"
 #include "comm.h"
 #include "nccl_rt.h"
@@ -367,7 +368,7 @@ int ensure_ws(sbr_ctx* h, int64_t n, int b, int nb, int mode, size_t* bytes_out,
 int validate(sbr_ctx* h, int mode, int64_t n, int b, int nb, const float* A, int64_t lda, const float* AB,
              int64_t ldab, const float* W, int64_t ldw) {
   if (!h) return -1;
-  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32) return -2;
+  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32 && mode != SBR_BF16_FP32ACC) return -2;
   if (n < 1) return -3;
   if (b < 1 || b > 64) return -4;
   if (nb < b || nb % b != 0 || nb > 4096) return -5;
@@ -438,7 +439,9 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
   // the TMA-fed tensor-core kernels need 16-byte aligned tile origins (OA origin r0 = c0 + b):
   // FP16 operands need b, nb multiples of 8, fp32 (3xTF32) multiples of 4; other (b, nb) run on
   // the fp32 SIMT kernels (more accurate than either mode's operands)
-  const bool tc16 = (mode == SBR_FP16_FP32ACC) && b % 8 == 0 && nb % 8 == 0;  // tcgen05 kind::f16 path
+  // tcgen05 kind::f16 path; SBR_BF16_FP32ACC is the same path with bfloat16 operands (f4 ablation)
+  const bool tc16 = (mode == SBR_FP16_FP32ACC || mode == SBR_BF16_FP32ACC) && b % 8 == 0 && nb % 8 == 0;
+  if (tc16) SBR_CK(set_op16_all(mode == SBR_BF16_FP32ACC, st), "operand format");
   // 3xTF32 on tcgen05 kind::tf32 (pass + Z + SYR2K); the SIMT fp32 kernels remain for A that
   // TMA cannot address (lda % 4 != 0) and for the SBR_TF32_TC=0 ablation
   const bool tc32 = mode == SBR_3XTF32 && h->tf32_tc && lda % 4 == 0 && ((uintptr_t)A & 15) == 0 && b % 4 == 0 &&
@@ -490,7 +493,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
       SBR_CK(cudaMemsetAsync(h->GH, 0, sizeof(float) * 2 * nb * nb, st), "zero G/H");
     }
     // fused FP16 chain (k_chain_fused.cu): one cooperative launch per panel + the pass
-    const bool fused = tc16 && h->fused && panel_mode_default(h) && nb <= 1024 && chain_fused_supported(b, M, h->nsm);
+    const bool fused = tc16 && mode == SBR_FP16_FP32ACC && h->fused && panel_mode_default(h) && nb <= 1024 && chain_fused_supported(b, M, h->nsm);
     // ---- a4 for panel t on every rank: W_t from the owner (dist), the pass over this rank's
     //      tiles (the 128-aligned grid of its column blocks when distributed), X_t summed
     auto pass_t = [&](int64_t tb) -> int {
@@ -1388,7 +1391,7 @@ int sbr_band_eigenvalues(sbr_handle_t h, int64_t n, int b, const float* AB, int6
 
 int sbr_eigenvalues(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A, int64_t lda, double* lam) {
   if (!h) return -1;
-  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32) return -2;
+  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32 && mode != SBR_BF16_FP32ACC) return -2;
   if (n < 1) return -3;
   if (b < 1 || b > 64) return -4;
   if (!lam) return -8;
@@ -1439,7 +1442,7 @@ int sbr_workspace_query(sbr_handle_t h, int64_t n, int b, int nb, int mode, size
   if (n < 1) return -2;
   if (b < 1 || b > 64) return -3;
   if (nb < b || nb % b != 0 || nb > 4096) return -4;
-  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32) return -5;
+  if (mode != SBR_FP16_FP32ACC && mode != SBR_3XTF32 && mode != SBR_BF16_FP32ACC) return -5;
   if (n <= b + 1) {
     *bytes = 0;
     return SBR_OK;
@@ -1573,7 +1576,7 @@ int sbr_reduce_dist(sbr_handle_t h, int mode, int64_t n, int b, int nb, float* A
     // SYR2K's tiles (configs 4/5: nb = 1024 / 2048)
     // FP16: the pass's 128-row tile groups (pass_dist_align); 3xTF32: 128-column tiles, b % 4 == 0 and
     // a 16-byte aligned A; both: the SYR2K's 256-column tiles
-    const bool ok16 = mode == SBR_FP16_FP32ACC && b % 8 == 0 && nb % pass_dist_align(b) == 0 && nb % 256 == 0;
+    const bool ok16 = (mode == SBR_FP16_FP32ACC || mode == SBR_BF16_FP32ACC) && b % 8 == 0 && nb % pass_dist_align(b) == 0 && nb % 256 == 0;
     const bool ok32 = mode == SBR_3XTF32 && h->tf32_tc && b % 4 == 0 && nb % 256 == 0 && lda % 4 == 0 &&
                       ((uintptr_t)A & 15) == 0;
     if (!ok16 && !ok32) {
@@ -1671,7 +1674,7 @@ __global__ void f32cm_to_f16rm_kernel(int64_t rows, int cols, const float* src, 
        e += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = e / cols;
     const int c = (int)(e % cols);
-    dst[r * ldd + c] = __float2half_rn(src[r + c * lds]);
+    dst[r * ldd + c] = cvt16(src[r + c * lds]);
   }
 }
 
@@ -1681,7 +1684,7 @@ __global__ void f16_to_f32_kernel(int64_t rows, int cols, const __half* src, int
        e += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = e % rows;
     const int c = (int)(e / rows);
-    dst[r + c * ldd] = __half2float(rowmajor ? src[r * lds + c] : src[r + c * lds]);
+    dst[r + c * ldd] = from16(rowmajor ? src[r * lds + c] : src[r + c * lds]);
   }
 }
 
@@ -2041,3 +2044,15 @@ extern "C" int sbr_test_pass_tiles(int64_t M, int b, int64_t t0, int64_t t1, int
   pass_tiles(M, b, t0, t1, IJ);
   return SBR_OK;
 }
+
+namespace sbr {
+SBR_OP16_SETTER(api)
+cudaError_t set_op16_all(int bf16, cudaStream_t st) {
+  for (auto f : {set_op16_chain, set_op16_gemm, set_op16_misc, set_op16_panel, set_op16_chol, set_op16_skinny,
+                 set_op16_pass, set_op16_api}) {
+    const cudaError_t e = f(bf16, st);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaSuccess;
+}
+}  // namespace sbr
