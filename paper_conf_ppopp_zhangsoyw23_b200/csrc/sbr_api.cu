@@ -781,7 +781,12 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
                "W merge");
         h->launches += 2;
       }
-      if (tc32) {  // ---- a4 (3xTF32 on tcgen05): OA frozen = A + strip copy, 32 W columns per launch
+      if (tc32 && knob(KNOB_TF32_SIMT_PASS) && !dist) {   // test knob: the SIMT fp32 pass inside the
+        // 3xTF32 reduction (attributes the mode's error between the pass and the other kernels)
+        Scope sc(h, SBR_K_PASS, 4.0 * M * M / 2 + 8.0 * M * b, 2.0 * M * M * b);
+        SBR_CK(sym_pass(M, b, OA, lda, h->Strip, ldn, sw, Wb + tb * ldwb, ldwb, h->Xb + tb * ldn, ldn, st), "pass");
+        h->launches += 1;
+      } else if (tc32) {  // ---- a4 (3xTF32 on tcgen05): OA frozen = A + strip copy, 32 W columns per launch
         Scope sc(h, SBR_K_PASS, (4.0 * M * M / 2 + 12.0 * M * b) / P, 3 * 2.0 * M * M * b / P);
         // distributed: the padding rows between X_t's columns are zeroed too (the all-reduce spans them)
         SBR_CK(zero_matrix(dist ? ldn : M, b, h->Xb + tb * ldn, ldn, st), "zero X_t");
