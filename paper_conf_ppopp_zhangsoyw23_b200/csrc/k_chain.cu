@@ -31,7 +31,7 @@ constexpr int KXB_RC = 64;   // r-chunk staged in shared memory per iteration
 // halves each warp's dependent chain and doubles the resident warps), 8 if that launch fails.
 // NG = 32-column groups of b (1: b <= 32, 2: b <= 64).
 template <int CL, int NG>
-__global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
+SBR_DEV void kxb_body(const KxbArgs& a, int qblk) {
   constexpr int NB = 32 * NG;
   constexpr int LA = KXB_RC * KXB_QT / 256;   // A elements staged per thread per chunk
   constexpr int LB = KXB_RC * NB / 256;       // B elements staged per thread per chunk
@@ -42,7 +42,7 @@ __global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int k = a.k, b = a.b;
   const bool lazy = a.mode == 0;
-  const int q0 = blockIdx.x * KXB_QT;
+  const int q0 = qblk * KXB_QT;
   const int rank = (int)cluster.block_rank();
   const int rper = (k + CL - 1) / CL;
   const int rb = rank * rper, re = min(k, rb + rper);
@@ -135,13 +135,13 @@ __global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
     }
   }
   if (lazy) {
-    if (blockIdx.x == 0 && rank == 0) {   // upper <- lower on the b x b diagonal block of the panel's columns
+    if (qblk == 0 && rank == 0) {   // upper <- lower on the b x b diagonal block of the panel's columns
       for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
         const int i = e % b, j = e / b;
         if (i < j) a.Adiag[i + (int64_t)j * a.lda] = a.Adiag[j + (int64_t)i * a.lda];
       }
     }
-  } else {   // G -> fp16, column-major (k contiguous): B operand of the merge GEMM
+  } else if (a.Gh) {   // G -> fp16, column-major (k contiguous): B operand of the merge GEMM
     const int64_t nth = (int64_t)gridDim.x * gridDim.y * blockDim.x;
     const int64_t tid = ((int64_t)blockIdx.y * gridDim.x + blockIdx.x) * blockDim.x + threadIdx.x;
     for (int64_t e = tid; e < (int64_t)k * b; e += nth) {
@@ -150,6 +150,11 @@ __global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
     }
   }
   cluster.sync();   // keep this CTA's partials alive until every reader is done
+}
+
+template <int CL, int NG>
+__global__ void __launch_bounds__(256) kxb_kernel(KxbArgs a) {
+  kxb_body<CL, NG>(a, blockIdx.x);
 }
 
 template <int CL, int NG>
@@ -203,9 +208,8 @@ template <int BB>  // BB >= b, multiple of 16; rows per CTA sized for 48 KB of s
 constexpr int pp_rows() { return BB <= 16 ? 128 : 64; }   // 8-16 loads per thread and array, ~3 CTAs per SM
 
 template <int BB>
-__global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
-    postpass_kernel(int64_t M, int b, const float* __restrict__ X, int64_t ldx, const float* __restrict__ W,
-                    int64_t ldw, __half* Xh, int64_t ldxh, float* WtXtt, int64_t ldwtx) {
+SBR_DEV void postpass_body(int64_t M, int b, const float* __restrict__ X, int64_t ldx, const float* __restrict__ W,
+                           int64_t ldw, __half* Xh, int64_t ldxh, float* WtXtt, int64_t ldwtx, int vblk) {
   constexpr int PP_ROWS = pp_rows<BB>();
   constexpr int BI = BB / 16;   // register block BI x BI per thread (16 x 16 thread grid)
   __shared__ float Xs[PP_ROWS][BB + 1];
@@ -214,7 +218,7 @@ __global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
   cg::cluster_group cluster = cg::this_cluster();
   pdl_trigger();
   pdl_wait();
-  const int64_t rbeg = (int64_t)blockIdx.x * PP_ROWS;
+  const int64_t rbeg = (int64_t)vblk * PP_ROWS;
   const int nr = (int)(M - rbeg < PP_ROWS ? (M - rbeg > 0 ? M - rbeg : 0) : PP_ROWS);
   constexpr int LU = PP_ROWS * BB / 256;   // elements per thread and array, all loads issued before any store
   float xv[LU], wv[LU];
@@ -286,6 +290,68 @@ __global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
     atomicAdd(WtXtt + i + (int64_t)j * ldwtx, s);
   }
   cluster.sync();
+}
+
+template <int BB>
+__global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
+    postpass_kernel(int64_t M, int b, const float* __restrict__ X, int64_t ldx, const float* __restrict__ W,
+                    int64_t ldw, __half* Xh, int64_t ldxh, float* WtXtt, int64_t ldwtx) {
+  postpass_body<BB>(M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt, ldwtx, blockIdx.x);
+}
+
+// The postpass of panel t and the MERGE kxb of panel t (W^T X_t = H - (W^T X) G; G -> fp16 is a
+// separate small launch before the merge GEMM) in ONE launch: CTAs [0, npp) are the postpass's,
+// the rest form the kxb's 8-CTA clusters.  Both read only what the pass and the merge left
+// behind and write disjoint parts of W^T X (diagonal block / column + row block).
+template <int BB, int NG>
+__global__ void __cluster_dims__(PP_CL, 1, 1) __launch_bounds__(256)
+    postpass_merge_kernel(int64_t M, int b, const float* __restrict__ X, int64_t ldx, const float* __restrict__ W,
+                          int64_t ldw, __half* Xh, int64_t ldxh, float* WtXtt, int64_t ldwtx, KxbArgs a, int npp) {
+  if ((int)blockIdx.x < npp)
+    postpass_body<BB>(M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt, ldwtx, blockIdx.x);
+  else
+    kxb_body<PP_CL, NG>(a, ((int)blockIdx.x - npp) / PP_CL);
+}
+
+cudaError_t launch_postpass_merge(int64_t M, int b, const float* X, int64_t ldx, const float* W, int64_t ldw,
+                                  __half* Xh, int64_t ldxh, float* WtXtt, int64_t ldwtx, const KxbArgs& a,
+                                  cudaStream_t st) {
+  if (M <= 0) return cudaSuccess;
+  KxbArgs m = a;
+  m.mode = 1;
+  m.Gh = nullptr;
+  if (b > 32) {   // both kernels' static shared memory together exceeds 48 KB: two launches
+    const cudaError_t e = launch_kxb(m, st);
+    if (e != cudaSuccess) return e;
+    return launch_postpass(M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt, ldwtx, st);
+  }
+  const int rows = b <= 16 ? pp_rows<16>() : pp_rows<32>();
+  const int64_t g = (M + rows - 1) / rows;
+  const int npp = (int)((g + PP_CL - 1) / PP_CL * PP_CL);
+  const int nk = a.k > 0 ? (a.k + KXB_QT - 1) / KXB_QT : 0;
+  const dim3 grid((unsigned)(npp + nk * PP_CL));
+  if (b <= 16)
+    return launch_pdl(postpass_merge_kernel<16, 1>, grid, dim3(256), 0, st, M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt,
+                      ldwtx, m, npp);
+  return launch_pdl(postpass_merge_kernel<32, 1>, grid, dim3(256), 0, st, M, b, X, ldx, W, ldw, Xh, ldxh, WtXtt,
+                    ldwtx, m, npp);
+}
+
+__global__ void __launch_bounds__(256) g_to_half_kernel(int k, int b, const float* __restrict__ G, int64_t ldg,
+                                                        __half* Gh, int64_t ldgh) {
+  pdl_trigger();
+  pdl_wait();
+  const int e = blockIdx.x * blockDim.x + threadIdx.x;
+  if (e < k * b) {
+    const int r = e % k, p = e / k;
+    Gh[r + (int64_t)p * ldgh] = cvt16(__ldcg(G + r + (int64_t)p * ldg));
+  }
+}
+
+cudaError_t launch_g_to_half(int k, int b, const float* G, int64_t ldg, __half* Gh, int64_t ldgh, cudaStream_t st) {
+  if (k <= 0 || b <= 0) return cudaSuccess;
+  return launch_pdl(g_to_half_kernel, dim3((unsigned)((k * b + 255) / 256)), dim3(256), 0, st, k, b, G, ldg, Gh,
+                    ldgh);
 }
 
 cudaError_t launch_postpass(int64_t M, int b, const float* X, int64_t ldx, const float* W, int64_t ldw, __half* Xh,

@@ -270,6 +270,13 @@ cudaError_t launch_kxb(const KxbArgs& a, cudaStream_t st);
 // after the pass: Xh[r*ldxh + p] = fp16(X[r + p*ldx]) and WtXtt[i + j*ldw] += sum_r W[r,i] X[r,j]
 cudaError_t launch_postpass(int64_t M, int b, const float* X, int64_t ldx, const float* W, int64_t ldw, __half* Xh,
                             int64_t ldxh, float* WtXtt, int64_t ldwtx, cudaStream_t st);
+// the postpass and the MERGE kxb's W^T X_t column block (a.Gh unused) as ONE launch of 8-CTA
+// clusters (independent work, one dependent step fewer on the per-panel chain); b > 32: two launches
+cudaError_t launch_postpass_merge(int64_t M, int b, const float* X, int64_t ldx, const float* W, int64_t ldw,
+                                  __half* Xh, int64_t ldxh, float* WtXtt, int64_t ldwtx, const KxbArgs& a,
+                                  cudaStream_t st);
+// Gh[r + p*ldgh] = fp16(G[r + p*ldg]), r < k, p < b (PDL; the merge GEMM's B operand)
+cudaError_t launch_g_to_half(int k, int b, const float* G, int64_t ldg, __half* Gh, int64_t ldgh, cudaStream_t st);
 
 // The fused per-panel chain of the FP16 mode (k_chain_fused.cu): ONE cooperative launch per
 // panel t does the previous pass's tail (Xh, W^T X diagonal block), the lazy update, the panel

@@ -723,18 +723,7 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           q.ldd = nb;
           q.num_sms = h->nsm;
           SBR_CK(launch_skinny_tn(q, st), "Y^T W0, X^T W0");
-          KxbArgs ka{};
-          ka.mode = 1;
-          ka.k = k;
-          ka.b = b;
-          ka.WtX = h->WtX;
-          ka.ldwx = nb;
-          ka.G = Gt;
-          ka.H = Ht;
-          ka.ldg = nb;
-          ka.Gh = h->Gh;
-          ka.ldgh = h->ldk;
-          SBR_CK(launch_kxb(ka, st), "W^T X_t, G -> fp16");
+          SBR_CK(launch_g_to_half(k, b, Gt, nb, h->Gh, h->ldk, st), "G -> fp16");   // merge GEMM's B operand
           SkinnyNN mq{};
           mq.A0 = h->Wrh;
           mq.A1 = nullptr;
@@ -763,11 +752,28 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
         }
         // ---- a4: pass X_t = OA W_t on tcgen05 (fp16 shadow of the frozen OA); X_t zeroed at block start
         if (int prc = pass_t(tb)) return prc;
-        if (leadJ) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block)
+        if (leadJ) {  // X_t -> fp16 row-major (operand of later lazy updates); W_t^T X_t (b x b diagonal block);
+                      // t >= 1: in the same launch W_{<t}^T X_t = H - (W^T X) G (the merge's kxb, reading R2),
+                      // which nothing needs before the next lazy update
           Scope sc(h, SBR_K_WMERGE, 4.0 * M * b * 2 + 2.0 * M * b, 2.0 * M * b * b);
-          SBR_CK(launch_postpass(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb,
-                                 st),
-                 "postpass");
+          if (t >= 1) {
+            KxbArgs ka{};
+            ka.mode = 1;
+            ka.k = k;
+            ka.b = b;
+            ka.WtX = h->WtX;
+            ka.ldwx = nb;
+            ka.G = Gt;
+            ka.H = Ht;
+            ka.ldg = nb;
+            SBR_CK(launch_postpass_merge(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk,
+                                         h->WtX + tb + tb * nb, nb, ka, st),
+                   "postpass + merge kxb");
+          } else {
+            SBR_CK(launch_postpass(M, b, h->Xb + tb * M, M, Wt, ldwb, h->Xh + tb, h->ldk, h->WtX + tb + tb * nb, nb,
+                                   st),
+                   "postpass");
+          }
           h->launches += 1;
         }
         continue;
