@@ -83,7 +83,7 @@ int func_blocks_per_sm(const void* fn, int threads, size_t smem);
 int current_device_sms();
 
 // test-only experiment knobs (sbr_testing.h sbr_test_set_knob); 0 unless a test set them
-enum Knob { KNOB_PASS_EXPER = 0, KNOB_TF32_SIMT_PASS = 1, KNOB_COUNT = 8 };
+enum Knob { KNOB_PASS_EXPER = 0, KNOB_TF32_SIMT_PASS = 1, KNOB_SYR2K_BAND = 2, KNOB_COUNT = 8 };
 int knob(Knob k);
 
 template <typename... KArgs, typename... Args>

@@ -52,14 +52,14 @@ template <bool TF> struct GCfg {
 // (H x 128 rows of [Y | Z], which stay L2-resident), so B is read from DRAM once per band
 // instead of once per tile row (the operands of a large block, 2 x M x 2nb, exceed L2).
 template <int MODE, int BN>
-SBR_DEV void gemm_tile(int t, int ntn, int ntm, int& I, int& Jc) {
+SBR_DEV void gemm_tile(int t, int ntn, int ntm, int& I, int& Jc, int H) {
   if (MODE != 0) {
     I = t / ntn;
     Jc = t % ntn;
     return;
   }
   constexpr int r = BN / G_BM;                       // 1 or 2
-  constexpr int H = BN == 256 ? 64 : 32;             // band height in tile rows (A band <= ~64 MB)
+  // H: band height in tile rows (A band <= ~64 MB at the default 64 / 32)
   for (int I0 = 0; I0 < ntm; I0 += H) {
     const int I1 = min(I0 + H, ntm), Hs = I1 - I0;
     const int F = I0 / r + 1;                        // columns with every band row valid
@@ -119,7 +119,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
                    const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
                    const GemmSegs segs, int arow0, int brow0, int64_t Mrows, int64_t Ncols, int ntn, int ntiles,
                    float* C, int64_t ldc, __half* __restrict__ shadow, int64_t ldsh, const float* __restrict__ X,
-                   int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off, const GemmOwn own) {
+                   int64_t ldx, void* __restrict__ Zout, int64_t ldz, int64_t zlo_off, const GemmOwn own, int bandH) {
   using Cfg = GCfg<TF>;
   constexpr int BK = TF ? 32 : 64;   // K elements per 128-byte row chunk
   constexpr int G_BN = Cfg::BN, G_NS = Cfg::NS, G_STAGE = Cfg::STAGE;
@@ -155,7 +155,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       int st = 0; uint32_t ph = 0;
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
         int I, Jc;
-        gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
+        gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
         if (!own.owned((int64_t)Jc * G_BN)) continue;
         for (int kc = 0; kc < nk; ++kc) {
           const int sg = kc / kpb, kin = (kc % kpb) * BK;
@@ -180,7 +180,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
         if (own.P > 1) {
           int I, Jc;
-          gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
+          gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
           if (!own.owned((int64_t)Jc * G_BN)) continue;
         }
         for (int kc = 0; kc < nk; ++kc) {
@@ -220,7 +220,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
-      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
+      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
       if (!own.owned((int64_t)Jc * G_BN)) continue;
       float acc[64];
 #pragma unroll
@@ -273,7 +273,7 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
       int I, Jc;
-      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc);
+      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
       if (!own.owned((int64_t)Jc * G_BN)) continue;
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();
@@ -396,7 +396,8 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   }
   return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
                     (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
-                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off, own);
+                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off, own,
+                    knob(KNOB_SYR2K_BAND) > 0 ? knob(KNOB_SYR2K_BAND) : (G_BN == 256 ? 64 : 32));
 }
 
 cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, false>(p, st); }
