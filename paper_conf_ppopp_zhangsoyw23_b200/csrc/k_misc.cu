@@ -288,6 +288,8 @@ cudaError_t extract_band(int64_t n, int b, float* A, int64_t lda, float* AB, int
 }
 
 __global__ void mirror_lower_block_kernel(int b, float* A, int64_t lda) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   for (int e = threadIdx.x; e < b * b; e += blockDim.x) {
     const int i = e % b, j = e / b;
     if (i < j) A[i + (int64_t)j * lda] = A[j + (int64_t)i * lda];
@@ -295,8 +297,7 @@ __global__ void mirror_lower_block_kernel(int b, float* A, int64_t lda) {
 }
 
 cudaError_t mirror_lower_block(int b, float* A, int64_t lda, cudaStream_t st) {
-  mirror_lower_block_kernel<<<1, 256, 0, st>>>(b, A, lda);
-  return cudaGetLastError();
+  return launch_pdl(mirror_lower_block_kernel, dim3(1), dim3(256), 0, st, b, A, lda);
 }
 
 // P[q, p] = X(c+p, q) - sum_r WtX[q, r] Y(c+p, r)   (k x b), i.e.
@@ -320,6 +321,8 @@ cudaError_t lazy_small_p(int k, int b, const float* Xc, int64_t ldx, const float
 
 // WtX[k+p, q] = WtX[q, k+p]  for q < k, p < b
 __global__ void mirror_wtx_kernel(int k, int b, float* WtX, int64_t ld) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   const int q = blockIdx.x * blockDim.x + threadIdx.x;
   const int p = blockIdx.y;
   if (q < k) WtX[(k + p) + (int64_t)q * ld] = WtX[q + (int64_t)(k + p) * ld];
@@ -327,8 +330,7 @@ __global__ void mirror_wtx_kernel(int k, int b, float* WtX, int64_t ld) {
 
 cudaError_t mirror_wtx(int k, int b, float* WtX, int64_t ld, cudaStream_t st) {
   if (k <= 0) return cudaSuccess;
-  mirror_wtx_kernel<<<dim3((k + 127) / 128, b), 128, 0, st>>>(k, b, WtX, ld);
-  return cudaGetLastError();
+  return launch_pdl(mirror_wtx_kernel, dim3((k + 127) / 128, b), dim3(128), 0, st, k, b, WtX, ld);
 }
 
 // Wo[:, c] = W[:, c] on the rows block J = c / nb acts on (r >= J nb + b), zero above
@@ -350,9 +352,23 @@ cudaError_t copy_block_w(int64_t n, int b, int nb, const float* W, int64_t ldw, 
   return cudaGetLastError();
 }
 
+// a kernel, not cudaMemset2DAsync: a memset node between two PDL launches would end the chain's
+// launch overlap (the per-panel steps of the 3xTF32 / SIMT paths zero small blocks every panel)
+__global__ void zero_matrix_kernel(int64_t rows, int64_t cols, float* A, int64_t lda) {
+  pdl_trigger();
+  pdl_wait();
+  const int64_t tot = rows * cols;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < tot; e += (int64_t)gridDim.x * blockDim.x)
+    A[e % rows + (e / rows) * lda] = 0.f;
+}
+
 cudaError_t zero_matrix(int64_t rows, int64_t cols, float* A, int64_t lda, cudaStream_t st) {
   if (rows <= 0 || cols <= 0) return cudaSuccess;
-  return cudaMemset2DAsync(A, lda * sizeof(float), 0, rows * sizeof(float), cols, st);
+  const int64_t tot = rows * cols;
+  if (tot > ((int64_t)1 << 22))   // block-start buffers (not on the per-panel chain): the copy engine
+    return cudaMemset2DAsync(A, lda * sizeof(float), 0, rows * sizeof(float), cols, st);
+  return launch_pdl(zero_matrix_kernel, dim3((unsigned)std::min<int64_t>((tot + 255) / 256, 148 * 16)), dim3(256), 0,
+                    st, rows, cols, A, lda);
 }
 
 // a0: fp16 shadow of the lower triangle of 2^k A: strict lower as is, HALF the diagonal, zero

@@ -495,6 +495,8 @@ cudaError_t set_identity(int64_t n, float* Q, int64_t ldq, cudaStream_t st) {
 
 __global__ void split_tf32_w_kernel(int64_t rows, int b, int bn, const float* __restrict__ W, int64_t ldw,
                                     float* __restrict__ dst, int64_t ldd) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   const int64_t total = rows * bn;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = i % rows, c = i / rows;
@@ -514,8 +516,7 @@ cudaError_t split_tf32_w(int64_t rows, int b, int bn, const float* W, int64_t ld
   if (rows <= 0) return cudaSuccess;
   const int64_t total = rows * bn;
   const int grid = (int)std::min<int64_t>((total + 255) / 256, 148 * 8);
-  split_tf32_w_kernel<<<grid, 256, 0, st>>>(rows, b, bn, W, ldw, dst, ldd);
-  return cudaGetLastError();
+  return launch_pdl(split_tf32_w_kernel, dim3(grid), dim3(256), 0, st, rows, b, bn, W, ldw, dst, ldd);
 }
 
 }  // namespace sbr

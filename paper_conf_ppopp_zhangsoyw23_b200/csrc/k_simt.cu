@@ -14,6 +14,8 @@ __global__ void __launch_bounds__(256) gemm_tn_kernel(int64_t rows, int64_t chun
                                                       const float* __restrict__ A, int64_t lda,
                                                       const float* __restrict__ B, int64_t ldb, float* C,
                                                       int64_t ldc) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   __shared__ float As[TN_KC][TN_T + 1];
   __shared__ float Bs[TN_KC][TN_T + 1];
   const int i0 = blockIdx.x * TN_T, j0 = blockIdx.y * TN_T;
@@ -58,6 +60,8 @@ __global__ void __launch_bounds__(256) skinny_tn32_kernel(int64_t rows, int64_t 
                                                           const float* __restrict__ A, int64_t lda,
                                                           const float* __restrict__ B, int64_t ldb, float* C,
                                                           int64_t ldc) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   constexpr int KC = 64, TI = 64, TJ = 32;
   __shared__ float As[TI][KC + 1];
   __shared__ float Bs[TJ][KC + 1];
@@ -127,8 +131,8 @@ cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, i
     int64_t chunk = std::max<int64_t>((rows + want - 1) / want, 128);
     chunk = (chunk + 63) / 64 * 64;
     const int gz = (int)((rows + chunk - 1) / chunk);
-    skinny_tn32_kernel<<<dim3(gx, 1, gz), 256, 0, st>>>(rows, chunk, m1, n2, alpha, A, lda, B, ldb, C, ldc);
-    return cudaGetLastError();
+    return launch_pdl(skinny_tn32_kernel, dim3(gx, 1, gz), dim3(256), 0, st, rows, chunk, m1, n2, alpha, A, lda, B, ldb,
+                      C, ldc);
   }
   const int gx = (m1 + TN_T - 1) / TN_T, gy = (n2 + TN_T - 1) / TN_T;
   int64_t want = std::max<int64_t>(1, 296 / (gx * gy));
@@ -136,8 +140,8 @@ cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, i
   chunk = std::max<int64_t>(chunk, 256);
   chunk = (chunk + TN_KC - 1) / TN_KC * TN_KC;
   const int gz = (int)((rows + chunk - 1) / chunk);
-  gemm_tn_kernel<<<dim3(gx, gy, gz), 256, 0, st>>>(rows, chunk, m1, n2, alpha, A, lda, B, ldb, C, ldc);
-  return cudaGetLastError();
+  return launch_pdl(gemm_tn_kernel, dim3(gx, gy, gz), dim3(256), 0, st, rows, chunk, m1, n2, alpha, A, lda, B, ldb, C,
+                    ldc);
 }
 
 // ---------------------------------------------------------------- gemm_nn
@@ -149,6 +153,8 @@ __global__ void __launch_bounds__(256) gemm_nn_kernel(int64_t M, int N, int K, f
                                                       const float* __restrict__ B, int64_t ldb, bool transB,
                                                       float beta, const float* C, int64_t ldc, float* D,
                                                       int64_t ldd) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   __shared__ float As[NN_KC][NN_T + 1];
   __shared__ float Bs[NN_KC][NN_T + 1];
   const int64_t i0 = (int64_t)blockIdx.x * NN_T;
@@ -210,6 +216,8 @@ __global__ void __launch_bounds__(256) skinny_upd_kernel(int64_t M, int N, int K
                                                          const float* __restrict__ A, int64_t lda,
                                                          const float* __restrict__ B, int64_t ldb, bool transB,
                                                          float* D, int64_t ldd) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   constexpr int RB = 128, KC = 32, NC = 32 * NG;
   __shared__ __align__(16) float As[KC][RB];
   __shared__ __align__(16) float Bs[KC][NC];
@@ -298,14 +306,14 @@ cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_
     const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
     ks = (K + kper - 1) / kper;
     if (N <= 32)
-      skinny_upd_kernel<1><<<dim3(gx, ks), 256, 0, st>>>(M, N, K, kper, alpha, A, lda, B, ldb, transB, D, ldd);
-    else
-      skinny_upd_kernel<2><<<dim3(gx, ks), 256, 0, st>>>(M, N, K, kper, alpha, A, lda, B, ldb, transB, D, ldd);
-    return cudaGetLastError();
+      return launch_pdl(skinny_upd_kernel<1>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
+                        transB, D, ldd);
+    return launch_pdl(skinny_upd_kernel<2>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
+                      transB, D, ldd);
   }
   dim3 grid((unsigned)((M + NN_T - 1) / NN_T), (N + NN_T - 1) / NN_T);
-  gemm_nn_kernel<<<grid, 256, 0, st>>>(M, N, K, alpha, A, lda, B, ldb, transB, beta, C, ldc, D, ldd);
-  return cudaGetLastError();
+  return launch_pdl(gemm_nn_kernel, grid, dim3(256), 0, st, M, N, K, alpha, A, lda, B, ldb, transB, beta, C, ldc, D,
+                    ldd);
 }
 
 // ---------------------------------------------------------------- sym_pass (SIMT v1)

@@ -16,6 +16,8 @@ __global__ void __launch_bounds__(256) small_gemm_kernel(int m, int n, int K, fl
                                                          int64_t lda, const float* __restrict__ B, int64_t ldb,
                                                          int transB, float beta, const float* __restrict__ C,
                                                          int64_t ldc, int transC, float* D, int64_t ldd) {
+  pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
+  pdl_wait();
   __shared__ float As[SG_KC][SG_T + 1];
   __shared__ float Bs[SG_KC][SG_T + 1];
   const int i0 = blockIdx.x * SG_T, j0 = blockIdx.y * SG_T;
@@ -68,9 +70,8 @@ cudaError_t small_gemm(int m, int n, int K, float alpha, const float* A, int64_t
   cudaError_t e = zero_matrix(m, n, D, ldd, st);
   if (e != cudaSuccess) return e;
   dim3 grid((m + SG_T - 1) / SG_T, (n + SG_T - 1) / SG_T, std::max(1, (K + SG_SPLIT - 1) / SG_SPLIT));
-  small_gemm_kernel<<<grid, 256, 0, st>>>(m, n, K, alpha, A, lda, B, ldb, transB ? 1 : 0, beta, C, ldc,
-                                          transC ? 1 : 0, D, ldd);
-  return cudaGetLastError();
+  return launch_pdl(small_gemm_kernel, grid, dim3(256), 0, st, m, n, K, alpha, A, lda, B, ldb, transB ? 1 : 0, beta, C,
+                    ldc, transC ? 1 : 0, D, ldd);
 }
 
 // D[b x b] += A[rows x b]^T B[rows x b]   (fp32, column-major; D zeroed here)
