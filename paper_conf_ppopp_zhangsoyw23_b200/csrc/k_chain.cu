@@ -126,7 +126,8 @@ SBR_DEV void kxb_body(const KxbArgs& a, int qblk) {
     if (q < k) {
       if (lazy) {
         const float d = __ldcg(a.X + (a.c + p) + (int64_t)q * a.ldx) - s;
-        a.Ph[(int64_t)p * a.ldph + q] = cvt16(d);
+        if (a.Ph) a.Ph[(int64_t)p * a.ldph + q] = cvt16(d);
+        if (a.P32) a.P32[q + (int64_t)p * a.ldp32] = d;
       } else {
         const float d = __ldcg(a.H + q + (int64_t)p * a.ldg) - s;
         WtX[q + (int64_t)(k + p) * ldwx] = d;

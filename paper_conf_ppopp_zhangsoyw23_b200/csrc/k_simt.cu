@@ -211,11 +211,15 @@ __global__ void __launch_bounds__(256) gemm_nn_kernel(int64_t M, int N, int K, f
 // is 128-row blocks x a K split sized to fill every SM twice; partial sums go to D with fp32
 // atomics (D = C in place, beta = 1).  Per thread 4 rows x NG*4 columns; A / B chunks of 32 K
 // staged through shared memory with a register prefetch of the next chunk.
+// A second segment (K1 > 0) appends A1 op(B1) along K: D += alpha (A op(B) + A1 op(B1)) in one
+// launch (the 3xTF32 lazy update X Y_c^T + Y P).
 template <int NG>   // NG = N / 32 rounded up (1 or 2)
 __global__ void __launch_bounds__(256) skinny_upd_kernel(int64_t M, int N, int K, int kper, float alpha,
                                                          const float* __restrict__ A, int64_t lda,
                                                          const float* __restrict__ B, int64_t ldb, bool transB,
-                                                         float* D, int64_t ldd) {
+                                                         float* D, int64_t ldd, int K0,
+                                                         const float* __restrict__ A1, int64_t lda1,
+                                                         const float* __restrict__ B1, int64_t ldb1, bool transB1) {
   pdl_trigger();   // 3xTF32 / SIMT chain: launched with PDL (launch_pdl), waits before any access
   pdl_wait();
   constexpr int RB = 128, KC = 32, NC = 32 * NG;
@@ -236,17 +240,21 @@ __global__ void __launch_bounds__(256) skinny_upd_kernel(int64_t M, int N, int K
       const int e = threadIdx.x + q * 256, ii = e & (RB - 1), kk = e >> 7;
       const int64_t i = i0 + ii;
       const int k = k0 + kk;
-      ra[q] = (i < M && k < ke) ? __ldg(A + i + (int64_t)k * lda) : 0.f;
+      ra[q] = (i < M && k < ke) ? __ldg(k < K0 ? A + i + (int64_t)k * lda : A1 + i + (int64_t)(k - K0) * lda1) : 0.f;
     }
 #pragma unroll
-    for (int q = 0; q < 4 * NG; ++q) {   // B: 32 k x NC columns
+    for (int q = 0; q < 4 * NG; ++q) {   // B: 32 k x NC columns (the layout of the chunk's first segment)
       const int e = threadIdx.x + q * 256;
+      const bool tb = (k0 < K0) ? transB : transB1;
       int kk, jj;
-      if (transB) { jj = e % NC; kk = e / NC; } else { kk = e % KC; jj = e / KC; }
+      if (tb) { jj = e % NC; kk = e / NC; } else { kk = e % KC; jj = e / KC; }
       const int k = k0 + kk;
-      rbv[q] = (k < ke && jj < N) ? __ldg(transB ? B + jj + (int64_t)k * ldb : B + k + (int64_t)jj * ldb) : 0.f;
+      const float* bp = k < K0 ? (transB ? B + jj + (int64_t)k * ldb : B + k + (int64_t)jj * ldb)
+                               : (transB1 ? B1 + jj + (int64_t)(k - K0) * ldb1 : B1 + (k - K0) + (int64_t)jj * ldb1);
+      rbv[q] = (k < ke && jj < N) ? __ldg(bp) : 0.f;
     }
   };
+  bool tbs = transB;   // B layout of the chunk whose loads are in rbv
   auto store = [&]() {
 #pragma unroll
     for (int q = 0; q < 16; ++q) {
@@ -256,13 +264,14 @@ __global__ void __launch_bounds__(256) skinny_upd_kernel(int64_t M, int N, int K
 #pragma unroll
     for (int q = 0; q < 4 * NG; ++q) {
       const int e = threadIdx.x + q * 256;
-      if (transB) Bs[e / NC][e % NC] = rbv[q];
+      if (tbs) Bs[e / NC][e % NC] = rbv[q];
       else Bs[e % KC][e / KC] = rbv[q];
     }
   };
   if (kb < ke) load(kb);
   for (int k0 = kb; k0 < ke; k0 += KC) {
     __syncthreads();
+    tbs = (k0 < K0) ? transB : transB1;
     store();
     __syncthreads();
     if (k0 + KC < ke) load(k0 + KC);   // next chunk's loads in flight during this chunk's FMAs
@@ -307,13 +316,30 @@ cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_
     ks = (K + kper - 1) / kper;
     if (N <= 32)
       return launch_pdl(skinny_upd_kernel<1>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
-                        transB, D, ldd);
+                        transB, D, ldd, K, (const float*)nullptr, (int64_t)0, (const float*)nullptr, (int64_t)0, false);
     return launch_pdl(skinny_upd_kernel<2>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
-                      transB, D, ldd);
+                      transB, D, ldd, K, (const float*)nullptr, (int64_t)0, (const float*)nullptr, (int64_t)0, false);
   }
   dim3 grid((unsigned)((M + NN_T - 1) / NN_T), (N + NN_T - 1) / NN_T);
   return launch_pdl(gemm_nn_kernel, grid, dim3(256), 0, st, M, N, K, alpha, A, lda, B, ldb, transB, beta, C, ldc, D,
                     ldd);
+}
+
+// D += alpha (A0 op(B0) + A1 op(B1)), N <= 64, K0 + K1 along K, D in place (fp32 atomics)
+cudaError_t skinny_upd2(int64_t M, int N, int K0, const float* A0, int64_t lda0, const float* B0, int64_t ldb0,
+                        bool transB0, int K1, const float* A1, int64_t lda1, const float* B1, int64_t ldb1,
+                        bool transB1, float alpha, float* D, int64_t ldd, cudaStream_t st) {
+  const int K = K0 + K1;
+  if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
+  const int gx = (int)((M + 127) / 128);
+  int ks = std::max(1, std::min((K + 63) / 64, (2 * 148 + gx - 1) / gx));
+  const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
+  ks = (K + kper - 1) / kper;
+  if (N <= 32)
+    return launch_pdl(skinny_upd_kernel<1>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A0, lda0, B0, ldb0,
+                      transB0, D, ldd, K0, A1, lda1, B1, ldb1, transB1);
+  return launch_pdl(skinny_upd_kernel<2>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A0, lda0, B0, ldb0,
+                    transB0, D, ldd, K0, A1, lda1, B1, ldb1, transB1);
 }
 
 // ---------------------------------------------------------------- sym_pass (SIMT v1)

@@ -64,6 +64,9 @@ cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, i
                     const float* B, int64_t ldb, float* C, int64_t ldc, cudaStream_t st);
 // D[M x N] = beta*C + alpha * A[M x K] op(B)  ; op(B) = B (K x N, ld) or B^T (B is N x K)
 // C and D may alias (in place).
+cudaError_t skinny_upd2(int64_t M, int N, int K0, const float* A0, int64_t lda0, const float* B0, int64_t ldb0,
+                        bool transB0, int K1, const float* A1, int64_t lda1, const float* B1, int64_t ldb1,
+                        bool transB1, float alpha, float* D, int64_t ldd, cudaStream_t st);
 cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_t lda,
                     const float* B, int64_t ldb, bool transB, float beta, const float* C, int64_t ldc,
                     float* D, int64_t ldd, cudaStream_t st);
@@ -261,7 +264,8 @@ struct KxbArgs {
   int k, b;
   float* WtX; int64_t ldwx;
   const float* Y; int64_t ldy; const float* X; int64_t ldx; int64_t c;   // LAZY
-  __half* Ph; int64_t ldph;
+  __half* Ph; int64_t ldph;      // fp16 P^T (FP16 chain) ...
+  float* P32 = nullptr; int64_t ldp32 = 0;   // ... and/or fp32 P[q + p*ldp32] (3xTF32 / SIMT chain)
   float* Adiag; int64_t lda;
   const float* G; const float* H; int64_t ldg;                           // MERGE
   __half* Gh; int64_t ldgh;

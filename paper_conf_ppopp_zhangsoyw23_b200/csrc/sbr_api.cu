@@ -638,13 +638,29 @@ int reduce_device(sbr_ctx* h, int mode, int64_t n, int b, int nb, float* A, int6
           h->launches += 2;
         } else {
           Scope sc(h, SBR_K_LAZY, 4.0 * rows * (2.0 * k + 2 * b), 4.0 * rows * k * b);
-          SBR_CK(small_gemm(k, b, k, -1.f, h->WtX, nb, h->Yb + c, ldn, true, 1.f, h->Xb + c, ldn, true, h->Pb, k, st), "lazy_p");
-          SBR_CK(mirror_lower_block(b, Ablk, lda, st), "mirror");
-          SBR_CK(gemm_nn(rows, b, k, -1.f, h->Xb + c, ldn, h->Yb + c, ldn, true, 1.f, Ablk, lda, Ablk, lda, st),
-                 "lazy X Yc^T");
-          SBR_CK(gemm_nn(rows, b, k, -1.f, h->Yb + c, ldn, h->Pb, k, false, 1.f, Ablk, lda, Ablk, lda, st),
-                 "lazy Y P");
-          h->launches += 4;
+          // P = X_c^T - (W^T X) Y_c^T (k x b, fp32) and the diagonal block's mirror: the kxb kernel of the
+          // FP16 chain with an fp32 output; then A_p -= X Y_c^T + Y P as ONE two-segment skinny update
+          KxbArgs ka{};
+          ka.mode = 0;
+          ka.k = k;
+          ka.b = b;
+          ka.WtX = h->WtX;
+          ka.ldwx = nb;
+          ka.Y = h->Yb;
+          ka.ldy = ldn;
+          ka.X = h->Xb;
+          ka.ldx = ldn;
+          ka.c = c;
+          ka.Ph = nullptr;
+          ka.P32 = h->Pb;
+          ka.ldp32 = k;
+          ka.Adiag = Ablk;
+          ka.lda = lda;
+          SBR_CK(launch_kxb(ka, st), "lazy P");
+          SBR_CK(skinny_upd2(rows, b, k, h->Xb + c, ldn, h->Yb + c, ldn, true, k, h->Yb + c, ldn, h->Pb, k, false, -1.f,
+                             Ablk, lda, st),
+                 "lazy X Y_c^T + Y P");
+          h->launches += 2;
         }
       }
       if (leadJ) {  // ---- a1/a2: TSQR + reconstruction
