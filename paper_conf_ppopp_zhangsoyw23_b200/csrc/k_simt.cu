@@ -126,10 +126,10 @@ cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, i
                     int64_t ldb, float* C, int64_t ldc, cudaStream_t st) {
   if (rows <= 0 || m1 <= 0 || n2 <= 0) return cudaSuccess;
   if (n2 <= 32) {
-    // ~4 CTAs per SM (126 registers, 25 KB smem: 2 fit per SM, the rest hides the tail): measured
+    // ~8 CTAs per SM (126 registers, 25 KB smem: 2 resident, the rest hides the tail): measured
     // 2 per SM left 18% of the warp slots active (ncu, config 3) with a half-empty second wave
     const int gx = (m1 + 63) / 64;
-    int64_t want = std::max<int64_t>(1, (4 * 148 + gx - 1) / gx);
+    int64_t want = std::max<int64_t>(1, (8 * 148 + gx - 1) / gx);
     int64_t chunk = std::max<int64_t>((rows + want - 1) / want, 64);
     chunk = (chunk + 63) / 64 * 64;
     const int gz = (int)((rows + chunk - 1) / chunk);
@@ -313,7 +313,7 @@ cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_
   if (M <= 0 || N <= 0) return cudaSuccess;
   if (N <= 64 && beta == 1.f && C == D && ldc == ldd && K > 0) {   // in-place skinny update
     const int gx = (int)((M + 127) / 128);
-    int ks = std::max(1, std::min((K + 63) / 64, (4 * 148 + gx - 1) / gx));   // ~4 CTAs per SM (64 registers)
+    int ks = std::max(1, std::min((K + 63) / 64, (8 * 148 + gx - 1) / gx));   // ~8 CTAs per SM (64 registers: 4 resident)
     const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
     ks = (K + kper - 1) / kper;
     if (N <= 32)
@@ -334,7 +334,7 @@ cudaError_t skinny_upd2(int64_t M, int N, int K0, const float* A0, int64_t lda0,
   const int K = K0 + K1;
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   const int gx = (int)((M + 127) / 128);
-  int ks = std::max(1, std::min((K + 63) / 64, (4 * 148 + gx - 1) / gx));   // ~4 CTAs per SM (64 registers)
+  int ks = std::max(1, std::min((K + 63) / 64, (8 * 148 + gx - 1) / gx));   // ~8 CTAs per SM (64 registers: 4 resident)
   const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
   ks = (K + kper - 1) / kper;
   if (N <= 32)
