@@ -313,7 +313,10 @@ cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_
   if (M <= 0 || N <= 0) return cudaSuccess;
   if (N <= 64 && beta == 1.f && C == D && ldc == ldd && K > 0) {   // in-place skinny update
     const int gx = (int)((M + 127) / 128);
-    int ks = std::max(1, std::min((K + 63) / 64, (8 * 148 + gx - 1) / gx));   // ~8 CTAs per SM (64 registers: 4 resident)
+    // N <= 32: ~8 CTAs per SM (64 registers: 4 resident; ncu at config 3 saw 25% of the warp slots at
+    // 2 per SM); N = 64 keeps 2 per SM (config 5: more K splits doubled the 128 x 64 atomic flushes)
+    const int per = N <= 32 ? 8 : 2;
+    int ks = std::max(1, std::min((K + 63) / 64, (per * 148 + gx - 1) / gx));
     const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
     ks = (K + kper - 1) / kper;
     if (N <= 32)
@@ -334,7 +337,8 @@ cudaError_t skinny_upd2(int64_t M, int N, int K0, const float* A0, int64_t lda0,
   const int K = K0 + K1;
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   const int gx = (int)((M + 127) / 128);
-  int ks = std::max(1, std::min((K + 63) / 64, (8 * 148 + gx - 1) / gx));   // ~8 CTAs per SM (64 registers: 4 resident)
+  const int per = N <= 32 ? 8 : 2;   // as gemm_nn's in-place branch
+  int ks = std::max(1, std::min((K + 63) / 64, (per * 148 + gx - 1) / gx));
   const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
   ks = (K + kper - 1) / kper;
   if (N <= 32)
