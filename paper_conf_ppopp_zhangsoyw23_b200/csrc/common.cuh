@@ -83,8 +83,18 @@ int func_blocks_per_sm(const void* fn, int threads, size_t smem);
 int current_device_sms();
 
 // test-only experiment knobs (sbr_testing.h sbr_test_set_knob); 0 unless a test set them
-enum Knob { KNOB_PASS_EXPER = 0, KNOB_TF32_SIMT_PASS = 1, KNOB_SYR2K_BAND = 2, KNOB_COUNT = 8 };
+enum Knob { KNOB_PASS_EXPER = 0, KNOB_TF32_SIMT_PASS = 1, KNOB_SYR2K_BAND = 2, KNOB_SYR2K_MC = 3, KNOB_COUNT = 8 };
 int knob(Knob k);
+
+// A plain launch of a kernel that also calls pdl_trigger / pdl_wait (no-ops then): used where an
+// early-launched dependent grid measured slower (config 5's b = 64 SIMT merge: 726 -> 868 ms on PDL,
+// its 64-wide gemm_tn and in-place update park resident CTAs beside their predecessors).
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_plain(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                                Args&&... args) {
+  kern<<<grid, block, smem, st>>>(std::forward<Args>(args)...);
+  return cudaGetLastError();
+}
 
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_pdl(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,

@@ -51,14 +51,14 @@ template <bool TF> struct GCfg {
 // in flight then share one or two B panels (rows Jc of [Z | Y]) and sweep the band's A panels
 // (H x 128 rows of [Y | Z], which stay L2-resident), so B is read from DRAM once per band
 // instead of once per tile row (the operands of a large block, 2 x M x 2nb, exceed L2).
-template <int MODE, int BN>
+template <int MODE, int BN, int BMU = G_BM>   // BMU: rows of one work unit (G_BM, or 2 G_BM for a CTA pair)
 SBR_DEV void gemm_tile(int t, int ntn, int ntm, int& I, int& Jc, int H) {
   if (MODE != 0) {
     I = t / ntn;
     Jc = t % ntn;
     return;
   }
-  constexpr int r = BN / G_BM;                       // 1 or 2
+  constexpr int r = BN / BMU;                        // 1 or 2
   // H: band height in tile rows (A band <= ~64 MB at the default 64 / 32)
   for (int I0 = 0; I0 < ntm; I0 += H) {
     const int I1 = min(I0 + H, ntm), Hs = I1 - I0;
@@ -113,7 +113,11 @@ struct GemmSegs {
   int amap[6], acol[6], bmap[6], bcol[6];
 };
 
-template <int MODE, bool TF>
+// MC = 2 (FP16 SYR2K): CTA pairs (clusters of 2) take work units of two 128-row tiles with the same
+// column tile Jc; each CTA loads its own A rows and HALF of the shared B tile, multicast into both
+// CTAs' shared memory, so B crosses L2 -> SM once per pair (the SYR2K's operand stream per tile was
+// 1.5 MB at K = 2 nb); each CTA's MMA commit frees the stage in both CTAs (empty count = 2).
+template <int MODE, bool TF, int MC = 1>
 __global__ void __launch_bounds__(G_THREADS, 1)
     gemm_tc_kernel(const __grid_constant__ CUtensorMap mapA0, const __grid_constant__ CUtensorMap mapA1,
                    const __grid_constant__ CUtensorMap mapB0, const __grid_constant__ CUtensorMap mapB1, int kpb,
@@ -134,28 +138,35 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   const int warp = warp_id(), lane = lane_id();
   pdl_trigger();
   if (threadIdx.x == 0) {
-    for (int i = 0; i < G_NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < G_NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], MC); }
     for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 32 * G_EPI_WARPS); }
     mbar_fence_init();
   }
+  const int crank = MC > 1 ? (int)cluster_ctarank() : 0;
+  // work units: one tile (MC = 1) or a pair of vertically adjacent tiles (MC = 2), unit u covers
+  // tile rows MC u .. MC u + MC - 1; this CTA takes row I = MC Iu + crank
+  const int u0 = MC > 1 ? (int)blockIdx.x / MC : (int)blockIdx.x;
+  const int ustride = MC > 1 ? (int)gridDim.x / MC : (int)gridDim.x;
   if (warp == 0 && lane == 0) {
     tma_prefetch(&mapA0); tma_prefetch(&mapB0); tma_prefetch(&mapA1); tma_prefetch(&mapB1);
   }
   if (warp == 2) tmem_alloc(tmem_slot, 512);
   tc_fence_before();
   __syncthreads();
+  if (MC > 1) cluster_sync_all();   // the peer's barriers are initialised before any multicast / commit
   tc_fence_after();
   const uint32_t tmem = *tmem_slot;
   pdl_wait();
   const int nk = segs.n * kpb;
-  const int ntm = (int)((Mrows + G_BM - 1) / G_BM);
+  const int ntm = (int)((Mrows + G_BM * MC - 1) / (G_BM * MC));   // unit rows
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
       int st = 0; uint32_t ph = 0;
-      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      for (int t = u0; t < ntiles; t += ustride) {
         int I, Jc;
-        gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
+        gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
+        I = I * MC + crank;
         if (!own.owned((int64_t)Jc * G_BN)) continue;
         for (int kc = 0; kc < nk; ++kc) {
           const int sg = kc / kpb, kin = (kc % kpb) * BK;
@@ -163,8 +174,12 @@ __global__ void __launch_bounds__(G_THREADS, 1)
           mbar_expect_tx(&full[st], G_STAGE);
           uint8_t* sa = smem + st * G_STAGE;
           tma_load_2d(sa, segs.amap[sg] ? &mapA1 : &mapA0, &full[st], segs.acol[sg] + kin, arow0 + I * G_BM);
-          tma_load_2d(sa + G_SA, segs.bmap[sg] ? &mapB1 : &mapB0, &full[st], segs.bcol[sg] + kin,
-                      brow0 + Jc * G_BN);
+          if (MC > 1)   // this CTA's half of the B tile, into both CTAs (half-height box maps)
+            tma_load_2d_mc(sa + G_SA + crank * (G_BN / MC) * G_ROWB, segs.bmap[sg] ? &mapB1 : &mapB0, &full[st],
+                           segs.bcol[sg] + kin, brow0 + Jc * G_BN + crank * (G_BN / MC), (uint16_t)((1u << MC) - 1));
+          else
+            tma_load_2d(sa + G_SA, segs.bmap[sg] ? &mapB1 : &mapB0, &full[st], segs.bcol[sg] + kin,
+                        brow0 + Jc * G_BN);
           if (++st == G_NS) { st = 0; ph ^= 1; }
         }
       }
@@ -177,10 +192,10 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       const uint32_t s0 = smem_u32(smem);
       // accumulation groups: fp16 one per tile; 3xTF32 every FLUSH k-chunks (drained by the epilogue)
       const int ch = TF ? Cfg::FLUSH : nk;
-      for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+      for (int t = u0; t < ntiles; t += ustride) {
         if (own.P > 1) {
           int I, Jc;
-          gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
+          gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
           if (!own.owned((int64_t)Jc * G_BN)) continue;
         }
         for (int kc = 0; kc < nk; ++kc) {
@@ -201,7 +216,8 @@ __global__ void __launch_bounds__(G_THREADS, 1)
               mma_f16(d, sdesc_sw128(sa + s * 32, 16, 1024), sdesc_sw128(sb + s * 32, 16, 1024), idesc,
                       (kc % ch > 0 || s > 0) ? 1u : 0u);
           }
-          mma_commit(&empty[st]);
+          if (MC > 1) mma_commit_mc(&empty[st], (uint16_t)((1u << MC) - 1));
+          else mma_commit(&empty[st]);
           if (++st == G_NS) { st = 0; ph ^= 1; }
           if (kc % ch == ch - 1 || kc == nk - 1) {
             mma_commit(&acc_full[ab]);
@@ -218,9 +234,10 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     const int ngroups = (nk + Cfg::FLUSH - 1) / Cfg::FLUSH;
     int ab = 0; uint32_t aph = 0;
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int t = u0; t < ntiles; t += ustride) {
       int I, Jc;
-      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
+      gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
+      I = I * MC + crank;
       if (!own.owned((int64_t)Jc * G_BN)) continue;
       float acc[64];
 #pragma unroll
@@ -271,9 +288,10 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     const int rit = q * 32 + lane;
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     int ab = 0; uint32_t aph = 0;
-    for (int t = blockIdx.x; t < ntiles; t += gridDim.x) {
+    for (int t = u0; t < ntiles; t += ustride) {
       int I, Jc;
-      gemm_tile<MODE, G_BN>(t, ntn, ntm, I, Jc, bandH);
+      gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
+      I = I * MC + crank;
       if (!own.owned((int64_t)Jc * G_BN)) continue;
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();
@@ -327,15 +345,16 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   }
   tc_fence_before();
   __syncthreads();
+  if (MC > 1) cluster_sync_all();   // the peer may still multicast into / commit to this CTA's smem
   if (warp == 2) {
     tc_fence_after();
     tmem_dealloc(tmem, 512);
   }
 }
 
-template <int MODE, bool TF>
+template <int MODE, bool TF, int MC = 1>
 static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
-  auto kern = gemm_tc_kernel<MODE, TF>;
+  auto kern = gemm_tc_kernel<MODE, TF, MC>;
   constexpr int BK = TF ? 32 : 64;
   constexpr int G_BN = GCfg<TF>::BN, G_SMEM = GCfg<TF>::SMEM;
   {
@@ -347,10 +366,11 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   // map width: the K columns (fp16) or the [hi | lo] columns (3xTF32: lo at lo_off)
   const uint64_t wid = TF ? (uint64_t)(p.lo_off + p.K) : (uint64_t)p.K;
   if ((e = make_tmap_2d(&mA0, p.A0, !TF, wid, p.a_rows, p.ld_a, BK, G_BM)) != cudaSuccess) return e;
-  if ((e = make_tmap_2d(&mB0, p.B0, !TF, wid, p.b_rows, p.ld_b, BK, G_BN)) != cudaSuccess) return e;
+  // MC = 2: each CTA of a pair loads half of the B tile (box of BN / 2 rows), multicast to both
+  if ((e = make_tmap_2d(&mB0, p.B0, !TF, wid, p.b_rows, p.ld_b, BK, G_BN / MC)) != cudaSuccess) return e;
   if (MODE == 0) {
     if ((e = make_tmap_2d(&mA1, p.A1, !TF, wid, p.a_rows, p.ld_a, BK, G_BM)) != cudaSuccess) return e;
-    if ((e = make_tmap_2d(&mB1, p.B1, !TF, wid, p.b_rows, p.ld_b, BK, G_BN)) != cudaSuccess) return e;
+    if ((e = make_tmap_2d(&mB1, p.B1, !TF, wid, p.b_rows, p.ld_b, BK, G_BN / MC)) != cudaSuccess) return e;
   } else {
     mA1 = mA0;
     mB1 = mB0;
@@ -372,17 +392,18 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
         sg.bcol[s] = q == 1 ? lo : 0;
       }
   }
-  const int ntm = (int)((p.Mrows + G_BM - 1) / G_BM);
+  constexpr int BMU = G_BM * MC;   // rows of one work unit (a tile, or a CTA pair's two tiles)
+  const int ntm = (int)((p.Mrows + BMU - 1) / BMU);
   const int ntn = (int)((p.Ncols + G_BN - 1) / G_BN);
-  int ntiles;
+  int ntiles;   // work units
   if (MODE == 0) {
     ntiles = 0;
-    for (int i = 0; i < ntm; ++i) ntiles += i * G_BM / G_BN + 1;
+    for (int i = 0; i < ntm; ++i) ntiles += i * BMU / G_BN + 1;
   } else {
     ntiles = ntm * ntn;
   }
   if (ntiles == 0) return cudaSuccess;
-  const int grid = std::min(ntiles, p.num_sms);
+  const int grid = std::min(ntiles * MC, p.num_sms / MC * MC);
   GemmOwn own;
   if (p.own_P > 1) {
     // every BN-wide output tile must lie inside one column block: an nb-aligned origin (nb % BN == 0),
@@ -394,13 +415,37 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
     own.org = p.own_org;
     own.nbo = p.nbo;
   }
-  return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
-                    (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
-                    TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off, own,
-                    knob(KNOB_SYR2K_BAND) > 0 ? knob(KNOB_SYR2K_BAND) : (G_BN == 256 ? 64 : 32));
+  // raster band height in units: the same ~16K (FP16) / 4K (3xTF32) rows of A per band
+  const int bandH = knob(KNOB_SYR2K_BAND) > 0 ? knob(KNOB_SYR2K_BAND) : (G_BN == 256 ? 64 : 32) / MC;
+  if (MC == 1)
+    return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
+                      (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
+                      TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off, own, bandH);
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(G_THREADS);
+  cfg.dynamicSmemBytes = G_SMEM;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = MC;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  at[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0, (int)p.brow0, p.Mrows, p.Ncols,
+                            ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
+                            TF ? (void*)p.Zs : (void*)p.Zh, p.ldz, p.zlo_off >= 0 ? p.zlo_off : p.lo_off, own,
+                            bandH);
 }
 
-cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, false>(p, st); }
+// FP16 SYR2K: CTA pairs with the B tile multicast (KNOB_SYR2K_MC = 1 selects the single-CTA kernel, ablation)
+cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) {
+  if (knob(KNOB_SYR2K_MC) == 1) return launch_gemm_t<0, false, 1>(p, st);
+  return launch_gemm_t<0, false, 2>(p, st);
+}
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, false>(p, st); }
 cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, true>(p, st); }
 cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, true>(p, st); }

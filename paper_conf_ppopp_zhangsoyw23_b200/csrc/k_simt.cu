@@ -142,7 +142,7 @@ cudaError_t gemm_tn(int64_t rows, int m1, int n2, float alpha, const float* A, i
   chunk = std::max<int64_t>(chunk, 256);
   chunk = (chunk + TN_KC - 1) / TN_KC * TN_KC;
   const int gz = (int)((rows + chunk - 1) / chunk);
-  return launch_pdl(gemm_tn_kernel, dim3(gx, gy, gz), dim3(256), 0, st, rows, chunk, m1, n2, alpha, A, lda, B, ldb, C,
+  return launch_plain(gemm_tn_kernel, dim3(gx, gy, gz), dim3(256), 0, st, rows, chunk, m1, n2, alpha, A, lda, B, ldb, C,
                     ldc);
 }
 
@@ -322,7 +322,7 @@ cudaError_t gemm_nn(int64_t M, int N, int K, float alpha, const float* A, int64_
     if (N <= 32)
       return launch_pdl(skinny_upd_kernel<1>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
                         transB, D, ldd, K, (const float*)nullptr, (int64_t)0, (const float*)nullptr, (int64_t)0, false);
-    return launch_pdl(skinny_upd_kernel<2>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
+    return launch_plain(skinny_upd_kernel<2>, dim3(gx, ks), dim3(256), 0, st, M, N, K, kper, alpha, A, lda, B, ldb,
                       transB, D, ldd, K, (const float*)nullptr, (int64_t)0, (const float*)nullptr, (int64_t)0, false);
   }
   dim3 grid((unsigned)((M + NN_T - 1) / NN_T), (N + NN_T - 1) / NN_T);
@@ -337,7 +337,7 @@ cudaError_t skinny_upd2(int64_t M, int N, int K0, const float* A0, int64_t lda0,
   const int K = K0 + K1;
   if (M <= 0 || N <= 0 || K <= 0) return cudaSuccess;
   const int gx = (int)((M + 127) / 128);
-  const int per = N <= 32 ? 8 : 2;   // as gemm_nn's in-place branch
+  const int per = 8;   // the two-segment lazy update: K = 2k, ~8 CTAs per SM helped at b = 32 and 64
   int ks = std::max(1, std::min((K + 63) / 64, (per * 148 + gx - 1) / gx));
   const int kper = ((K + ks - 1) / ks + 31) / 32 * 32;
   ks = (K + kper - 1) / kper;

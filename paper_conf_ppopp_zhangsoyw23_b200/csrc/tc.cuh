@@ -71,6 +71,25 @@ SBR_DEV void tma_load_2d_hint(void* dst, const CUtensorMap* map, uint64_t* bar, 
       : "memory");
 }
 
+// Multicast 2-D tile load: the box lands at the same shared-memory offset in every CTA of ctaMask
+// (this cluster), and completes its bytes on the barrier at the same offset in each of them.
+SBR_DEV void tma_load_2d_mc(void* dst, const CUtensorMap* map, uint64_t* bar, int c_inner, int c_outer,
+                            uint16_t mask) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+      " [%0], [%1, {%3, %4}], [%2], %5;" ::"r"(smem_u32(dst)),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(smem_u32(bar)), "r"(c_inner), "r"(c_outer), "h"(mask)
+      : "memory");
+}
+SBR_DEV uint32_t cluster_ctarank() {
+  uint32_t r;
+  asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+  return r;
+}
+SBR_DEV void cluster_sync_all() {
+  asm volatile("barrier.cluster.arrive.aligned;\nbarrier.cluster.wait.aligned;" ::: "memory");
+}
+
 // ------------------------------------------------------------------ tcgen05
 SBR_DEV void tmem_alloc(uint32_t* dst_smem, uint32_t ncols) {  // whole warp
   asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(dst_smem)),
@@ -120,6 +139,12 @@ SBR_DEV void mma_tf32_ts(uint32_t d_tmem, uint32_t a_tmem, uint64_t bdesc, uint3
 // Arrive on bar when all previously issued tcgen05 async ops of this thread complete.
 SBR_DEV void mma_commit(uint64_t* bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(smem_u32(bar))
+               : "memory");
+}
+// Same, arriving on the barrier at bar's offset in every CTA of ctaMask (this cluster).
+SBR_DEV void mma_commit_mc(uint64_t* bar, uint16_t mask) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;"
+               ::"r"(smem_u32(bar)), "h"(mask)
                : "memory");
 }
 
