@@ -51,8 +51,8 @@ def test_parity_vs_oracle(n, b, nb, mode):
     if mode == "3xtf32":
         assert ee <= 1e-5
         assert db <= 2e-4
-    else:
-        assert ee <= 1e-2
+    else:   # FP16: observed <= 2.1e-4 (n = 256 .. 1500); the paper's Table 4 reports ~1e-4
+        assert ee <= 1e-3
 
 
 def test_generator_bit_identical():
