@@ -105,22 +105,36 @@ def test_trivial_and_error_cases():
     assert ei.value.status == -5
 
 
-def test_reduce_host_matches_device():
+@pytest.mark.parametrize("mode", ["fp16", "3xtf32"])
+def test_reduce_host_matches_device(mode):
+    """sbr_reduce_host (host buffers, copies inside) against sbr_reduce (device buffers) and against
+    the oracle.  The fp32 / fp64 reductions of the kernels (atomics) sum in a run-dependent order and
+    SBR is backward- not forward-stable, so the two runs' bands are compared entry-wise AFTER the sign
+    normalisation of reading C1 to the ORACLE's band B (unique given dlarfg's signs), each within the
+    mode's forward tolerance, plus their spectra against each other."""
     import torch
 
     import paper_conf_ppopp_zhangsoyw23_b200 as sbr
 
     n, b, nb = 512, 16, 64
     a_host = workloads.random_symmetric(n, 77)
+    b_ref, lam_ref = _oracle(a_host, b)
+    norm2 = float(np.max(np.abs(lam_ref)))
     h = sbr.Handle(0)
     a_dev = torch.from_numpy(a_host).cuda()
-    ab_dev, _ = h.reduce(a_dev, b, nb, mode="fp16")
+    ab_dev, _ = h.reduce(a_dev, b, nb, mode=mode)
     pinned = torch.from_numpy(a_host.copy()).pin_memory()
-    ab_host, _ = h.reduce_host(pinned, b, nb, mode="fp16")
+    ab_host, _ = h.reduce_host(pinned, b, nb, mode=mode)
     torch.cuda.synchronize()
-    # Same kernels, but fp32 reductions (atomics) sum in a different order, and SBR is
-    # backward- not forward-stable: compare the spectra of the two bands, not entries.
-    lam_h = np.linalg.eigvalsh(sbr.band_to_dense(ab_host.double()).numpy())
-    lam_d = np.linalg.eigvalsh(sbr.band_to_dense(ab_dev.double().cpu()).numpy())
-    assert np.max(np.abs(lam_h - lam_d)) <= 1e-3 * np.max(np.abs(lam_d))
+    bd = sbr.band_to_dense(ab_dev.double().cpu()).numpy()
+    bh = sbr.band_to_dense(ab_host.double()).numpy()
+    ref = sign_normalise(b_ref, b)
+    dd = float(np.max(np.abs(sign_normalise(bd, b) - ref))) / norm2
+    dh = float(np.max(np.abs(sign_normalise(bh, b) - ref))) / norm2
+    tol = 1e-4 if mode == "3xtf32" else 3e-2   # observed 9e-6 / 8.5e-3
+    print(f"host vs device {mode}: |B_dev - B_oracle| {dd:.1e}  |B_host - B_oracle| {dh:.1e}")
+    assert dd <= tol and dh <= tol
+    lam_h = np.linalg.eigvalsh(bh)
+    lam_d = np.linalg.eigvalsh(bd)
+    assert np.max(np.abs(lam_h - lam_d)) <= (1e-5 if mode == "3xtf32" else 1e-3) * norm2
     assert np.all(np.isfinite(ab_host.numpy()))
