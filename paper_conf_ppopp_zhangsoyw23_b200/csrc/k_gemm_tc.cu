@@ -143,8 +143,13 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     mbar_fence_init();
   }
   const int crank = MC > 1 ? (int)cluster_ctarank() : 0;
-  // work units: one tile (MC = 1) or a pair of vertically adjacent tiles (MC = 2), unit u covers
-  // tile rows MC u .. MC u + MC - 1; this CTA takes row I = MC Iu + crank
+  // work units: one tile (MC = 1) or a pair of tiles.  FP16 (128 x 256 tiles): the pair is two
+  // vertically adjacent tiles sharing B (this CTA takes row I = MC Iu + crank).  3xTF32 (128 x 128
+  // tiles): two horizontally adjacent tiles sharing A (column Jc = MC Jcu + crank), i.e. the unit is
+  // the FP16 mode's 128 x 256 footprint.
+  constexpr bool SHA = TF;
+  constexpr int UBM = (MC > 1 && !SHA) ? G_BM * MC : G_BM;
+  constexpr int UBN = (MC > 1 && SHA) ? G_BN * MC : G_BN;
   const int u0 = MC > 1 ? (int)blockIdx.x / MC : (int)blockIdx.x;
   const int ustride = MC > 1 ? (int)gridDim.x / MC : (int)gridDim.x;
   if (warp == 0 && lane == 0) {
@@ -158,23 +163,27 @@ __global__ void __launch_bounds__(G_THREADS, 1)
   const uint32_t tmem = *tmem_slot;
   pdl_wait();
   const int nk = segs.n * kpb;
-  const int ntm = (int)((Mrows + G_BM * MC - 1) / (G_BM * MC));   // unit rows
+  const int ntm = (int)((Mrows + UBM - 1) / UBM);   // unit rows
 
   if (warp == 0) {
     if (lane == 0) {  // ---------------- TMA producer
       int st = 0; uint32_t ph = 0;
       for (int t = u0; t < ntiles; t += ustride) {
         int I, Jc;
-        gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
-        I = I * MC + crank;
-        if (!own.owned((int64_t)Jc * G_BN)) continue;
+        gemm_tile<MODE, UBN, UBM>(t, ntn, ntm, I, Jc, bandH);
+        if (MC > 1) { if (SHA) Jc = Jc * MC + crank; else I = I * MC + crank; }
+        if (!own.owned((int64_t)(Jc - (SHA && MC > 1 ? crank : 0)) * G_BN)) continue;   // per UNIT: both CTAs agree
         for (int kc = 0; kc < nk; ++kc) {
           const int sg = kc / kpb, kin = (kc % kpb) * BK;
           mbar_wait(&empty[st], ph ^ 1);
           mbar_expect_tx(&full[st], G_STAGE);
           uint8_t* sa = smem + st * G_STAGE;
-          tma_load_2d(sa, segs.amap[sg] ? &mapA1 : &mapA0, &full[st], segs.acol[sg] + kin, arow0 + I * G_BM);
-          if (MC > 1)   // this CTA's half of the B tile, into both CTAs (half-height box maps)
+          if (MC > 1 && SHA)   // this CTA's half of the shared A tile, into both CTAs (half-height box maps)
+            tma_load_2d_mc(sa + crank * (G_BM / MC) * G_ROWB, segs.amap[sg] ? &mapA1 : &mapA0, &full[st],
+                           segs.acol[sg] + kin, arow0 + I * G_BM + crank * (G_BM / MC), (uint16_t)((1u << MC) - 1));
+          else
+            tma_load_2d(sa, segs.amap[sg] ? &mapA1 : &mapA0, &full[st], segs.acol[sg] + kin, arow0 + I * G_BM);
+          if (MC > 1 && !SHA)   // this CTA's half of the B tile, into both CTAs (half-height box maps)
             tma_load_2d_mc(sa + G_SA + crank * (G_BN / MC) * G_ROWB, segs.bmap[sg] ? &mapB1 : &mapB0, &full[st],
                            segs.bcol[sg] + kin, brow0 + Jc * G_BN + crank * (G_BN / MC), (uint16_t)((1u << MC) - 1));
           else
@@ -195,8 +204,9 @@ __global__ void __launch_bounds__(G_THREADS, 1)
       for (int t = u0; t < ntiles; t += ustride) {
         if (own.P > 1) {
           int I, Jc;
-          gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
-          if (!own.owned((int64_t)Jc * G_BN)) continue;
+          gemm_tile<MODE, UBN, UBM>(t, ntn, ntm, I, Jc, bandH);
+          if (MC > 1) { if (SHA) Jc = Jc * MC + crank; else I = I * MC + crank; }
+          if (!own.owned((int64_t)(Jc - (SHA && MC > 1 ? crank : 0)) * G_BN)) continue;   // per UNIT: both CTAs agree
         }
         for (int kc = 0; kc < nk; ++kc) {
           if (kc % ch == 0) {
@@ -236,9 +246,9 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = u0; t < ntiles; t += ustride) {
       int I, Jc;
-      gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
-      I = I * MC + crank;
-      if (!own.owned((int64_t)Jc * G_BN)) continue;
+      gemm_tile<MODE, UBN, UBM>(t, ntn, ntm, I, Jc, bandH);
+      if (MC > 1) { if (SHA) Jc = Jc * MC + crank; else I = I * MC + crank; }
+      if (!own.owned((int64_t)(Jc - (SHA && MC > 1 ? crank : 0)) * G_BN)) continue;   // per UNIT: both CTAs agree
       float acc[64];
 #pragma unroll
       for (int c = 0; c < 64; ++c) acc[c] = 0.f;
@@ -290,9 +300,9 @@ __global__ void __launch_bounds__(G_THREADS, 1)
     int ab = 0; uint32_t aph = 0;
     for (int t = u0; t < ntiles; t += ustride) {
       int I, Jc;
-      gemm_tile<MODE, G_BN, G_BM * MC>(t, ntn, ntm, I, Jc, bandH);
-      I = I * MC + crank;
-      if (!own.owned((int64_t)Jc * G_BN)) continue;
+      gemm_tile<MODE, UBN, UBM>(t, ntn, ntm, I, Jc, bandH);
+      if (MC > 1) { if (SHA) Jc = Jc * MC + crank; else I = I * MC + crank; }
+      if (!own.owned((int64_t)(Jc - (SHA && MC > 1 ? crank : 0)) * G_BN)) continue;   // per UNIT: both CTAs agree
       mbar_wait(&acc_full[ab], aph);
       tc_fence_after();
       const int64_t row = (int64_t)I * G_BM + rit;
@@ -365,12 +375,13 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
   cudaError_t e;
   // map width: the K columns (fp16) or the [hi | lo] columns (3xTF32: lo at lo_off)
   const uint64_t wid = TF ? (uint64_t)(p.lo_off + p.K) : (uint64_t)p.K;
-  if ((e = make_tmap_2d(&mA0, p.A0, !TF, wid, p.a_rows, p.ld_a, BK, G_BM)) != cudaSuccess) return e;
-  // MC = 2: each CTA of a pair loads half of the B tile (box of BN / 2 rows), multicast to both
-  if ((e = make_tmap_2d(&mB0, p.B0, !TF, wid, p.b_rows, p.ld_b, BK, G_BN / MC)) != cudaSuccess) return e;
+  // MC = 2: each CTA of a pair loads half of the shared tile (B in FP16, A in 3xTF32), multicast to both
+  constexpr int ABOX = (MC > 1 && TF) ? G_BM / MC : G_BM, BBOX = (MC > 1 && !TF) ? G_BN / MC : G_BN;
+  if ((e = make_tmap_2d(&mA0, p.A0, !TF, wid, p.a_rows, p.ld_a, BK, ABOX)) != cudaSuccess) return e;
+  if ((e = make_tmap_2d(&mB0, p.B0, !TF, wid, p.b_rows, p.ld_b, BK, BBOX)) != cudaSuccess) return e;
   if (MODE == 0) {
-    if ((e = make_tmap_2d(&mA1, p.A1, !TF, wid, p.a_rows, p.ld_a, BK, G_BM)) != cudaSuccess) return e;
-    if ((e = make_tmap_2d(&mB1, p.B1, !TF, wid, p.b_rows, p.ld_b, BK, G_BN / MC)) != cudaSuccess) return e;
+    if ((e = make_tmap_2d(&mA1, p.A1, !TF, wid, p.a_rows, p.ld_a, BK, ABOX)) != cudaSuccess) return e;
+    if ((e = make_tmap_2d(&mB1, p.B1, !TF, wid, p.b_rows, p.ld_b, BK, BBOX)) != cudaSuccess) return e;
   } else {
     mA1 = mA0;
     mB1 = mB0;
@@ -392,13 +403,14 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
         sg.bcol[s] = q == 1 ? lo : 0;
       }
   }
-  constexpr int BMU = G_BM * MC;   // rows of one work unit (a tile, or a CTA pair's two tiles)
+  constexpr int BMU = (MC > 1 && !TF) ? G_BM * MC : G_BM;   // one work unit: a tile or a CTA pair's two
+  constexpr int BNU = (MC > 1 && TF) ? G_BN * MC : G_BN;
   const int ntm = (int)((p.Mrows + BMU - 1) / BMU);
-  const int ntn = (int)((p.Ncols + G_BN - 1) / G_BN);
+  const int ntn = (int)((p.Ncols + BNU - 1) / BNU);
   int ntiles;   // work units
   if (MODE == 0) {
     ntiles = 0;
-    for (int i = 0; i < ntm; ++i) ntiles += i * BMU / G_BN + 1;
+    for (int i = 0; i < ntm; ++i) ntiles += i * BMU / BNU + 1;
   } else {
     ntiles = ntm * ntn;
   }
@@ -409,14 +421,14 @@ static cudaError_t launch_gemm_t(const GemmTcLaunch& p, cudaStream_t st) {
     // every BN-wide output tile must lie inside one column block: an nb-aligned origin (nb % BN == 0),
     // or a region that fits in one block (the ragged last block)
     const bool one_block = p.own_org / p.nbo == (p.own_org + p.Ncols - 1) / p.nbo;
-    if (MODE != 0 || p.nbo % G_BN != 0 || (p.own_org % p.nbo != 0 && !one_block)) return cudaErrorInvalidValue;
+    if (MODE != 0 || p.nbo % BNU != 0 || (p.own_org % p.nbo != 0 && !one_block)) return cudaErrorInvalidValue;
     own.P = p.own_P;
     own.rank = p.own_rank;
     own.org = p.own_org;
     own.nbo = p.nbo;
   }
   // raster band height in units: the same ~16K (FP16) / 4K (3xTF32) rows of A per band
-  const int bandH = knob(KNOB_SYR2K_BAND) > 0 ? knob(KNOB_SYR2K_BAND) : (G_BN == 256 ? 64 : 32) / MC;
+  const int bandH = knob(KNOB_SYR2K_BAND) > 0 ? knob(KNOB_SYR2K_BAND) : (TF ? 32 : 64 / MC);
   if (MC == 1)
     return launch_pdl(kern, dim3(grid), dim3(G_THREADS), G_SMEM, st, mA0, mA1, mB0, mB1, kpb, sg, (int)p.arow0,
                       (int)p.brow0, p.Mrows, p.Ncols, ntn, ntiles, p.C, p.ldc, p.shadow, p.ld_shadow, p.X, p.ldx,
@@ -447,7 +459,11 @@ cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) {
   return launch_gemm_t<0, false, 2>(p, st);
 }
 cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, false>(p, st); }
-cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<0, true>(p, st); }
+// 3xTF32 SYR2K: CTA pairs sharing the A tile (KNOB_SYR2K_MC = 1: single CTAs, ablation)
+cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) {
+  if (knob(KNOB_SYR2K_MC) == 1) return launch_gemm_t<0, true, 1>(p, st);
+  return launch_gemm_t<0, true, 2>(p, st);
+}
 cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, true>(p, st); }
 cudaError_t launch_gemm_split_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<2, true>(p, st); }
 cudaError_t launch_gemm_sub_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<3, true>(p, st); }
