@@ -519,7 +519,7 @@ def main():
             "value": value,
             "unit": "TFLOP/s",
             "n_gpus": world,
-            "scaling": "strong" if world > 1 else "weak",
+            "scaling": "strong",   # one matrix at any N (N = 1 included: the SCALE run divides the same work)
             "steps": args.steps,
             "warmup": args.warmup,
             "ms_per_step": ms_per_step,
