@@ -458,13 +458,19 @@ cudaError_t launch_syr2k_tc(const GemmTcLaunch& p, cudaStream_t st) {
   if (knob(KNOB_SYR2K_MC) == 1) return launch_gemm_t<0, false, 1>(p, st);
   return launch_gemm_t<0, false, 2>(p, st);
 }
-cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, false>(p, st); }
+cudaError_t launch_zform_tc(const GemmTcLaunch& p, cudaStream_t st) {   // CTA pairs sharing B (W^T X)
+  if (knob(KNOB_SYR2K_MC) == 1) return launch_gemm_t<1, false, 1>(p, st);
+  return launch_gemm_t<1, false, 2>(p, st);
+}
 // 3xTF32 SYR2K: CTA pairs sharing the A tile (KNOB_SYR2K_MC = 1: single CTAs, ablation)
 cudaError_t launch_syr2k_tf32(const GemmTcLaunch& p, cudaStream_t st) {
   if (knob(KNOB_SYR2K_MC) == 1) return launch_gemm_t<0, true, 1>(p, st);
   return launch_gemm_t<0, true, 2>(p, st);
 }
-cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<1, true>(p, st); }
+cudaError_t launch_zform_tf32(const GemmTcLaunch& p, cudaStream_t st) {   // CTA pairs sharing A (Y)
+  if (knob(KNOB_SYR2K_MC) == 1) return launch_gemm_t<1, true, 1>(p, st);
+  return launch_gemm_t<1, true, 2>(p, st);
+}
 cudaError_t launch_gemm_split_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<2, true>(p, st); }
 cudaError_t launch_gemm_sub_tf32(const GemmTcLaunch& p, cudaStream_t st) { return launch_gemm_t<3, true>(p, st); }
 
