@@ -452,12 +452,12 @@ static cudaError_t launch_pass_t(const PassLaunch& p, cudaStream_t st) {
                     p.X, p.ldx, exper, p.off, own, p.nbo);
 }
 
-static int pass_variant() {   // SBR_PASS_CFG (tuning experiments only): 0 = C8/NS4, 1 = C4/NS5, 2 = C2/NS6
+static int pass_variant() {   // SBR_PASS_CFG (tuning experiments only): 0 = C8/NS4, 1 = C4/NS5, 2 = C2/NS6, 3 = C12/NS3
   static int v = -1;
   if (v < 0) {
     const char* e = getenv("SBR_PASS_CFG");
     v = e ? atoi(e) : 0;
-    if (v < 0 || v > 2) v = 0;
+    if (v < 0 || v > 3) v = 0;
   }
   return v;
 }
@@ -468,6 +468,8 @@ cudaError_t launch_pass_tc(const PassLaunch& p, cudaStream_t st) {
     switch (pass_variant()) {
       case 1: return launch_pass_t<32, 4, 5>(p, st);
       case 2: return launch_pass_t<32, 2, 6>(p, st);
+      case 3: if (p.own_P <= 1) return launch_pass_t<32, 12, 3>(p, st);   // (dist: groups must tile nb)
+              return launch_pass_t<32, 8, 4>(p, st);
       default: return launch_pass_t<32, 8, 4>(p, st);
     }
   }
